@@ -37,6 +37,7 @@ def lib() -> ctypes.CDLL:
         L.orc_unpack.argtypes = [vp, vp, i64]
         L.orc_jacobi_sweep.argtypes = [vp, vp, i64, i32, vp, i32]
         L.orc_jacobi_run.argtypes = [vp, vp, i64, i32, i32]
+        L.orc_jacobi_sweep_rect.argtypes = [vp, vp, i64, i64, i32]
         L.orc_sparse_rows.argtypes = [vp, vp, i64, i64, i32, vp]
         L.orc_gemm_rows_f64.argtypes = [vp, vp, i64, i64, i64, vp, i64, vp, i32]
         L.orc_kmeans_assign.argtypes = [vp, i64, i32, i32, vp, vp, i32]
@@ -110,6 +111,11 @@ def jacobi_sweep(src: np.ndarray, dst: np.ndarray, P: int = 1, track: bool = Fal
     bms = np.zeros((P, nwords(N * N)), dtype=np.uint32) if track else None
     lib().orc_jacobi_sweep(src.ctypes.data, dst.ctypes.data, N, P, _p(bms), nthreads)
     return bms
+
+
+def jacobi_sweep_rect(src: np.ndarray, dst: np.ndarray, nthreads: int = 0) -> None:
+    rows, cols = src.shape
+    lib().orc_jacobi_sweep_rect(src.ctypes.data, dst.ctypes.data, rows, cols, nthreads)
 
 
 def jacobi_run(A: np.ndarray, B: np.ndarray, S: int, nthreads: int = 1) -> None:

@@ -118,7 +118,8 @@ class Model:
                     out["interpartition"] += (P - 1) * (16 + 16 * runs + elems * rg.esize)
                     nchunks = len(np.unique(np.nonzero(wm)[0] // ch)) if elems else 0
                     out["paper_protocol"] += (P - 1) * nchunks * (ch * rg.esize + ch // 8)
-                    rg.host_valid[wm] = False
+                # the host copy is treated as stale as a whole: the dirty sets live on the devices
+                rg.host_valid[:] = False
         for k, v in out.items():
             self.stats[k] += v
         self.stats["loops"] += 1

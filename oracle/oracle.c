@@ -140,6 +140,19 @@ void orc_jacobi_sweep(const float* src, float* dst, int64_t N, int P, uint32_t* 
     }
 }
 
+/* The same sweep on a rows x cols array (rows [1, rows-1), columns [1, cols-1)); used to time
+ * the oracle on full-width bands of the C2 field (bench.py cpu_baseline). */
+void orc_jacobi_sweep_rect(const float* src, float* dst, int64_t rows, int64_t cols, int nthreads) {
+    #pragma omp parallel for schedule(static) num_threads(nthr(nthreads))
+    for (int64_t i = 1; i < rows - 1; ++i) {
+        for (int64_t j = 1; j < cols - 1; ++j) {
+            float ns = src[(i - 1) * cols + j] + src[(i + 1) * cols + j];
+            float we = src[i * cols + j - 1] + src[i * cols + j + 1];
+            dst[i * cols + j] = 0.25f * (ns + we);
+        }
+    }
+}
+
 /* S sweeps alternating A -> B -> A ...: sweep s reads A if s is even (else B) and writes the
  * other. Result in A for even S (reading W1). B must hold a copy of A on entry. */
 void orc_jacobi_run(float* A, float* B, int64_t N, int S, int nthreads) {

@@ -1,0 +1,84 @@
+// Internal launch interface of the sm_100a kernels (no torch types; plain pointers and sizes).
+// Every launcher enqueues on `s`, adds the number of kernels it launched to *launches, and
+// returns the launch error (cudaSuccess if all launches were accepted).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime_api.h>
+
+namespace accmg {
+namespace k {
+
+// Two-level dirty bits of one replica (L133-135): l1 = 1 bit per element (bit b of word w is
+// element 32w+b), l2 = 1 bit per chunk of 2^l2_shift elements. l1 == nullptr: no tracking.
+struct Track {
+    uint32_t* l1;
+    uint32_t* l2;
+    int l2_shift;
+};
+
+// Up to 64 device pointers passed by value in the kernel parameter block (no staging copy).
+constexpr int kMaxPtrs = 64;
+struct PtrList {
+    void* p[kMaxPtrs];
+    int n;
+};
+
+// ---- loop bodies -----------------------------------------------------------------------------
+// 5-point Jacobi on rows [r0, r1) x cols [c0, c1) of a rows x cols fp32 array (global indices).
+// impl: 0 = auto, 1 = register sliding window (LDG.128), 2 = TMA-staged shared-memory tiles.
+cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
+                     int64_t c0, int64_t c1, Track t, int impl, cudaStream_t s, int64_t* launches);
+
+// Test body: rows i in [r0, r1) with i % period == 0: out[i][:] = in[i][:] + 1.0f.
+cudaError_t sparse_rows(const float* in, float* out, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
+                        int64_t period, Track t, cudaStream_t s, int64_t* launches);
+
+// k-means assignment + reductiontoarray over points [p0, p1): member[p] = argmin_c (fmaf chain),
+// sums[member][j] += x*2^shift (int64), counts[member] += 1 into the partition's partials.
+// err_flag (device int) is set to 1 if some x is not on the 2^-shift grid.
+cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int64_t* sums, int64_t* counts,
+                          int64_t p0, int64_t p1, int d, int kc, int shift, int* err_flag, cudaStream_t s,
+                          int64_t* launches);
+// k-means update over clusters [c0, c1); tracked writes of centroids, sums, counts.
+cudaError_t kmeans_update(int64_t* sums, int64_t* counts, float* cen, int64_t c0, int64_t c1, int d, int shift,
+                          Track t_sums, Track t_counts, Track t_cen, cudaStream_t s, int64_t* launches);
+
+// bf16 x bf16 -> fp32 GEMM of rows [m0, m1) of C = A.B (A [M][K], B [K][N], C [M][N], row-major),
+// tcgen05.mma with TMEM accumulators and TMA operand staging.
+cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M, int64_t N, int64_t K,
+                      int64_t m0, int64_t m1, cudaStream_t s, int64_t* launches);
+
+// ---- coherence: compaction of dirty runs, scatter into peer replicas -------------------------
+constexpr int kTileWords = 2048;   // bitmap words per compaction tile (65536 elements)
+
+// Pass 1: per-tile counts {run starts, run ends, elements} of tiles holding a dirty chunk
+// (chunks with a clear L2 bit are skipped without reading L1); also records each tile's first
+// and last word (neighbours for pass 3, which clears L1 as it goes).
+cudaError_t compact_count(const uint32_t* l1, const uint32_t* l2, int64_t nwords, int chunk_words_log2,
+                          int64_t ntiles, int64_t* tile_counts, uint32_t* tile_edges, cudaStream_t s,
+                          int64_t* launches);
+// Pass 2 (one block): exclusive scan of the tile counts; totals[0..3] = {n_runs, n_elems,
+// dirty_chunks, n_run_ends}; clears the L2 bits. (The packed header is totals[0..1].)
+cudaError_t compact_scan(const int64_t* tile_counts, int64_t ntiles, int64_t* tile_offs, int64_t* totals,
+                         uint32_t* l2, int64_t nl2words, cudaStream_t s, int64_t* launches);
+// Pass 3: run starts/ends and payload into the canonical packed buffer; clears L1 words.
+cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t ntiles, const int64_t* tile_counts,
+                          const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
+                          int esize, uint8_t* packed, int64_t n_runs, cudaStream_t s, int64_t* launches);
+// Scatter the runs of a canonical packed buffer into ndst replicas at the same global indices.
+// scratch: >= 2 * kScatterBlocks int64.
+constexpr int kScatterBlocks = 592;  // 4 x 148 SMs
+cudaError_t scatter_packed(const uint8_t* packed, int64_t n_runs, const PtrList& dsts, int esize,
+                           int64_t* scratch, cudaStream_t s, int64_t* launches);
+
+// ---- reductions (reductiontoarray merge, L112) -------------------------------------------------
+// acc[i] += srcs.p[j][i] for every j, then dsts.p[j][i] += acc[i] for every j (int64 elements).
+cudaError_t reduce_sum_i64(int64_t* acc, const PtrList& srcs, int64_t n, cudaStream_t s, int64_t* launches);
+cudaError_t apply_add_i64(const PtrList& dsts, const int64_t* acc, int64_t n, cudaStream_t s, int64_t* launches);
+
+// Device-side bitwise AND test of two bitmaps (debug_checks): *flag |= any(a & b).
+cudaError_t bitmap_overlap(const uint32_t* a, const uint32_t* b, int64_t nwords, int* flag, cudaStream_t s,
+                           int64_t* launches);
+
+}  // namespace k
+}  // namespace accmg

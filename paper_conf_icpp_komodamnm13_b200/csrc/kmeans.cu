@@ -1,0 +1,259 @@
+// Loop bodies of the k-means workload (config C4; KMEANS is the paper's Rodinia application,
+// Table II, with 2 parallel loops and a reductiontoarray, L75-77/L89-91/L112).
+//
+// Assignment loop over points p (this partition's chunk):
+//   best = 0, bestd = +inf; for c: acc = 0; for j: diff = x[p][j] - cen[c][j]; acc = fmaf(diff, diff, acc);
+//   if (acc < bestd) {bestd = acc; best = c}      (ties -> lowest c; reading in DESIGN.md)
+//   member[p] = best;  sums[best][j] += x[p][j] (exact: int64 fixed point x*2^shift);  counts[best] += 1
+// Hierarchical reduction (L112): shared-memory accumulators per block, then one global atomic per
+// non-zero entry into the partition's partial, then (runtime) across partitions / GPUs.
+//
+// FP32-pipe bound (2*k*d flops per point, no tensor-core form preserves the exact fmaf order that
+// the bit-exact argmin needs). Two points share each packed __fadd2_rn / __ffma2_rn
+// (Blackwell FADD2/FFMA2: two fp32 lanes per instruction, each rounded exactly like the scalar op),
+// so the per-distance operation order is the scalar one; each thread owns 4 points; centroids
+// are staged in shared memory pre-negated and duplicated as float2 (-c, -c) so one LDS.128 feeds
+// two dims of two packed operations.
+#include <cuda_fp16.h>
+
+#include "kernels.h"
+#include "track.cuh"
+
+namespace accmg {
+namespace k {
+namespace {
+
+constexpr int kThreads = 256;
+constexpr int kPPT = 4;  // points per thread (2 packed pairs)
+
+__device__ __forceinline__ int64_t fixed_of(float x, float scale, int* err) {
+    const float v = x * scale;  // exact: power-of-two scaling
+    if (!(v == rintf(v) && fabsf(v) < 2147483648.0f)) atomicOr(err, 1);
+    return (int64_t)v;
+}
+
+// Block-level accumulation into shared memory, then flush to the partition's partial (global).
+__device__ __forceinline__ void flush_block(unsigned long long* s_sum, unsigned long long* s_cnt, int64_t* sums,
+                                            int64_t* counts, int kc, int d) {
+    __syncthreads();
+    for (int i = threadIdx.x; i < kc * d; i += blockDim.x)
+        if (s_sum[i]) atomicAdd(reinterpret_cast<unsigned long long*>(sums) + i, s_sum[i]);
+    for (int i = threadIdx.x; i < kc; i += blockDim.x)
+        if (s_cnt[i]) atomicAdd(reinterpret_cast<unsigned long long*>(counts) + i, s_cnt[i]);
+}
+
+template <int D>
+__global__ void __launch_bounds__(kThreads)
+assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __restrict__ member,
+         int64_t* __restrict__ sums, int64_t* __restrict__ counts, int64_t p0, int64_t p1, int kc, int shift,
+         int* err) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    float2* s_nc = reinterpret_cast<float2*>(smem);                                  // kc*D  (-c,-c)
+    unsigned long long* s_sum = reinterpret_cast<unsigned long long*>(s_nc + kc * D);  // kc*D
+    unsigned long long* s_cnt = s_sum + kc * D;                                      // kc
+    for (int i = threadIdx.x; i < kc * D; i += kThreads) {
+        const float c = -cen[i];
+        s_nc[i] = make_float2(c, c);
+        s_sum[i] = 0ull;
+    }
+    for (int i = threadIdx.x; i < kc; i += kThreads) s_cnt[i] = 0ull;
+    __syncthreads();
+    const float scale = (float)(1 << shift);
+    const int64_t n = p1 - p0;
+    const int64_t ngroups = (n + kPPT - 1) / kPPT;
+    for (int64_t grp = (int64_t)blockIdx.x * kThreads + threadIdx.x; grp < ngroups;
+         grp += (int64_t)gridDim.x * kThreads) {
+        const int64_t pb = p0 + grp * kPPT;
+        float2 xa[D], xb[D];  // (point0, point1), (point2, point3)
+        bool ok[kPPT];
+#pragma unroll
+        for (int q = 0; q < kPPT; ++q) ok[q] = pb + q < p1;
+#pragma unroll
+        for (int j = 0; j < D; j += 4) {
+            float4 v[kPPT];
+#pragma unroll
+            for (int q = 0; q < kPPT; ++q)
+                v[q] = ok[q] ? __ldg(reinterpret_cast<const float4*>(x + (pb + q) * D + j)) : make_float4(0.f, 0.f, 0.f, 0.f);
+            xa[j] = make_float2(v[0].x, v[1].x); xb[j] = make_float2(v[2].x, v[3].x);
+            xa[j + 1] = make_float2(v[0].y, v[1].y); xb[j + 1] = make_float2(v[2].y, v[3].y);
+            xa[j + 2] = make_float2(v[0].z, v[1].z); xb[j + 2] = make_float2(v[2].z, v[3].z);
+            xa[j + 3] = make_float2(v[0].w, v[1].w); xb[j + 3] = make_float2(v[2].w, v[3].w);
+        }
+        float bd[kPPT];
+        int bi[kPPT];
+#pragma unroll
+        for (int q = 0; q < kPPT; ++q) { bd[q] = __int_as_float(0x7f800000); bi[q] = 0; }
+#pragma unroll 2
+        for (int c = 0; c < kc; ++c) {
+            float2 aa = make_float2(0.f, 0.f), ab = make_float2(0.f, 0.f);
+            const float4* nc4 = reinterpret_cast<const float4*>(s_nc + c * D);
+#pragma unroll
+            for (int j = 0; j < D; j += 2) {
+                const float4 nc = nc4[j / 2];  // (-c_j, -c_j, -c_{j+1}, -c_{j+1})
+                const float2 n0 = make_float2(nc.x, nc.y), n1 = make_float2(nc.z, nc.w);
+                float2 da = __fadd2_rn(xa[j], n0), db = __fadd2_rn(xb[j], n0);
+                aa = __ffma2_rn(da, da, aa);
+                ab = __ffma2_rn(db, db, ab);
+                da = __fadd2_rn(xa[j + 1], n1);
+                db = __fadd2_rn(xb[j + 1], n1);
+                aa = __ffma2_rn(da, da, aa);
+                ab = __ffma2_rn(db, db, ab);
+            }
+            if (aa.x < bd[0]) { bd[0] = aa.x; bi[0] = c; }
+            if (aa.y < bd[1]) { bd[1] = aa.y; bi[1] = c; }
+            if (ab.x < bd[2]) { bd[2] = ab.x; bi[2] = c; }
+            if (ab.y < bd[3]) { bd[3] = ab.y; bi[3] = c; }
+        }
+#pragma unroll
+        for (int q = 0; q < kPPT; ++q) {
+            if (!ok[q]) continue;
+            member[pb + q] = bi[q];
+            atomicAdd(s_cnt + bi[q], 1ull);
+#pragma unroll
+            for (int j = 0; j < D; ++j) {
+                const float xv = q == 0 ? xa[j].x : q == 1 ? xa[j].y : q == 2 ? xb[j].x : xb[j].y;
+                atomicAdd(s_sum + bi[q] * D + j, (unsigned long long)fixed_of(xv, scale, err));
+            }
+        }
+    }
+    flush_block(s_sum, s_cnt, sums, counts, kc, D);
+}
+
+// Generic d (any d <= 32): one point per thread, scalar fmaf chain in the same order.
+__global__ void __launch_bounds__(kThreads)
+assign_generic(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __restrict__ member,
+               int64_t* __restrict__ sums, int64_t* __restrict__ counts, int64_t p0, int64_t p1, int d, int kc,
+               int shift, int* err) {
+    extern __shared__ __align__(16) unsigned char smem[];
+    float* s_c = reinterpret_cast<float*>(smem);
+    unsigned long long* s_sum = reinterpret_cast<unsigned long long*>(smem + ((kc * d * 4 + 15) / 16) * 16);
+    unsigned long long* s_cnt = s_sum + kc * d;
+    for (int i = threadIdx.x; i < kc * d; i += kThreads) { s_c[i] = cen[i]; s_sum[i] = 0ull; }
+    for (int i = threadIdx.x; i < kc; i += kThreads) s_cnt[i] = 0ull;
+    __syncthreads();
+    const float scale = (float)(1 << shift);
+    for (int64_t p = p0 + (int64_t)blockIdx.x * kThreads + threadIdx.x; p < p1; p += (int64_t)gridDim.x * kThreads) {
+        float xv[32];
+        for (int j = 0; j < d; ++j) xv[j] = x[p * d + j];
+        float bd = __int_as_float(0x7f800000);
+        int bi = 0;
+        for (int c = 0; c < kc; ++c) {
+            float acc = 0.f;
+            for (int j = 0; j < d; ++j) {
+                const float df = __fsub_rn(xv[j], s_c[c * d + j]);
+                acc = __fmaf_rn(df, df, acc);
+            }
+            if (acc < bd) { bd = acc; bi = c; }
+        }
+        member[p] = bi;
+        atomicAdd(s_cnt + bi, 1ull);
+        for (int j = 0; j < d; ++j) atomicAdd(s_sum + bi * d + j, (unsigned long long)fixed_of(xv[j], scale, err));
+    }
+    flush_block(s_sum, s_cnt, sums, counts, kc, d);
+}
+
+// Update loop, element pass: e = c*d + j over clusters [c0, c1):
+//   if counts[c] > 0: cen[e] = (float)(((double)sums[e] * 2^-shift) / (double)counts[c]);  sums[e] = 0.
+template <bool TRACK>
+__global__ void __launch_bounds__(kThreads)
+update_elems(int64_t* __restrict__ sums, const int64_t* __restrict__ counts, float* __restrict__ cen, int64_t c0,
+             int64_t c1, int d, int shift, Track ts, Track tc) {
+    const int64_t e0 = c0 * d, e1 = c1 * d;
+    const double inv = 1.0 / (double)(1ll << shift);  // exact power of two
+    int64_t cs = -1, cc = -1;
+    for (int64_t base = e0 + (int64_t)blockIdx.x * kThreads; base < e1; base += (int64_t)gridDim.x * kThreads) {
+        const int64_t e = base + threadIdx.x;
+        const bool ok = e < e1;
+        bool wc = false;
+        if (ok) {
+            const int64_t c = e / d;
+            const int64_t cnt = counts[c];
+            if (cnt > 0) {
+                cen[e] = (float)(__dmul_rn((double)sums[e], inv) / (double)cnt);
+                wc = true;
+            }
+            sums[e] = 0;
+        }
+        if constexpr (TRACK) {
+            const int64_t wb = base + (threadIdx.x & ~31);
+            if (ts.l1) dev::track_warp<1>(ts.l1, ts.l2, ts.l2_shift, wb, ok ? 1u : 0u, cs);
+            if (tc.l1) dev::track_warp<1>(tc.l1, tc.l2, tc.l2_shift, wb, wc ? 1u : 0u, cc);
+        }
+    }
+}
+
+// Update loop, cluster pass: counts[c] = 0 for c in [c0, c1) (after the element pass read them).
+template <bool TRACK>
+__global__ void __launch_bounds__(kThreads)
+update_counts(int64_t* __restrict__ counts, int64_t c0, int64_t c1, Track t) {
+    int64_t l2c = -1;
+    for (int64_t base = c0 + (int64_t)blockIdx.x * kThreads; base < c1; base += (int64_t)gridDim.x * kThreads) {
+        const int64_t c = base + threadIdx.x;
+        if (c < c1) counts[c] = 0;
+        if constexpr (TRACK) {
+            if (t.l1) dev::track_warp<1>(t.l1, t.l2, t.l2_shift, base + (threadIdx.x & ~31), c < c1 ? 1u : 0u, l2c);
+        }
+    }
+}
+
+int sm_count() {
+    static int n = 0;
+    if (!n) {
+        int dev = 0;
+        cudaGetDevice(&dev);
+        cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev);
+        if (n <= 0) n = 148;
+    }
+    return n;
+}
+
+}  // namespace
+
+cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int64_t* sums, int64_t* counts,
+                          int64_t p0, int64_t p1, int d, int kc, int shift, int* err_flag, cudaStream_t s,
+                          int64_t* launches) {
+    if (p1 <= p0) return cudaSuccess;
+    const int sms = sm_count();
+    if (d == 16 && (reinterpret_cast<uintptr_t>(x) % 16) == 0) {
+        const size_t smem = (size_t)kc * 16 * 8 + (size_t)kc * 16 * 8 + (size_t)kc * 8;
+        if (smem > 200 * 1024) return cudaErrorNotSupported;
+        cudaError_t e = cudaFuncSetAttribute(assign_d<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        int per_sm = 0;
+        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, assign_d<16>, kThreads, smem);
+        const int64_t groups = (p1 - p0 + kPPT - 1) / kPPT;
+        int64_t blocks = (groups + kThreads - 1) / kThreads;
+        const int64_t cap = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
+        if (blocks > cap) blocks = cap;
+        assign_d<16><<<(unsigned)blocks, kThreads, smem, s>>>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag);
+    } else {
+        const size_t smem = (((size_t)kc * d * 4 + 15) / 16) * 16 + (size_t)kc * d * 8 + (size_t)kc * 8;
+        if (smem > 200 * 1024) return cudaErrorNotSupported;
+        cudaError_t e = cudaFuncSetAttribute(assign_generic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        if (e != cudaSuccess) return e;
+        int64_t blocks = (p1 - p0 + kThreads - 1) / kThreads;
+        if (blocks > (int64_t)sms * 4) blocks = (int64_t)sms * 4;
+        assign_generic<<<(unsigned)blocks, kThreads, smem, s>>>(x, cen, member, sums, counts, p0, p1, d, kc, shift, err_flag);
+    }
+    if (launches) *launches += 1;
+    return cudaGetLastError();
+}
+
+cudaError_t kmeans_update(int64_t* sums, int64_t* counts, float* cen, int64_t c0, int64_t c1, int d, int shift,
+                          Track t_sums, Track t_counts, Track t_cen, cudaStream_t s, int64_t* launches) {
+    if (c1 <= c0) return cudaSuccess;
+    const bool tr = t_sums.l1 || t_cen.l1;
+    int64_t nb = ((c1 - c0) * d + kThreads - 1) / kThreads;
+    if (nb > 1184) nb = 1184;
+    if (tr) update_elems<true><<<(unsigned)nb, kThreads, 0, s>>>(sums, counts, cen, c0, c1, d, shift, t_sums, t_cen);
+    else update_elems<false><<<(unsigned)nb, kThreads, 0, s>>>(sums, counts, cen, c0, c1, d, shift, t_sums, t_cen);
+    int64_t nc = (c1 - c0 + kThreads - 1) / kThreads;
+    if (nc > 1184) nc = 1184;
+    if (t_counts.l1) update_counts<true><<<(unsigned)nc, kThreads, 0, s>>>(counts, c0, c1, t_counts);
+    else update_counts<false><<<(unsigned)nc, kThreads, 0, s>>>(counts, c0, c1, t_counts);
+    if (launches) *launches += 2;
+    return cudaGetLastError();
+}
+
+}  // namespace k
+}  // namespace accmg

@@ -1,0 +1,1059 @@
+// accmg runtime: the C ABI of include/accmg.h.
+//
+// Host side of one offloaded parallel loop (§III.A, three BSP steps):
+//   1. task mapping (L108): dim 0 of the iteration space is divided into P contiguous chunks;
+//   2. data loader (L117-125 §IV.C): per region, each partition needs its declared window
+//      (distribution policy, L121-123) or the whole array (replica policy, L121); what it does not
+//      already hold is pulled — from the partition that holds it (device copy or NCCL) or from the
+//      host copy — and nothing moves when the read pattern repeats (L125);
+//   3. body kernels on every local partition (loop bodies of csrc/*.cu);
+//   4. inter-GPU communication manager (L127-137 §IV.D): declared writes move ownership (the data
+//      follows lazily when a later loop reads it); undeclared writes were tracked with two-level
+//      dirty bits, are compacted into packed runs and scattered into every other replica;
+//      reductiontoarray destinations are merged block -> GPU -> across GPUs (L112);
+//   5. global barrier (L64): stream order on each process; NCCL ops order across processes.
+//
+// State per region: one full-extent replica per local partition (global indices, so the index
+// rewriting of L110 is the identity) and a validity table: for every partition (all ranks keep the
+// whole table, identical everywhere because every call is collective) the set of element intervals
+// whose value there is current, plus this process's host-copy validity.
+#include "accmg.h"
+
+#include <cuda_runtime_api.h>
+
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "intervals.h"
+#include "kernels.h"
+#include "nccl_dl.h"
+
+using accmg::IntervalSet;
+using accmg::Ival;
+namespace k = accmg::k;
+
+namespace {
+
+struct Trk {  // dirty-bit tracking + packed send buffer of one local replica (L133-135)
+    uint32_t* l1 = nullptr;
+    uint32_t* l2 = nullptr;
+    int64_t nwords = 0, nl2 = 0, ntiles = 0;
+    int64_t* tile_counts = nullptr;
+    int64_t* tile_offs = nullptr;
+    uint32_t* tile_edges = nullptr;
+    int64_t* totals = nullptr;  // device {n_runs, n_elems, dirty_chunks, n_run_ends}
+    uint8_t* packed = nullptr;
+    int64_t packed_cap = 0, packed_bytes = 0, n_runs = 0, n_elems = 0, dirty_chunks = 0;
+    uint32_t* snap_l1 = nullptr;
+    uint32_t* snap_l2 = nullptr;
+    bool has_snap = false, has_packed = false;
+};
+
+}  // namespace
+
+struct accmg_region_s {
+    int64_t id = 0;
+    uint8_t* host = nullptr;
+    int64_t esize = 0, extent = 0;
+    std::vector<uint8_t*> dev;       // V local replicas (full extent)
+    std::vector<IntervalSet> valid;  // P partitions
+    IntervalSet host_valid;          // this process's host copy
+    std::vector<Trk> trk;            // V
+    std::vector<int64_t*> partial;   // V reduction partials (REDUCE_SUM)
+};
+
+namespace {
+
+struct Prof {
+    cudaEvent_t a, b;
+    int kind;  // 0 body, 1 compaction, 2 exchange
+};
+
+struct State {
+    bool init = false;
+    accmg_config cfg{};
+    int P = 1, W = 1, rank = 0, V = 1;
+    bool dry = false, nccl_all = false;
+    int64_t chunk_bytes = 1 << 20;
+    cudaStream_t stream = nullptr;
+    accmg::NcclApi* nccl = nullptr;
+    ncclComm_t comm = nullptr;
+    int sticky = 0;
+    std::string err = "no error";
+    std::vector<accmg_region_s*> regions;
+    int64_t next_id = 1;
+    accmg_stats st{};
+    int64_t* scratch = nullptr;     // scatter scratch
+    int64_t* h_pin = nullptr;       // pinned host staging (sizes)
+    int64_t* d_sizes = nullptr;     // 4*P int64 (send + all-gathered sizes)
+    int* d_flag = nullptr;
+    uint8_t* recv = nullptr;
+    int64_t recv_cap = 0;
+    std::vector<Prof> prof;
+    std::vector<cudaEvent_t> ev_free;
+};
+
+State S;
+
+int fail(int code, const std::string& msg, bool sticky) {
+    if (sticky && !S.sticky) S.sticky = code;
+    S.err = msg;
+    return code;
+}
+
+#define CUDA_TRY(x)                                                                                   \
+    do {                                                                                              \
+        cudaError_t e_ = (x);                                                                         \
+        if (e_ != cudaSuccess) {                                                                      \
+            if (e_ == cudaErrorMemoryAllocation) {                                                    \
+                cudaGetLastError();                                                                   \
+                return fail(ACCMG_ENOMEM, std::string(#x) + ": " + cudaGetErrorString(e_), false);  \
+            }                                                                                         \
+            return fail(ACCMG_ECUDA, std::string(#x) + ": " + cudaGetErrorString(e_), true);        \
+        }                                                                                             \
+    } while (0)
+
+#define NCCL_TRY(x)                                                                                         \
+    do {                                                                                                    \
+        ncclResult_t r_ = (x);                                                                              \
+        if (r_ != ncclSuccess) return fail(ACCMG_ENCCL, std::string(#x) + ": " + S.nccl->GetErrorString(r_), true); \
+    } while (0)
+
+#define TRY(x)                  \
+    do {                        \
+        int rc_ = (x);          \
+        if (rc_ != 0) return rc_; \
+    } while (0)
+
+#define GUARD()                                                            \
+    do {                                                                   \
+        if (S.sticky) return S.sticky;                                     \
+        if (!S.init) return fail(ACCMG_ESTATE, "accmg: not initialised", false); \
+        if (!S.dry) CUDA_TRY(cudaSetDevice(S.cfg.device));                 \
+    } while (0)
+
+inline int rank_of(int g) { return g / S.V; }
+inline bool local(int g) { return rank_of(g) == S.rank; }
+inline int lidx(int g) { return g % S.V; }
+inline int first_local() { return S.rank * S.V; }
+
+void chunk_of(int64_t lo, int64_t hi, int P, int g, int64_t* a, int64_t* b) {
+    // L108: "the tasks in the parallel loop are equally divided among the GPUs" (reading G6)
+    __int128 n = hi - lo;
+    *a = lo + (int64_t)((n * g) / P);
+    *b = lo + (int64_t)((n * (g + 1)) / P);
+}
+
+// Union over iterations [a, b) of the localaccess windows (L87), clipped to [0, extent).
+IntervalSet window(const accmg_access& d, int64_t a, int64_t b, int64_t extent) {
+    if (a >= b) return IntervalSet();
+    int64_t lo = d.stride * a - d.left;
+    int64_t hi = d.stride * b + d.right;  // = stride*(b-1) + stride - 1 + right + 1
+    lo = std::max<int64_t>(lo, 0);
+    hi = std::min<int64_t>(hi, extent);
+    return IntervalSet(lo, hi);
+}
+
+int dmalloc(void** p, size_t bytes, bool system) {
+    if (bytes == 0) bytes = 16;
+    cudaError_t e = cudaMalloc(p, bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        return fail(ACCMG_ENOMEM, std::string("cudaMalloc(") + std::to_string(bytes) + "): " + cudaGetErrorString(e),
+                    false);
+    }
+    (system ? S.st.device_bytes_system : S.st.device_bytes_user) += (int64_t)bytes;
+    return 0;
+}
+
+void dfree(void* p, size_t bytes, bool system) {
+    if (!p) return;
+    cudaFree(p);
+    (system ? S.st.device_bytes_system : S.st.device_bytes_user) -= (int64_t)bytes;
+}
+
+cudaEvent_t ev_get() {
+    if (!S.ev_free.empty()) {
+        cudaEvent_t e = S.ev_free.back();
+        S.ev_free.pop_back();
+        return e;
+    }
+    cudaEvent_t e;
+    cudaEventCreate(&e);
+    return e;
+}
+
+struct ProfScope {
+    int kind;
+    cudaEvent_t a = nullptr;
+    explicit ProfScope(int kd) : kind(kd) {
+        if (S.cfg.profile && !S.dry) {
+            a = ev_get();
+            cudaEventRecord(a, S.stream);
+        }
+    }
+    ~ProfScope() {
+        if (a) {
+            cudaEvent_t b = ev_get();
+            cudaEventRecord(b, S.stream);
+            S.prof.push_back({a, b, kind});
+        }
+    }
+};
+
+int collect_prof() {
+    if (S.prof.empty()) return 0;
+    CUDA_TRY(cudaStreamSynchronize(S.stream));
+    for (auto& p : S.prof) {
+        float ms = 0.f;
+        cudaEventElapsedTime(&ms, p.a, p.b);
+        (p.kind == 0 ? S.st.ms_body : p.kind == 1 ? S.st.ms_compact : S.st.ms_exchange) += ms;
+        S.ev_free.push_back(p.a);
+        S.ev_free.push_back(p.b);
+    }
+    S.prof.clear();
+    return 0;
+}
+
+// ---- transfers between partitions (data loader pulls) -----------------------------------------
+struct Xfer {
+    accmg_region_s* r;
+    int dst, src;  // src = -1: the host copy of rank_of(dst)
+    int64_t lo, hi;
+};
+
+// Plans the pulls that make need[g] valid on every partition g; sources are chosen from the state
+// before the phase: partitions of the same process first, then other processes, ascending index;
+// the host copy only for what no partition holds.
+void plan_pulls(accmg_region_s* r, const std::vector<IntervalSet>& need, std::vector<Xfer>& out) {
+    for (int g = 0; g < S.P; ++g) {
+        IntervalSet miss = need[g];
+        miss.subtract(r->valid[g]);
+        if (miss.empty()) continue;
+        std::vector<int> order;
+        for (int h = 0; h < S.P; ++h)
+            if (h != g && rank_of(h) == rank_of(g)) order.push_back(h);
+        for (int h = 0; h < S.P; ++h)
+            if (rank_of(h) != rank_of(g)) order.push_back(h);
+        for (int h : order) {
+            if (miss.empty()) break;
+            IntervalSet piece = miss.intersect(r->valid[h]);
+            for (auto& iv : piece.items()) out.push_back({r, g, h, iv.lo, iv.hi});
+            miss.subtract(piece);
+        }
+        for (auto& iv : miss.items()) out.push_back({r, g, -1, iv.lo, iv.hi});
+    }
+}
+
+int run_xfers(const std::vector<Xfer>& xs) {
+    // accounting (partition-to-partition bytes are whole-job totals, identical on every rank)
+    for (auto& x : xs) {
+        int64_t nb = (x.hi - x.lo) * x.r->esize;
+        if (x.src >= 0) {
+            S.st.bytes_interpartition += nb;
+            S.st.bytes_declared += nb;
+            if (rank_of(x.src) != rank_of(x.dst)) S.st.bytes_remote += nb;
+        } else if (local(x.dst)) {
+            S.st.bytes_h2d += nb;
+            if (!x.r->host_valid.contains(IntervalSet(x.lo, x.hi)))
+                return fail(ACCMG_ESTATE, "data loader: range valid on no partition and not on the host copy", false);
+        }
+    }
+    if (S.dry) return 0;
+    ProfScope ps(2);
+    bool any_nccl = false;
+    for (auto& x : xs) {
+        const size_t nb = (size_t)((x.hi - x.lo) * x.r->esize);
+        const int64_t off = x.lo * x.r->esize;
+        if (x.src < 0) {
+            if (local(x.dst))
+                CUDA_TRY(cudaMemcpyAsync(x.r->dev[lidx(x.dst)] + off, x.r->host + off, nb, cudaMemcpyHostToDevice,
+                                         S.stream));
+        } else if (local(x.src) && local(x.dst) && !S.nccl_all) {
+            CUDA_TRY(cudaMemcpyAsync(x.r->dev[lidx(x.dst)] + off, x.r->dev[lidx(x.src)] + off, nb,
+                                     cudaMemcpyDeviceToDevice, S.stream));
+        } else if (local(x.src) || local(x.dst)) {
+            any_nccl = true;
+        }
+    }
+    if (any_nccl) {
+        NCCL_TRY(S.nccl->GroupStart());
+        for (auto& x : xs) {
+            if (x.src < 0) continue;
+            const bool viaN = rank_of(x.src) != rank_of(x.dst) || S.nccl_all;
+            if (!viaN) continue;
+            const size_t nb = (size_t)((x.hi - x.lo) * x.r->esize);
+            const int64_t off = x.lo * x.r->esize;
+            if (local(x.src))
+                NCCL_TRY(S.nccl->Send(x.r->dev[lidx(x.src)] + off, nb, ncclUint8, rank_of(x.dst), S.comm, S.stream));
+            if (local(x.dst))
+                NCCL_TRY(S.nccl->Recv(x.r->dev[lidx(x.dst)] + off, nb, ncclUint8, rank_of(x.src), S.comm, S.stream));
+        }
+        NCCL_TRY(S.nccl->GroupEnd());
+    }
+    return 0;
+}
+
+// ---- tracking buffers ---------------------------------------------------------------------------
+int chunk_elems(const accmg_region_s* r) { return (int)std::max<int64_t>(S.chunk_bytes / r->esize, 32); }
+
+int ensure_trk(accmg_region_s* r, int li) {
+    Trk& t = r->trk[li];
+    if (t.l1) return 0;
+    const int64_t ce = chunk_elems(r);
+    t.nwords = (r->extent + 31) / 32;
+    const int64_t nchunks = (r->extent + ce - 1) / ce;
+    t.nl2 = (nchunks + 31) / 32;
+    t.ntiles = (t.nwords + k::kTileWords - 1) / k::kTileWords;
+    TRY(dmalloc((void**)&t.l1, t.nwords * 4, true));
+    TRY(dmalloc((void**)&t.l2, t.nl2 * 4, true));
+    TRY(dmalloc((void**)&t.tile_counts, t.ntiles * 24, true));
+    TRY(dmalloc((void**)&t.tile_offs, t.ntiles * 24, true));
+    TRY(dmalloc((void**)&t.tile_edges, t.ntiles * 8, true));
+    TRY(dmalloc((void**)&t.totals, 64, true));
+    CUDA_TRY(cudaMemsetAsync(t.l1, 0, t.nwords * 4, S.stream));
+    CUDA_TRY(cudaMemsetAsync(t.l2, 0, t.nl2 * 4, S.stream));
+    if (S.cfg.debug_checks) {
+        TRY(dmalloc((void**)&t.snap_l1, t.nwords * 4, true));
+        TRY(dmalloc((void**)&t.snap_l2, t.nl2 * 4, true));
+    }
+    return 0;
+}
+
+int ensure_packed(Trk& t, int64_t bytes) {
+    if (t.packed_cap >= bytes) return 0;
+    int64_t cap = std::max<int64_t>(bytes, t.packed_cap + t.packed_cap / 2);
+    if (t.packed) {
+        CUDA_TRY(cudaStreamSynchronize(S.stream));
+        dfree(t.packed, t.packed_cap, true);
+        t.packed = nullptr;
+    }
+    TRY(dmalloc((void**)&t.packed, cap, true));
+    t.packed_cap = cap;
+    return 0;
+}
+
+int ensure_recv(int64_t bytes) {
+    if (S.recv_cap >= bytes) return 0;
+    if (S.recv) {
+        CUDA_TRY(cudaStreamSynchronize(S.stream));
+        dfree(S.recv, S.recv_cap, true);
+        S.recv = nullptr;
+    }
+    TRY(dmalloc((void**)&S.recv, bytes, true));
+    S.recv_cap = bytes;
+    return 0;
+}
+
+k::Track track_of(accmg_region_s* r, int li, bool on) {
+    k::Track t{nullptr, nullptr, 0};
+    if (!on) return t;
+    t.l1 = r->trk[li].l1;
+    t.l2 = r->trk[li].l2;
+    int sh = 0;
+    while ((1ll << sh) < chunk_elems(r)) ++sh;
+    t.l2_shift = sh;
+    return t;
+}
+
+// ---- bodies ---------------------------------------------------------------------------------------
+struct BodySpec {
+    int n;
+    int mode[5];
+    int esize[5];
+    int ndim;
+    size_t args;
+};
+
+bool body_spec(int id, BodySpec* b) {
+    switch (id) {
+        case ACCMG_BODY_JACOBI2D_5PT: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 2, sizeof(accmg_args_jacobi2d)}; return true;
+        case ACCMG_BODY_GEMM_BF16_F32: *b = {3, {ACCMG_R, ACCMG_R, ACCMG_W}, {2, 2, 4}, 2, sizeof(accmg_args_gemm)}; return true;
+        case ACCMG_BODY_KMEANS_ASSIGN:
+            *b = {5, {ACCMG_R, ACCMG_R, ACCMG_W, ACCMG_REDUCE_SUM, ACCMG_REDUCE_SUM}, {4, 4, 4, 8, 8}, 1,
+                  sizeof(accmg_args_kmeans)};
+            return true;
+        case ACCMG_BODY_KMEANS_UPDATE:
+            *b = {3, {ACCMG_RW, ACCMG_RW, ACCMG_W}, {8, 8, 4}, 1, sizeof(accmg_args_kmeans)};
+            return true;
+        case ACCMG_BODY_TEST_SPARSE_WRITE: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 1, sizeof(accmg_args_sparse)}; return true;
+        default: return false;
+    }
+}
+
+int validate_body(const accmg_bounds* bd, int body, const accmg_access* d, const void* args) {
+    auto bad = [](const std::string& m) { return fail(ACCMG_EINVAL, "loop_launch: " + m, false); };
+    auto ext = [&](int i) { return d[i].region->extent; };
+    switch (body) {
+        case ACCMG_BODY_JACOBI2D_5PT: {
+            auto a = static_cast<const accmg_args_jacobi2d*>(args);
+            if (a->rows < 3 || a->cols < 3) return bad("jacobi: rows, cols >= 3");
+            if (ext(0) != a->rows * a->cols || ext(1) != a->rows * a->cols) return bad("jacobi: region extent != rows*cols");
+            if (bd->lo[0] < 1 || bd->hi[0] > a->rows - 1 || bd->lo[1] < 1 || bd->hi[1] > a->cols - 1)
+                return bad("jacobi: bounds must lie in [1,rows-1) x [1,cols-1)");
+            if (d[0].region == d[1].region) return bad("jacobi: src and dst must differ");
+            return 0;
+        }
+        case ACCMG_BODY_TEST_SPARSE_WRITE: {
+            auto a = static_cast<const accmg_args_sparse*>(args);
+            if (a->rows < 1 || a->cols < 1 || a->period < 1) return bad("sparse: rows, cols, period >= 1");
+            if (ext(0) != a->rows * a->cols || ext(1) != a->rows * a->cols) return bad("sparse: extent != rows*cols");
+            if (bd->lo[0] < 0 || bd->hi[0] > a->rows) return bad("sparse: bounds outside [0,rows)");
+            if (d[0].region == d[1].region) return bad("sparse: in and out must differ");
+            return 0;
+        }
+        case ACCMG_BODY_GEMM_BF16_F32: {
+            auto a = static_cast<const accmg_args_gemm*>(args);
+            if (a->M < 1 || a->N < 1 || a->K < 1) return bad("gemm: M, N, K >= 1");
+            if (ext(0) != a->M * a->K || ext(1) != a->K * a->N || ext(2) != a->M * a->N) return bad("gemm: extents");
+            if (bd->lo[0] < 0 || bd->hi[0] > a->M || bd->lo[1] != 0 || bd->hi[1] != a->N)
+                return bad("gemm: bounds must be rows within [0,M) x all of [0,N)");
+            if (a->N % 16 != 0 || a->K % 64 != 0) return fail(ACCMG_EUNSUPPORTED, "gemm: needs N % 16 == 0, K % 64 == 0", false);
+            return 0;
+        }
+        case ACCMG_BODY_KMEANS_ASSIGN:
+        case ACCMG_BODY_KMEANS_UPDATE: {
+            auto a = static_cast<const accmg_args_kmeans*>(args);
+            if (a->n < 1 || a->d < 1 || a->k < 1 || a->shift < 0 || a->shift > 30) return bad("kmeans: n, d, k >= 1, shift in [0,30]");
+            if (a->d > 32 || a->k > 1024) return fail(ACCMG_EUNSUPPORTED, "kmeans: d <= 32, k <= 1024", false);
+            if (body == ACCMG_BODY_KMEANS_ASSIGN) {
+                if (ext(0) != a->n * a->d || ext(1) != (int64_t)a->k * a->d || ext(2) != a->n ||
+                    ext(3) != (int64_t)a->k * a->d || ext(4) != a->k)
+                    return bad("kmeans_assign: extents");
+                if (bd->lo[0] < 0 || bd->hi[0] > a->n) return bad("kmeans_assign: bounds outside [0,n)");
+            } else {
+                if (ext(0) != (int64_t)a->k * a->d || ext(1) != a->k || ext(2) != (int64_t)a->k * a->d)
+                    return bad("kmeans_update: extents");
+                if (bd->lo[0] < 0 || bd->hi[0] > a->k) return bad("kmeans_update: bounds outside [0,k)");
+            }
+            return 0;
+        }
+    }
+    return bad("unknown body");
+}
+
+int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const void* args, int g, int64_t a,
+                int64_t b, const std::vector<bool>& tracked) {
+    const int li = lidx(g);
+    auto P = [&](int i) { return d[i].region->dev[li]; };
+    auto T = [&](int i) { return track_of(d[i].region, li, tracked[i]); };
+    cudaError_t e = cudaSuccess;
+    int64_t* L = &S.st.kernel_launches;
+    switch (body) {
+        case ACCMG_BODY_JACOBI2D_5PT: {
+            auto x = static_cast<const accmg_args_jacobi2d*>(args);
+            e = k::jacobi2d((const float*)P(0), (float*)P(1), x->rows, x->cols, a, b, bd->lo[1], bd->hi[1], T(1), 0,
+                            S.stream, L);
+            break;
+        }
+        case ACCMG_BODY_TEST_SPARSE_WRITE: {
+            auto x = static_cast<const accmg_args_sparse*>(args);
+            e = k::sparse_rows((const float*)P(0), (float*)P(1), x->rows, x->cols, a, b, x->period, T(1), S.stream, L);
+            break;
+        }
+        case ACCMG_BODY_GEMM_BF16_F32: {
+            auto x = static_cast<const accmg_args_gemm*>(args);
+            e = k::gemm_bf16((const uint16_t*)P(0), (const uint16_t*)P(1), (float*)P(2), x->M, x->N, x->K, a, b,
+                             S.stream, L);
+            break;
+        }
+        case ACCMG_BODY_KMEANS_ASSIGN: {
+            auto x = static_cast<const accmg_args_kmeans*>(args);
+            e = k::kmeans_assign((const float*)P(0), (const float*)P(1), (int32_t*)P(2), d[3].region->partial[li],
+                                 d[4].region->partial[li], a, b, x->d, x->k, x->shift, S.d_flag + 1, S.stream, L);
+            break;
+        }
+        case ACCMG_BODY_KMEANS_UPDATE: {
+            auto x = static_cast<const accmg_args_kmeans*>(args);
+            e = k::kmeans_update((int64_t*)P(0), (int64_t*)P(1), (float*)P(2), a, b, x->d, x->shift, T(0), T(1), T(2),
+                                 S.stream, L);
+            break;
+        }
+    }
+    if (e == cudaErrorNotSupported) return fail(ACCMG_EUNSUPPORTED, "body not supported on this build/shape", false);
+    CUDA_TRY(e);
+    S.st.body_launches += 1;
+    return 0;
+}
+
+// ---- coherence of undeclared writes (L129-135) -----------------------------------------------------
+int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
+    // 1. per local replica: (debug snapshot), count, scan
+    {
+        ProfScope ps(1);
+        for (auto* r : regs)
+            for (int li = 0; li < S.V; ++li) {
+                Trk& t = r->trk[li];
+                if (S.cfg.debug_checks) {
+                    CUDA_TRY(cudaMemcpyAsync(t.snap_l1, t.l1, t.nwords * 4, cudaMemcpyDeviceToDevice, S.stream));
+                    CUDA_TRY(cudaMemcpyAsync(t.snap_l2, t.l2, t.nl2 * 4, cudaMemcpyDeviceToDevice, S.stream));
+                    t.has_snap = true;
+                }
+                int cw = 0;
+                while ((1ll << cw) < chunk_elems(r) / 32) ++cw;
+                CUDA_TRY(k::compact_count(t.l1, t.l2, t.nwords, cw, t.ntiles, t.tile_counts, t.tile_edges, S.stream,
+                                          &S.st.kernel_launches));
+                CUDA_TRY(k::compact_scan(t.tile_counts, t.ntiles, t.tile_offs, t.totals, t.l2, t.nl2, S.stream,
+                                         &S.st.kernel_launches));
+            }
+        if (S.cfg.debug_checks) {
+            CUDA_TRY(cudaMemsetAsync(S.d_flag, 0, sizeof(int), S.stream));
+            for (auto* r : regs)
+                for (int a = 0; a < S.V; ++a)
+                    for (int b = a + 1; b < S.V; ++b)
+                        CUDA_TRY(k::bitmap_overlap(r->trk[a].snap_l1, r->trk[b].snap_l1, r->trk[a].nwords, S.d_flag,
+                                                   S.stream, &S.st.kernel_launches));
+        }
+    }
+    // 2. sizes to the host (one synchronisation for all regions)
+    int slot = 0;
+    for (auto* r : regs)
+        for (int li = 0; li < S.V; ++li, ++slot)
+            CUDA_TRY(cudaMemcpyAsync(S.h_pin + 4 * slot, r->trk[li].totals, 32, cudaMemcpyDeviceToHost, S.stream));
+    if (S.cfg.debug_checks)
+        CUDA_TRY(cudaMemcpyAsync((int*)(S.h_pin + 4 * slot), S.d_flag, sizeof(int), cudaMemcpyDeviceToHost, S.stream));
+    CUDA_TRY(cudaStreamSynchronize(S.stream));
+    if (S.cfg.debug_checks && *(int*)(S.h_pin + 4 * slot))
+        return fail(ACCMG_ECONFLICT, "two partitions wrote the same replicated element (L62: no dependences)", false);
+    slot = 0;
+    for (auto* r : regs)
+        for (int li = 0; li < S.V; ++li, ++slot) {
+            Trk& t = r->trk[li];
+            t.n_runs = S.h_pin[4 * slot];
+            t.n_elems = S.h_pin[4 * slot + 1];
+            t.dirty_chunks = S.h_pin[4 * slot + 2];
+            if (S.h_pin[4 * slot + 3] != t.n_runs) return fail(ACCMG_ECUDA, "compaction: run starts != run ends", true);
+            t.packed_bytes = 16 + 16 * t.n_runs + r->esize * t.n_elems;
+            TRY(ensure_packed(t, t.packed_bytes));
+            CUDA_TRY(cudaMemcpyAsync(t.packed, t.totals, 16, cudaMemcpyDeviceToDevice, S.stream));
+            ProfScope ps(1);
+            CUDA_TRY(k::compact_write(t.l1, t.nwords, t.ntiles, t.tile_counts, t.tile_offs, t.tile_edges, r->dev[li],
+                                      (int)r->esize, t.packed, t.n_runs, S.stream, &S.st.kernel_launches));
+            t.has_packed = true;
+        }
+    // 3. sizes of every partition's packet (all-gather across processes when needed)
+    std::vector<int64_t> runs(S.P * regs.size()), elems(S.P * regs.size()), chunks(S.P * regs.size());
+    const bool multi = S.W > 1 || S.nccl_all;
+    if (multi) {
+        // layout per rank: [region][local] x {runs, elems, chunks, pad}
+        const int64_t per = (int64_t)regs.size() * S.V * 4;
+        slot = 0;
+        for (auto* r : regs)
+            for (int li = 0; li < S.V; ++li, ++slot) {
+                S.h_pin[4 * slot] = r->trk[li].n_runs;
+                S.h_pin[4 * slot + 1] = r->trk[li].n_elems;
+                S.h_pin[4 * slot + 2] = r->trk[li].dirty_chunks;
+                S.h_pin[4 * slot + 3] = 0;
+            }
+        CUDA_TRY(cudaMemcpyAsync(S.d_sizes, S.h_pin, per * 8, cudaMemcpyHostToDevice, S.stream));
+        NCCL_TRY(S.nccl->AllGather(S.d_sizes, S.d_sizes + per, per, ncclInt64, S.comm, S.stream));
+        CUDA_TRY(cudaMemcpyAsync(S.h_pin, S.d_sizes + per, per * S.W * 8, cudaMemcpyDeviceToHost, S.stream));
+        CUDA_TRY(cudaStreamSynchronize(S.stream));
+        for (int q = 0; q < S.W; ++q)
+            for (size_t ri = 0; ri < regs.size(); ++ri)
+                for (int li = 0; li < S.V; ++li) {
+                    const int64_t* v = S.h_pin + q * per + 4 * (ri * S.V + li);
+                    const int g = q * S.V + li;
+                    runs[ri * S.P + g] = v[0];
+                    elems[ri * S.P + g] = v[1];
+                    chunks[ri * S.P + g] = v[2];
+                }
+    } else {
+        for (size_t ri = 0; ri < regs.size(); ++ri)
+            for (int li = 0; li < S.V; ++li) {
+                runs[ri * S.P + li] = regs[ri]->trk[li].n_runs;
+                elems[ri * S.P + li] = regs[ri]->trk[li].n_elems;
+                chunks[ri * S.P + li] = regs[ri]->trk[li].dirty_chunks;
+            }
+    }
+    // accounting: every packet is delivered to the P-1 other partitions (reading W8)
+    for (size_t ri = 0; ri < regs.size(); ++ri) {
+        const int64_t es = regs[ri]->esize, ce = chunk_elems(regs[ri]);
+        for (int g = 0; g < S.P; ++g) {
+            const int64_t hdr = 16 + 16 * runs[ri * S.P + g], pay = es * elems[ri * S.P + g];
+            S.st.bytes_undeclared_headers += (S.P - 1) * hdr;
+            S.st.bytes_undeclared_payload += (S.P - 1) * pay;
+            S.st.bytes_interpartition += (S.P - 1) * (hdr + pay);
+            S.st.bytes_paper_protocol += (S.P - 1) * chunks[ri * S.P + g] * (ce * es + ce / 8);
+            if (multi) S.st.bytes_remote += (int64_t)(S.W - 1 + (S.nccl_all ? 1 : 0)) * (hdr + pay);
+        }
+    }
+    // 4. exchange + scatter
+    ProfScope ps(2);
+    if (!multi) {
+        for (auto* r : regs)
+            for (int li = 0; li < S.V; ++li) {
+                k::PtrList dl{};
+                for (int h = 0; h < S.V; ++h)
+                    if (h != li) dl.p[dl.n++] = r->dev[h];
+                CUDA_TRY(k::scatter_packed(r->trk[li].packed, r->trk[li].n_runs, dl, (int)r->esize, S.scratch, S.stream,
+                                           &S.st.kernel_launches));
+            }
+        return 0;
+    }
+    // receive every packet that comes from another process (or, in NCCL_ALL mode, from anyone) once
+    int64_t need = 0;
+    std::vector<int64_t> roff(S.P * regs.size(), -1);
+    for (size_t ri = 0; ri < regs.size(); ++ri)
+        for (int g = 0; g < S.P; ++g) {
+            if (local(g) && !S.nccl_all) continue;
+            roff[ri * S.P + g] = need;
+            need += (16 + 16 * runs[ri * S.P + g] + regs[ri]->esize * elems[ri * S.P + g] + 255) / 256 * 256;
+        }
+    TRY(ensure_recv(need));
+    NCCL_TRY(S.nccl->GroupStart());
+    for (size_t ri = 0; ri < regs.size(); ++ri)
+        for (int g = 0; g < S.P; ++g) {
+            const size_t nb = (size_t)(16 + 16 * runs[ri * S.P + g] + regs[ri]->esize * elems[ri * S.P + g]);
+            if (local(g))
+                for (int q = 0; q < S.W; ++q)
+                    if (q != S.rank || S.nccl_all)
+                        NCCL_TRY(S.nccl->Send(regs[ri]->trk[lidx(g)].packed, nb, ncclUint8, q, S.comm, S.stream));
+            if (roff[ri * S.P + g] >= 0)
+                NCCL_TRY(S.nccl->Recv(S.recv + roff[ri * S.P + g], nb, ncclUint8, rank_of(g), S.comm, S.stream));
+        }
+    NCCL_TRY(S.nccl->GroupEnd());
+    for (size_t ri = 0; ri < regs.size(); ++ri) {
+        accmg_region_s* r = regs[ri];
+        for (int g = 0; g < S.P; ++g) {
+            k::PtrList dl{};
+            for (int h = 0; h < S.V; ++h)
+                if (first_local() + h != g) dl.p[dl.n++] = r->dev[h];
+            const uint8_t* src = roff[ri * S.P + g] >= 0 ? S.recv + roff[ri * S.P + g] : r->trk[lidx(g)].packed;
+            if (roff[ri * S.P + g] < 0 && !local(g)) continue;
+            CUDA_TRY(k::scatter_packed(src, runs[ri * S.P + g], dl, (int)r->esize, S.scratch, S.stream,
+                                       &S.st.kernel_launches));
+        }
+    }
+    return 0;
+}
+
+// ---- reductiontoarray merge (L112: block -> GPU -> across GPUs) ------------------------------------
+int merge_reduce(accmg_region_s* r) {
+    ProfScope ps(2);
+    k::PtrList src{};
+    for (int li = 1; li < S.V; ++li) src.p[src.n++] = r->partial[li];
+    CUDA_TRY(k::reduce_sum_i64(r->partial[0], src, r->extent, S.stream, &S.st.kernel_launches));
+    if (S.W > 1 || S.nccl_all)
+        NCCL_TRY(S.nccl->AllReduce(r->partial[0], r->partial[0], (size_t)r->extent, ncclInt64, ncclSum, S.comm, S.stream));
+    k::PtrList dl{};
+    for (int li = 0; li < S.V; ++li) dl.p[dl.n++] = r->dev[li];
+    CUDA_TRY(k::apply_add_i64(dl, r->partial[0], r->extent, S.stream, &S.st.kernel_launches));
+    return 0;
+}
+
+// Device-side precondition failures of bodies (d_flag[1]) surface at the next synchronising call.
+int check_data_flag() {
+    if (S.dry) return 0;
+    CUDA_TRY(cudaMemcpyAsync(S.h_pin, S.d_flag, 2 * sizeof(int), cudaMemcpyDeviceToHost, S.stream));
+    CUDA_TRY(cudaStreamSynchronize(S.stream));
+    if (((int*)S.h_pin)[1]) {
+        CUDA_TRY(cudaMemsetAsync(S.d_flag + 1, 0, sizeof(int), S.stream));
+        return fail(ACCMG_EDATA, "kmeans: a point is not on the 2^-shift fixed-point grid (|x*2^shift| < 2^31)", false);
+    }
+    return 0;
+}
+
+void free_region(accmg_region_s* r) {
+    if (!S.dry) {
+        cudaStreamSynchronize(S.stream);
+        for (auto p : r->dev) dfree(p, r->extent * r->esize, false);
+        for (auto& t : r->trk) {
+            dfree(t.l1, t.nwords * 4, true);
+            dfree(t.l2, t.nl2 * 4, true);
+            dfree(t.tile_counts, t.ntiles * 24, true);
+            dfree(t.tile_offs, t.ntiles * 24, true);
+            dfree(t.tile_edges, t.ntiles * 8, true);
+            dfree(t.totals, 64, true);
+            dfree(t.packed, t.packed_cap, true);
+            dfree(t.snap_l1, t.nwords * 4, true);
+            dfree(t.snap_l2, t.nl2 * 4, true);
+        }
+        for (auto p : r->partial) dfree(p, r->extent * 8, true);
+    }
+    delete r;
+}
+
+}  // namespace
+
+// =================================================================================================
+extern "C" {
+
+int accmg_nccl_unique_id(uint8_t out[128]) {
+    if (!out) return fail(ACCMG_EINVAL, "nccl_unique_id: null", false);
+    const char* why = nullptr;
+    accmg::NcclApi* n = accmg::nccl_api(&why);
+    if (!n) return fail(ACCMG_ENCCL, why ? why : "NCCL unavailable", false);
+    ncclUniqueId id;
+    ncclResult_t r = n->GetUniqueId(&id);
+    if (r != ncclSuccess) return fail(ACCMG_ENCCL, n->GetErrorString(r), false);
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+    std::memcpy(out, &id, 128);
+    return 0;
+}
+
+int accmg_init(const accmg_config* cfg) {
+    if (S.init) return fail(ACCMG_ESTATE, "init: already initialised", false);
+    if (!cfg) return fail(ACCMG_EINVAL, "init: null config", false);
+    const accmg_config c = *cfg;
+    if (c.world_size < 1 || c.rank < 0 || c.rank >= c.world_size) return fail(ACCMG_EINVAL, "init: bad world_size/rank", false);
+    if (c.num_partitions < 1 || c.num_partitions % c.world_size != 0)
+        return fail(ACCMG_EINVAL, "init: num_partitions must be a positive multiple of world_size", false);
+    if (c.num_partitions > 64) return fail(ACCMG_EUNSUPPORTED, "init: at most 64 partitions", false);
+    int64_t cb = c.dirty_chunk_bytes ? c.dirty_chunk_bytes : (1 << 20);
+    if (cb < 256 || (cb & (cb - 1))) return fail(ACCMG_EINVAL, "init: dirty_chunk_bytes must be a power of two >= 256", false);
+    if (c.exchange_mode != ACCMG_XCHG_AUTO && c.exchange_mode != ACCMG_XCHG_NCCL_ALL)
+        return fail(ACCMG_EINVAL, "init: bad exchange_mode", false);
+    S = State();
+    S.cfg = c;
+    S.P = c.num_partitions;
+    S.W = c.world_size;
+    S.rank = c.rank;
+    S.V = S.P / S.W;
+    S.dry = c.device < 0;
+    S.nccl_all = c.exchange_mode == ACCMG_XCHG_NCCL_ALL;
+    S.chunk_bytes = cb;
+    if (S.dry) {
+        S.init = true;
+        return 0;
+    }
+    CUDA_TRY(cudaSetDevice(c.device));
+    CUDA_TRY(cudaStreamCreateWithFlags(&S.stream, cudaStreamNonBlocking));
+    TRY(dmalloc((void**)&S.scratch, 2 * k::kScatterBlocks * 8, true));
+    TRY(dmalloc((void**)&S.d_sizes, (size_t)4 * 8 * 16 * S.P * (S.W + 1), true));
+    TRY(dmalloc((void**)&S.d_flag, 16, true));
+    CUDA_TRY(cudaHostAlloc((void**)&S.h_pin, (size_t)4 * 8 * 16 * S.P * (S.W + 1) + 64, cudaHostAllocDefault));
+    CUDA_TRY(cudaMemsetAsync(S.d_flag, 0, 16, S.stream));
+    if (S.W > 1 || S.nccl_all) {
+        const char* why = nullptr;
+        S.nccl = accmg::nccl_api(&why);
+        if (!S.nccl) return fail(ACCMG_ENCCL, why ? why : "NCCL unavailable", true);
+        ncclUniqueId id;
+        if (S.W == 1) NCCL_TRY(S.nccl->GetUniqueId(&id));
+        else std::memcpy(&id, c.nccl_unique_id, 128);
+        NCCL_TRY(S.nccl->CommInitRank(&S.comm, S.W, id, S.rank));
+    }
+    S.init = true;
+    return 0;
+}
+
+int accmg_finalize(void) {
+    if (!S.init) return fail(ACCMG_ESTATE, "finalize: not initialised", false);
+    if (!S.dry) {
+        cudaSetDevice(S.cfg.device);
+        cudaStreamSynchronize(S.stream);
+    }
+    for (auto* r : S.regions) free_region(r);
+    S.regions.clear();
+    if (!S.dry) {
+        dfree(S.scratch, 0, true);
+        dfree(S.d_sizes, 0, true);
+        dfree(S.d_flag, 0, true);
+        dfree(S.recv, 0, true);
+        if (S.h_pin) cudaFreeHost(S.h_pin);
+        for (auto& p : S.prof) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
+        for (auto e : S.ev_free) cudaEventDestroy(e);
+        if (S.comm) S.nccl->CommDestroy(S.comm);
+        if (S.stream) cudaStreamDestroy(S.stream);
+    }
+    S = State();
+    return 0;
+}
+
+int accmg_region_create(void* host_array, size_t elem_size, int64_t extent, accmg_region* out) {
+    GUARD();
+    if (!host_array || !out || extent < 1) return fail(ACCMG_EINVAL, "region_create: null pointer or extent < 1", false);
+    if (elem_size != 1 && elem_size != 2 && elem_size != 4 && elem_size != 8)
+        return fail(ACCMG_EINVAL, "region_create: elem_size must be 1, 2, 4 or 8", false);
+    auto* r = new accmg_region_s();
+    r->id = S.next_id++;
+    r->host = static_cast<uint8_t*>(host_array);
+    r->esize = (int64_t)elem_size;
+    r->extent = extent;
+    r->valid.assign(S.P, IntervalSet());
+    r->host_valid = IntervalSet(0, extent);
+    r->trk.assign(S.V, Trk());
+    r->dev.assign(S.V, nullptr);
+    r->partial.assign(S.V, nullptr);
+    if (!S.dry) {
+        for (int li = 0; li < S.V; ++li) {
+            int rc = dmalloc((void**)&r->dev[li], (size_t)(extent * elem_size), false);
+            if (rc) {
+                free_region(r);
+                return rc;
+            }
+        }
+    }
+    S.regions.push_back(r);
+    *out = r;
+    return 0;
+}
+
+int accmg_region_destroy(accmg_region r) {
+    GUARD();
+    auto it = std::find(S.regions.begin(), S.regions.end(), r);
+    if (it == S.regions.end()) return fail(ACCMG_EINVAL, "region_destroy: unknown region", false);
+    S.regions.erase(it);
+    free_region(r);
+    return 0;
+}
+
+int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_access* descs, int n_descs,
+                      const void* args, size_t args_bytes) {
+    GUARD();
+    if (!bounds || !descs || !args) return fail(ACCMG_EINVAL, "loop_launch: null argument", false);
+    if (n_descs < 1 || n_descs > 16) return fail(ACCMG_EINVAL, "loop_launch: n_descs must be 1..16", false);
+    BodySpec spec;
+    if (!body_spec(body_id, &spec)) return fail(ACCMG_EINVAL, "loop_launch: unknown body_id", false);
+    if (args_bytes != spec.args) return fail(ACCMG_EINVAL, "loop_launch: args_bytes does not match the body", false);
+    if (bounds->ndim != spec.ndim) return fail(ACCMG_EINVAL, "loop_launch: wrong bounds.ndim for the body", false);
+    for (int i = 0; i < bounds->ndim; ++i)
+        if (bounds->hi[i] < bounds->lo[i]) return fail(ACCMG_EINVAL, "loop_launch: bounds hi < lo", false);
+    if (n_descs != spec.n) return fail(ACCMG_EINVAL, "loop_launch: wrong number of descriptors for the body", false);
+    for (int i = 0; i < n_descs; ++i) {
+        const accmg_access& d = descs[i];
+        if (std::find(S.regions.begin(), S.regions.end(), d.region) == S.regions.end())
+            return fail(ACCMG_EINVAL, "loop_launch: descriptor " + std::to_string(i) + " has an unknown region", false);
+        if (d.mode != spec.mode[i]) return fail(ACCMG_EINVAL, "loop_launch: descriptor " + std::to_string(i) + " has the wrong mode", false);
+        if (d.region->esize != spec.esize[i])
+            return fail(ACCMG_EINVAL, "loop_launch: descriptor " + std::to_string(i) + " has the wrong element size", false);
+        if (d.declared && (d.stride <= 0 || d.left < 0 || d.right < 0))
+            return fail(ACCMG_EINVAL, "loop_launch: declared window needs stride > 0, left/right >= 0", false);
+        if (d.mode == ACCMG_REDUCE_SUM && d.declared)
+            return fail(ACCMG_EINVAL, "loop_launch: REDUCE_SUM destinations are replicated (declared = 0)", false);
+        for (int j = 0; j < i; ++j)
+            if (descs[j].region == d.region) return fail(ACCMG_EINVAL, "loop_launch: a region appears twice", false);
+    }
+    TRY(validate_body(bounds, body_id, descs, args));
+
+    // 1. task mapping (L108)
+    std::vector<int64_t> ca(S.P), cb(S.P);
+    for (int g = 0; g < S.P; ++g) chunk_of(bounds->lo[0], bounds->hi[0], S.P, g, &ca[g], &cb[g]);
+    // 2. needs per descriptor: declared window (distribution) or whole array (replica)
+    std::vector<std::vector<IntervalSet>> need(n_descs, std::vector<IntervalSet>(S.P));
+    for (int i = 0; i < n_descs; ++i)
+        for (int g = 0; g < S.P; ++g)
+            need[i][g] = descs[i].declared ? window(descs[i], ca[g], cb[g], descs[i].region->extent)
+                                           : IntervalSet(0, descs[i].region->extent);
+    // owner computes: declared write windows must not overlap (G14)
+    for (int i = 0; i < n_descs; ++i)
+        if (descs[i].declared && (descs[i].mode & ACCMG_W))
+            for (int g = 0; g < S.P; ++g)
+                for (int h = 0; h < g; ++h)
+                    if (need[i][g].overlaps(need[i][h]))
+                        return fail(ACCMG_ECONFLICT, "declared write windows of two partitions overlap (G14)", false);
+    // 3. data loader: plan all pulls from the pre-phase state, then run them
+    std::vector<Xfer> xs;
+    for (int i = 0; i < n_descs; ++i) plan_pulls(descs[i].region, need[i], xs);
+    TRY(run_xfers(xs));
+    for (int i = 0; i < n_descs; ++i)
+        for (int g = 0; g < S.P; ++g) descs[i].region->valid[g].add(need[i][g]);
+
+    std::vector<bool> tracked(n_descs, false);
+    std::vector<accmg_region_s*> tracked_regs;
+    for (int i = 0; i < n_descs; ++i)
+        if ((descs[i].mode & ACCMG_W) && descs[i].mode != ACCMG_REDUCE_SUM && !descs[i].declared) {
+            tracked[i] = true;
+            tracked_regs.push_back(descs[i].region);
+        }
+    if (!S.dry) {
+        for (auto* r : tracked_regs)
+            for (int li = 0; li < S.V; ++li) TRY(ensure_trk(r, li));
+        for (int i = 0; i < n_descs; ++i)
+            if (descs[i].mode == ACCMG_REDUCE_SUM) {
+                accmg_region_s* r = descs[i].region;
+                for (int li = 0; li < S.V; ++li) {
+                    if (!r->partial[li]) TRY(dmalloc((void**)&r->partial[li], r->extent * 8, true));
+                    CUDA_TRY(cudaMemsetAsync(r->partial[li], 0, r->extent * 8, S.stream));
+                }
+            }
+        // 4. bodies on this process's partitions
+        {
+            ProfScope ps(0);
+            for (int li = 0; li < S.V; ++li) {
+                const int g = first_local() + li;
+                if (cb[g] > ca[g]) TRY(launch_body(body_id, bounds, descs, args, g, ca[g], cb[g], tracked));
+            }
+        }
+        // 5. coherence
+        if (!tracked_regs.empty()) TRY(propagate_dirty(tracked_regs));
+        for (int i = 0; i < n_descs; ++i)
+            if (descs[i].mode == ACCMG_REDUCE_SUM) TRY(merge_reduce(descs[i].region));
+    }
+    for (int i = 0; i < n_descs; ++i) {
+        accmg_region_s* r = descs[i].region;
+        if (descs[i].mode == ACCMG_REDUCE_SUM) {
+            S.st.bytes_reduce += 2 * (int64_t)(S.P - 1) * r->extent * 8;
+            S.st.bytes_interpartition += 2 * (int64_t)(S.P - 1) * r->extent * 8;
+            r->host_valid.clear();
+        } else if (descs[i].mode & ACCMG_W) {
+            if (descs[i].declared) {
+                // the writer becomes the only holder of its write window
+                for (int g = 0; g < S.P; ++g)
+                    for (int h = 0; h < S.P; ++h)
+                        if (h != g) r->valid[h].subtract(need[i][g]);
+                for (int g = 0; g < S.P; ++g) r->host_valid.subtract(need[i][g]);
+            } else {
+                r->host_valid.clear();  // any element may have changed; every replica is coherent again
+            }
+        }
+    }
+    S.st.loops += 1;
+    return 0;
+}
+
+static int sync_host_impl(accmg_region r, bool owned) {
+    GUARD();
+    if (std::find(S.regions.begin(), S.regions.end(), r) == S.regions.end())
+        return fail(ACCMG_EINVAL, "sync_to_host: unknown region", false);
+    if (!owned && S.W > 1) {
+        // make this process's first partition hold everything no local partition holds
+        std::vector<IntervalSet> need(S.P);
+        for (int q = 0; q < S.W; ++q) {
+            IntervalSet held;
+            for (int li = 0; li < S.V; ++li) held.add(r->valid[q * S.V + li]);
+            IntervalSet m(0, r->extent);
+            m.subtract(held);
+            need[q * S.V].add(m);
+            need[q * S.V].add(r->valid[q * S.V]);
+        }
+        std::vector<Xfer> xs;
+        plan_pulls(r, need, xs);
+        TRY(run_xfers(xs));
+        for (int g = 0; g < S.P; ++g) r->valid[g].add(need[g]);
+    }
+    TRY(check_data_flag());
+    IntervalSet todo(0, r->extent);
+    todo.subtract(r->host_valid);
+    // full: copy each missing piece from the lowest-index local holder;
+    // owned: only pieces whose lowest-index holder overall is local
+    for (int g = 0; g < S.P && !todo.empty(); ++g) {
+        if (!owned && !local(g)) continue;
+        IntervalSet piece = todo.intersect(r->valid[g]);
+        todo.subtract(piece);
+        if (!local(g)) continue;
+        for (auto& iv : piece.items()) {
+            const int64_t off = iv.lo * r->esize, nb = (iv.hi - iv.lo) * r->esize;
+            S.st.bytes_d2h += nb;
+            if (!S.dry)
+                CUDA_TRY(cudaMemcpyAsync(r->host + off, r->dev[lidx(g)] + off, (size_t)nb, cudaMemcpyDeviceToHost, S.stream));
+            r->host_valid.add(iv.lo, iv.hi);
+        }
+    }
+    if (!S.dry) CUDA_TRY(cudaStreamSynchronize(S.stream));
+    if (!owned && !todo.empty()) return fail(ACCMG_ESTATE, "sync_to_host: range valid nowhere", false);
+    return 0;
+}
+
+int accmg_sync_to_host(accmg_region r) { return sync_host_impl(r, false); }
+int accmg_sync_to_host_owned(accmg_region r) { return sync_host_impl(r, true); }
+
+int accmg_barrier(void) {
+    GUARD();
+    if (!S.dry) CUDA_TRY(cudaStreamSynchronize(S.stream));
+    return check_data_flag();
+}
+
+int accmg_get_stats(accmg_stats* out) {
+    GUARD();
+    if (!out) return fail(ACCMG_EINVAL, "get_stats: null", false);
+    if (!S.dry) {
+        TRY(collect_prof());
+        TRY(check_data_flag());
+    }
+    *out = S.st;
+    return 0;
+}
+
+int accmg_reset_stats(void) {
+    GUARD();
+    if (!S.dry) TRY(collect_prof());
+    const int64_t u = S.st.device_bytes_user, sy = S.st.device_bytes_system;
+    S.st = accmg_stats{};
+    S.st.device_bytes_user = u;
+    S.st.device_bytes_system = sy;
+    return 0;
+}
+
+const char* accmg_last_error(void) { return S.err.c_str(); }
+
+void* accmg_stream(void) { return S.init ? (void*)S.stream : nullptr; }
+
+int accmg_chunk(int64_t lo, int64_t hi, int num_partitions, int partition, int64_t* a, int64_t* b) {
+    if (!a || !b || num_partitions < 1 || partition < 0 || partition >= num_partitions || hi < lo)
+        return fail(ACCMG_EINVAL, "chunk: bad arguments", false);
+    chunk_of(lo, hi, num_partitions, partition, a, b);
+    return 0;
+}
+
+static int debug_region(accmg_region r, int partition, Trk** t) {
+    GUARD();
+    if (S.dry) return fail(ACCMG_ESTATE, "debug: not available in dry-run mode", false);
+    if (std::find(S.regions.begin(), S.regions.end(), r) == S.regions.end())
+        return fail(ACCMG_EINVAL, "debug: unknown region", false);
+    if (partition < 0 || partition >= S.P || !local(partition))
+        return fail(ACCMG_EINVAL, "debug: partition does not live on this process", false);
+    *t = &r->trk[lidx(partition)];
+    return 0;
+}
+
+int accmg_debug_dirty_bitmap(accmg_region r, int partition, uint32_t* out_words, int64_t nwords) {
+    Trk* t;
+    TRY(debug_region(r, partition, &t));
+    if (!t->has_snap) return fail(ACCMG_ESTATE, "debug: no bitmap snapshot (needs debug_checks=1 and an undeclared write)", false);
+    if (!out_words || nwords != t->nwords) return fail(ACCMG_EINVAL, "debug: nwords must be ceil(extent/32)", false);
+    CUDA_TRY(cudaMemcpyAsync(out_words, t->snap_l1, nwords * 4, cudaMemcpyDeviceToHost, S.stream));
+    CUDA_TRY(cudaStreamSynchronize(S.stream));
+    return 0;
+}
+
+int accmg_debug_chunk_bits(accmg_region r, int partition, uint32_t* out_words, int64_t nwords) {
+    Trk* t;
+    TRY(debug_region(r, partition, &t));
+    if (!t->has_snap) return fail(ACCMG_ESTATE, "debug: no bitmap snapshot (needs debug_checks=1 and an undeclared write)", false);
+    if (!out_words || nwords != t->nl2) return fail(ACCMG_EINVAL, "debug: wrong chunk-bit word count", false);
+    CUDA_TRY(cudaMemcpyAsync(out_words, t->snap_l2, nwords * 4, cudaMemcpyDeviceToHost, S.stream));
+    CUDA_TRY(cudaStreamSynchronize(S.stream));
+    return 0;
+}
+
+int accmg_debug_packed(accmg_region r, int partition, void* out, int64_t cap, int64_t* used) {
+    Trk* t;
+    TRY(debug_region(r, partition, &t));
+    if (!t->has_packed) return fail(ACCMG_ESTATE, "debug: no packed buffer yet", false);
+    if (used) *used = t->packed_bytes;
+    if (out && cap > 0) {
+        CUDA_TRY(cudaMemcpyAsync(out, t->packed, (size_t)std::min(cap, t->packed_bytes), cudaMemcpyDeviceToHost, S.stream));
+        CUDA_TRY(cudaStreamSynchronize(S.stream));
+    }
+    return 0;
+}
+
+int accmg_debug_replica(accmg_region r, int partition, void* out) {
+    Trk* t;
+    TRY(debug_region(r, partition, &t));
+    if (!out) return fail(ACCMG_EINVAL, "debug: null", false);
+    CUDA_TRY(cudaMemcpyAsync(out, r->dev[lidx(partition)], (size_t)(r->extent * r->esize), cudaMemcpyDeviceToHost, S.stream));
+    CUDA_TRY(cudaStreamSynchronize(S.stream));
+    return 0;
+}
+
+int accmg_debug_valid(accmg_region r, int partition, int64_t* out_pairs, int64_t cap, int64_t* n) {
+    if (S.sticky) return S.sticky;
+    if (!S.init) return fail(ACCMG_ESTATE, "accmg: not initialised", false);
+    if (std::find(S.regions.begin(), S.regions.end(), r) == S.regions.end())
+        return fail(ACCMG_EINVAL, "debug: unknown region", false);
+    if (partition < -1 || partition >= S.P) return fail(ACCMG_EINVAL, "debug: bad partition", false);
+    const IntervalSet& v = partition < 0 ? r->host_valid : r->valid[partition];
+    if (n) *n = (int64_t)v.items().size();
+    for (int64_t i = 0; i < cap && i < (int64_t)v.items().size(); ++i) {
+        out_pairs[2 * i] = v.items()[i].lo;
+        out_pairs[2 * i + 1] = v.items()[i].hi;
+    }
+    return 0;
+}
+
+}  // extern "C"

@@ -1,0 +1,87 @@
+// Fused write-tracking epilogue (north star (3); paper L110, L133-135 §IV.D.1): "the translator
+// inserts the additional operations to turn on the dirty bits for every writes accesses to the
+// replicated arrays", with a second-level bit per constant-size chunk.
+//
+// Warp-aggregated: a warp that wrote a contiguous span of 32*VEC elements (lane l owns elements
+// E0 + VEC*l + k, k < VEC, written iff bit k of its mask) builds the span's bit pattern with
+// VEC ballots, shifts it onto the absolute uint32 words and issues at most VEC+1 atomicOr
+// (one per touched word) instead of one per element. Every written element sets its bit
+// (also when the value is unchanged, reading G12); no bit is ever dropped because concurrent
+// writers of a word combine through atomicOr.
+#pragma once
+#include <cstdint>
+
+namespace accmg {
+namespace dev {
+
+constexpr unsigned kFull = 0xffffffffu;
+
+// bit m of an 8-bit value -> bit 4m
+__device__ __forceinline__ uint32_t spread4(uint32_t x) {
+    x &= 0xffu;
+    x = (x | (x << 12)) & 0x000F000Fu;
+    x = (x | (x << 6)) & 0x03030303u;
+    x = (x | (x << 3)) & 0x11111111u;
+    return x;
+}
+
+// Sets the L2 (chunk) bits of elements [first, last] (inclusive, all written). `cache` holds the
+// last chunk this warp marked so steady marching re-issues nothing.
+__device__ __forceinline__ void track_l2(uint32_t* l2, int l2_shift, int64_t first, int64_t last, int64_t& cache) {
+    int64_t c0 = first >> l2_shift, c1 = last >> l2_shift;
+    if (c0 == c1 && c0 == cache) return;
+    for (int64_t c = c0; c <= c1; ++c) atomicOr(l2 + (c >> 5), 1u << (c & 31));
+    cache = c1;
+}
+
+// VEC = 4: lane l owns elements E0 + 4l + k (k < 4), written iff (nib >> k) & 1.
+// VEC = 1: lane l owns element E0 + l, written iff nib & 1.
+// Must be called by all 32 lanes of the warp (warp-uniform E0).
+template <int VEC>
+__device__ __forceinline__ void track_warp(uint32_t* __restrict__ l1, uint32_t* __restrict__ l2, int l2_shift,
+                                           int64_t E0, unsigned nib, int64_t& l2_cache) {
+    const int lane = threadIdx.x & 31;
+    uint32_t rel[VEC];
+    if (VEC == 4) {
+        uint32_t b0 = __ballot_sync(kFull, nib & 1u), b1 = __ballot_sync(kFull, nib & 2u);
+        uint32_t b2 = __ballot_sync(kFull, nib & 4u), b3 = __ballot_sync(kFull, nib & 8u);
+        if ((b0 | b1 | b2 | b3) == 0u) return;
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) {
+            int sh = 8 * q;
+            rel[q] = spread4(b0 >> sh) | (spread4(b1 >> sh) << 1) | (spread4(b2 >> sh) << 2) |
+                     (spread4(b3 >> sh) << 3);
+        }
+    } else {
+        rel[0] = __ballot_sync(kFull, nib & 1u);
+        if (rel[0] == 0u) return;
+    }
+    const int s = (int)(E0 & 31);
+    const int64_t w0 = E0 >> 5;
+    // absolute word q (0..VEC) of the span
+    if (lane <= VEC) {
+        uint32_t lo = 0u, hi = 0u;  // rel[lane], rel[lane-1] without dynamic register indexing
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) {
+            lo = (q == lane) ? rel[q] : lo;
+            hi = (q == lane - 1) ? rel[q] : hi;
+        }
+        uint32_t v = (lo << s) | (s ? (hi >> (32 - s)) : 0u);
+        if (v) atomicOr(l1 + w0 + lane, v);
+    }
+    if (lane == 0) {
+        // first and last written element of the span
+        int f = -1, l = -1;
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) {
+            if (rel[q]) {
+                if (f < 0) f = 32 * q + __ffs(rel[q]) - 1;
+                l = 32 * q + 31 - __clz(rel[q]);
+            }
+        }
+        track_l2(l2, l2_shift, E0 + f, E0 + l, l2_cache);
+    }
+}
+
+}  // namespace dev
+}  // namespace accmg

@@ -1,0 +1,85 @@
+"""Drivers of the paper's workload loops through the C ABI (configs C1-C5 of BASELINE.json).
+
+Each driver issues the same sequence of accmg_* calls an OpenACC program annotated with the
+paper's directives would make (L81-93 §III.C): regions = data-region arrays, one
+accmg_loop_launch per `parallel loop`, declared windows = `localaccess`, REDUCE_SUM =
+`reductiontoarray`. Pure marshalling: all computation happens in libaccmg.so.
+"""
+from __future__ import annotations
+
+import numpy as np
+
+from . import accmg as A
+
+
+def jacobi_descs(src, dst, N: int, declared: bool):
+    """`localaccess` of the 5-point stencil on row-major N x N: iteration i reads rows i-1..i+1
+    (stride N, left = right = N) and writes row i (stride N) — L87 with reading G23."""
+    return [A.access(src, A.R, declared, N, N, N), A.access(dst, A.W, declared, N, 0, 0)]
+
+
+def jacobi_sweep(rA, rB, s: int, N: int, declared: bool) -> None:
+    src, dst = (rA, rB) if s % 2 == 0 else (rB, rA)
+    A.accmg_loop_launch(A.bounds([1, 1], [N - 1, N - 1]), A.BODY_JACOBI2D_5PT, jacobi_descs(src, dst, N, declared),
+                        A.accmg_args_jacobi2d(N, N))
+
+
+def jacobi_run(Ahost: np.ndarray, Bhost: np.ndarray, sweeps: int, declared: bool = True, per_loop_stats: bool = False):
+    """S sweeps A -> B -> A ... on an initialised runtime; host arrays are updated at the end.
+    Returns the list of per-loop stats deltas if per_loop_stats."""
+    N = Ahost.shape[0]
+    rA, rB = A.accmg_region_create(Ahost), A.accmg_region_create(Bhost)
+    per = []
+    try:
+        prev = A.accmg_get_stats() if per_loop_stats else None
+        for s in range(sweeps):
+            jacobi_sweep(rA, rB, s, N, declared)
+            if per_loop_stats:
+                cur = A.accmg_get_stats()
+                per.append({k: cur[k] - prev[k] for k in cur})
+                prev = cur
+        A.accmg_sync_to_host(rA)
+        A.accmg_sync_to_host(rB)
+    finally:
+        A.accmg_region_destroy(rA)
+        A.accmg_region_destroy(rB)
+    return per
+
+
+def kmeans_loops(rx, rcen, rmem, rsum, rcnt, n: int, d: int, k: int, shift: int = 8) -> None:
+    """One k-means iteration = the paper's 2 parallel loops (Table II: KMEANS has 2 loops)."""
+    args = A.accmg_args_kmeans(n, d, k, shift, 0)
+    A.accmg_loop_launch(A.bounds([0], [n]), A.BODY_KMEANS_ASSIGN,
+                        [A.access(rx, A.R, True, d, 0, 0), A.access(rcen, A.R), A.access(rmem, A.W, True, 1, 0, 0),
+                         A.access(rsum, A.REDUCE_SUM), A.access(rcnt, A.REDUCE_SUM)], args)
+    A.accmg_loop_launch(A.bounds([0], [k]), A.BODY_KMEANS_UPDATE,
+                        [A.access(rsum, A.RW), A.access(rcnt, A.RW), A.access(rcen, A.W)], args)
+
+
+def kmeans_run(x: np.ndarray, k: int, iters: int, shift: int = 8):
+    """Rodinia-style k-means (centroids start at the first k points). Returns (centroids, member)."""
+    n, d = x.shape
+    cen = np.ascontiguousarray(x[:k]).copy()
+    member = np.zeros(n, dtype=np.int32)
+    sums = np.zeros((k, d), dtype=np.int64)
+    cnt = np.zeros(k, dtype=np.int64)
+    regs = [A.accmg_region_create(a) for a in (x, cen, member, sums, cnt)]
+    try:
+        for _ in range(iters):
+            kmeans_loops(*regs, n, d, k, shift)
+        A.accmg_sync_to_host(regs[1])
+        A.accmg_sync_to_host(regs[2])
+    finally:
+        for r in regs:
+            A.accmg_region_destroy(r)
+    return cen, member
+
+
+def gemm_descs(rA, rB, rC, M: int, N: int, K: int):
+    """A rows declared (stride K), B replicated (no localaccess), C row-block writes (stride N)."""
+    return [A.access(rA, A.R, True, K, 0, 0), A.access(rB, A.R), A.access(rC, A.W, True, N, 0, 0)]
+
+
+def gemm_loop(rA, rB, rC, M: int, N: int, K: int) -> None:
+    A.accmg_loop_launch(A.bounds([0, 0], [M, N]), A.BODY_GEMM_BF16_F32, gemm_descs(rA, rB, rC, M, N, K),
+                        A.accmg_args_gemm(M, N, K))

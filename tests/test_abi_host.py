@@ -1,0 +1,174 @@
+"""C-ABI library on the CPU: it loads, exports every entry point of include/accmg.h, and its host
+logic (task mapping, window/pull planning, validity table, byte accounting, argument checks) —
+run in dry-run mode (device = -1: no CUDA call, no body) — matches the oracle's brute-force
+coherence model element by element. No GPU needed."""
+import numpy as np
+import pytest
+
+import oracle
+from oracle import model as M
+from paper_conf_icpp_komodamnm13_b200 import accmg as A
+from paper_conf_icpp_komodamnm13_b200 import workloads as WL
+
+
+@pytest.fixture
+def dry():
+    def start(P, **kw):
+        A.accmg_init(num_partitions=P, device=-1, **kw)
+    yield start
+    try:
+        A.accmg_finalize()
+    except A.AccmgError:
+        pass
+
+
+def test_exports_every_header_symbol():
+    syms = A.header_symbols()
+    assert len(syms) >= 19
+    for s in syms:
+        assert hasattr(A._lib, s), s
+
+
+def test_chunk_matches_oracle_partition():
+    for P in range(1, 10):
+        for n in range(0, 40):
+            for g in range(P):
+                assert A.accmg_chunk(3, 3 + n, P, g) == oracle.partition(3, 3 + n, P, g)
+
+
+def _intervals(mask):
+    m = np.concatenate(([0], mask.astype(np.int8), [0]))
+    d = np.diff(m)
+    return list(zip(np.flatnonzero(d == 1).tolist(), np.flatnonzero(d == -1).tolist()))
+
+
+def _compare_valid(regs_c, regs_m, P):
+    for rc, rm in zip(regs_c, regs_m):
+        for g in range(P):
+            assert A.accmg_debug_valid(rc, g) == _intervals(rm.valid[g]), g
+        assert A.accmg_debug_valid(rc, -1) == _intervals(rm.host_valid)
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 5, 8])
+def test_declared_jacobi_plan_vs_model(dry, P):
+    N, S = 40, 5
+    dry(P)
+    hA = np.zeros((N, N), np.float32)
+    hB = np.zeros((N, N), np.float32)
+    rA, rB = A.accmg_region_create(hA), A.accmg_region_create(hB)
+    mdl = M.Model(P)
+    mA, mB = mdl.region(N * N, 4), mdl.region(N * N, 4)
+    for s in range(S):
+        before = A.accmg_get_stats()
+        WL.jacobi_sweep(rA, rB, s, N, True)
+        after = A.accmg_get_stats()
+        src, dst = (mA, mB) if s % 2 == 0 else (mB, mA)
+        exp = mdl.loop(1, N - 1, [(src, M.R, 1, N, N, N), (dst, M.W, 1, N, 0, 0)])
+        assert after["bytes_declared"] - before["bytes_declared"] == exp["declared"]
+        assert after["bytes_h2d"] - before["bytes_h2d"] == exp["h2d"]
+        _compare_valid([rA, rB], [mA, mB], P)
+    A.accmg_sync_to_host(rA)
+    assert A.accmg_get_stats()["bytes_d2h"] == mdl.sync_to_host(mA)
+    _compare_valid([rA], [mA], P)
+
+
+@pytest.mark.parametrize("seed", range(12))
+def test_random_windows_plan_vs_model(dry, seed):
+    """Random localaccess windows (stride, left, right) over random loop bounds (L87)."""
+    rng = np.random.default_rng(seed)
+    P = int(rng.integers(1, 7))
+    rows, cols = int(rng.integers(4, 30)), int(rng.integers(3, 9))
+    dry(P)
+    h = [np.zeros(rows * cols, np.float32) for _ in range(2)]
+    rc = [A.accmg_region_create(x) for x in h]
+    mdl = M.Model(P)
+    rm = [mdl.region(rows * cols, 4) for _ in range(2)]
+    for it in range(4):
+        lo = int(rng.integers(0, 3))
+        hi = int(rng.integers(lo, rows + 1))
+        s = cols
+        l, r = int(rng.integers(0, 3 * cols)), int(rng.integers(0, 3 * cols))
+        src, dst = (0, 1) if it % 2 == 0 else (1, 0)
+        descs = [A.access(rc[src], A.R, True, s, l, r), A.access(rc[dst], A.W, True, s, 0, 0)]
+        args = A.accmg_args_sparse(rows, cols, 1)
+        before = A.accmg_get_stats()
+        A.accmg_loop_launch(A.bounds([lo], [hi]), A.BODY_TEST_SPARSE_WRITE, descs, args)
+        after = A.accmg_get_stats()
+        exp = mdl.loop(lo, hi, [(rm[src], M.R, 1, s, l, r), (rm[dst], M.W, 1, s, 0, 0)])
+        assert after["bytes_declared"] - before["bytes_declared"] == exp["declared"]
+        assert after["bytes_h2d"] - before["bytes_h2d"] == exp["h2d"]
+        _compare_valid(rc, rm, P)
+
+
+def test_c1_worked_example_dry(dry):
+    N, P = 256, 2
+    dry(P)
+    h = [np.zeros((N, N), np.float32) for _ in range(2)]
+    per = []
+    rA, rB = A.accmg_region_create(h[0]), A.accmg_region_create(h[1])
+    prev = A.accmg_get_stats()
+    for s in range(10):
+        WL.jacobi_sweep(rA, rB, s, N, True)
+        cur = A.accmg_get_stats()
+        per.append(cur["bytes_declared"] - prev["bytes_declared"])
+        prev = cur
+    assert per[0] == 0 and all(p == 2048 for p in per[2:])
+    # W_0 = [256, 32768) is owned by partition 0 after a write of the B array
+    assert A.accmg_debug_valid(rB, 0)[0][1] >= 32768
+
+
+def test_reduce_and_replica_bytes_dry(dry):
+    n, d, k, P = 1000, 16, 8, 4
+    dry(P)
+    x = np.zeros((n, d), np.float32)
+    regs = [A.accmg_region_create(a) for a in (x, np.zeros((k, d), np.float32), np.zeros(n, np.int32),
+                                                np.zeros((k, d), np.int64), np.zeros(k, np.int64))]
+    WL.kmeans_loops(*regs, n, d, k)
+    st = A.accmg_get_stats()
+    assert st["bytes_reduce"] == 2 * (P - 1) * (k * d + k) * 8
+    # x is distributed: each partition loads only its points from the host (L121-123)
+    assert st["bytes_h2d"] >= n * d * 4 and st["bytes_h2d"] < 2 * n * d * 4 + P * (k * d * 4 + 2 * (k * d + k) * 8)
+
+
+def test_argument_errors(dry):
+    dry(2)
+    N = 16
+    h = [np.zeros((N, N), np.float32) for _ in range(2)]
+    rA, rB = A.accmg_region_create(h[0]), A.accmg_region_create(h[1])
+    args = A.accmg_args_jacobi2d(N, N)
+    b = A.bounds([1, 1], [N - 1, N - 1])
+    good = WL.jacobi_descs(rA, rB, N, True)
+    with pytest.raises(A.AccmgError) as e:
+        A.accmg_loop_launch(b, 77, good, args)
+    assert e.value.code == A.EINVAL
+    with pytest.raises(A.AccmgError) as e:   # wrong mode for the body
+        A.accmg_loop_launch(b, A.BODY_JACOBI2D_5PT, [good[0], A.access(rB, A.R, True, N)], args)
+    assert e.value.code == A.EINVAL
+    with pytest.raises(A.AccmgError) as e:   # stride <= 0
+        A.accmg_loop_launch(b, A.BODY_JACOBI2D_5PT, [A.access(rA, A.R, True, 0, 0, 0), good[1]], args)
+    assert e.value.code == A.EINVAL
+    with pytest.raises(A.AccmgError) as e:   # same region twice
+        A.accmg_loop_launch(b, A.BODY_JACOBI2D_5PT, [good[0], A.access(rA, A.W, True, N)], args)
+    assert e.value.code == A.EINVAL
+    with pytest.raises(A.AccmgError) as e:   # bounds outside the interior
+        A.accmg_loop_launch(A.bounds([0, 1], [N - 1, N - 1]), A.BODY_JACOBI2D_5PT, good, args)
+    assert e.value.code == A.EINVAL
+    with pytest.raises(A.AccmgError) as e:   # overlapping declared writes (owner computes, G14)
+        A.accmg_loop_launch(b, A.BODY_JACOBI2D_5PT, [good[0], A.access(rB, A.W, True, N, N, 0)], args)
+    assert e.value.code == A.ECONFLICT
+    A.accmg_loop_launch(b, A.BODY_JACOBI2D_5PT, good, args)   # still usable (errors are not sticky)
+
+
+def test_state_errors():
+    with pytest.raises(A.AccmgError) as e:
+        A.accmg_barrier()
+    assert e.value.code == A.ESTATE
+    with pytest.raises(A.AccmgError) as e:
+        A.accmg_init(num_partitions=3, world_size=2, device=-1)
+    assert e.value.code == A.EINVAL
+    with pytest.raises(A.AccmgError) as e:
+        A.accmg_init(num_partitions=65, device=-1)
+    assert e.value.code == A.EUNSUPPORTED
+    with pytest.raises(A.AccmgError) as e:
+        A.accmg_init(num_partitions=1, device=-1, dirty_chunk_bytes=1000)
+    assert e.value.code == A.EINVAL
