@@ -1,0 +1,194 @@
+#!/usr/bin/env python3
+"""All five BASELINE.json configs on ONE B200 (bench.py is the driver's single-line C2 bench).
+
+Partitions P > 1 are virtual partitions on the one GPU (separate full-extent replicas, exchanges as
+device copies / scatter kernels), which exercises and times every coherence step of the multi-GPU
+path except the NVLink transfer itself. One JSON line per (config, P) on stdout:
+
+  python bench_configs.py --configs c1,c2,c3,c4,c5 --partitions 1,2,4,8
+
+Each line: loop iterations/s, ms per loop, per-phase CUDA-event times (body / compaction /
+exchange), inter-partition bytes per loop and the dominant kernel's roofline fraction; --check
+adds the k-means closed-form check (labels and exact means of the generated clusters). Oracle
+parity at these sizes lives in tests/test_gpu_fullsize.py (this script never loads the oracle).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import gen  # noqa: E402
+from paper_conf_icpp_komodamnm13_b200 import accmg as A  # noqa: E402
+from paper_conf_icpp_komodamnm13_b200 import workloads as WL  # noqa: E402
+
+
+def peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {"hbm_gbs": 6650.0, "bf16_tflops": 1590.0, "bf16_tflops_sustained": 1400.0}
+
+
+def emit(d):
+    print(json.dumps(d), flush=True)
+
+
+def per_loop(st, loops):
+    return {"ms_body": st["ms_body"] / loops, "ms_compact": st["ms_compact"] / loops,
+            "ms_exchange": st["ms_exchange"] / loops,
+            "bytes_interpartition": st["bytes_interpartition"] / loops,
+            "bytes_declared": st["bytes_declared"] / loops,
+            "bytes_undeclared_payload": st["bytes_undeclared_payload"] / loops,
+            "bytes_undeclared_headers": st["bytes_undeclared_headers"] / loops,
+            "bytes_paper_protocol": st["bytes_paper_protocol"] / loops,
+            "kernel_launches": st["kernel_launches"] / loops}
+
+
+def wall(fn):
+    A.accmg_barrier()
+    t0 = time.perf_counter()
+    fn()
+    A.accmg_barrier()
+    return time.perf_counter() - t0
+
+
+def jacobi_cfg(name, N, sweeps, P, declared, check):
+    Ah = gen.jacobi_field(2 if N > 256 else 1, N)
+    Bh = Ah.copy()
+    A.accmg_init(num_partitions=P, device=0, profile=1)
+    try:
+        rA, rB = A.accmg_region_create(Ah), A.accmg_region_create(Bh)
+        warm = 2
+        for s in range(warm):
+            WL.jacobi_sweep(rA, rB, s, N, declared)
+        A.accmg_barrier()
+        A.accmg_reset_stats()
+        t = wall(lambda: [WL.jacobi_sweep(rA, rB, s, N, declared) for s in range(warm, warm + sweeps)])
+        st = A.accmg_get_stats()
+        A.accmg_sync_to_host(rA)
+        A.accmg_sync_to_host(rB)
+    finally:
+        A.accmg_finalize()
+    pl = per_loop(st, sweeps)
+    body_bytes = 8 * (N - 2) * (N - 2) / P  # per partition launch
+    body_ms_launch = st["ms_body"] / max(st["body_launches"], 1)
+    out = {"config": name, "P": P, "N": N, "sweeps": sweeps, "declared": declared,
+           "iters_per_s": (N - 2) ** 2 * sweeps / t, "ms_per_loop": t / sweeps * 1e3, **pl,
+           "body_GBs": body_bytes / (body_ms_launch / 1e3) / 1e9}
+    out["body_frac_of_measured_hbm"] = out["body_GBs"] / peaks()["hbm_gbs"]
+    return out
+
+
+def gemm_cfg(N, P, reps, check):
+    pk = peaks()
+    Ab = gen.bf16_matrix(3, N, N, gen.BF16_INTS)
+    Bb = gen.bf16_matrix(4, N, N, gen.BF16_INTS)
+    C = np.zeros((N, N), dtype=np.float32)
+    A.accmg_init(num_partitions=P, device=0, profile=1)
+    try:
+        ra, rb, rc = A.accmg_region_create(Ab), A.accmg_region_create(Bb), A.accmg_region_create(C)
+        WL.gemm_loop(ra, rb, rc, N, N, N)  # warm-up (and copy-in)
+        A.accmg_barrier()
+        A.accmg_reset_stats()
+        t = wall(lambda: [WL.gemm_loop(ra, rb, rc, N, N, N) for _ in range(reps)])
+        st = A.accmg_get_stats()
+        A.accmg_sync_to_host(rc)
+    finally:
+        A.accmg_finalize()
+    flop = 2.0 * N ** 3
+    ms_launch = st["ms_body"] / max(st["body_launches"], 1)
+    out = {"config": "c3", "P": P, "N": N, "reps": reps, "iters_per_s": N * N * reps / t,
+           "ms_per_loop": t / reps * 1e3, **per_loop(st, reps),
+           "tflops": flop * reps / t / 1e12, "body_tflops_per_launch": flop / P / (ms_launch / 1e3) / 1e12}
+    out["frac_of_measured_bf16_burst"] = out["tflops"] / pk["bf16_tflops"]
+    out["frac_of_measured_bf16_sustained"] = out["tflops"] / pk.get("bf16_tflops_sustained", pk["bf16_tflops"])
+    return out
+
+
+def kmeans_cfg(n, iters, P, check):
+    d, k = 16, 256
+    t0 = time.perf_counter()
+    x, lab, _ = gen.kmeans_points(4, n, d, k, gen.KM_LATTICE, labels=True)
+    tgen = time.perf_counter() - t0
+    cen = np.ascontiguousarray(x[:k]).copy()
+    member = np.zeros(n, dtype=np.int32)
+    sums = np.zeros((k, d), dtype=np.int64)
+    cnt = np.zeros(k, dtype=np.int64)
+    A.accmg_init(num_partitions=P, device=0, profile=1)
+    try:
+        regs = [A.accmg_region_create(a) for a in (x, cen, member, sums, cnt)]
+        WL.kmeans_loops(*regs, n, d, k)  # iteration 1 (copy-in) untimed
+        A.accmg_barrier()
+        A.accmg_reset_stats()
+        t = wall(lambda: [WL.kmeans_loops(*regs, n, d, k) for _ in range(iters - 1)])
+        st = A.accmg_get_stats()
+        A.accmg_sync_to_host(regs[1])
+        A.accmg_sync_to_host(regs[2])
+    finally:
+        A.accmg_finalize()
+    its = iters - 1
+    ms_assign = st["ms_body"] / its  # body time includes the (tiny) update loop
+    lane_ops = 2.0 * n * k * d
+    out = {"config": "c4", "P": P, "n": n, "iters_timed": its, "iters_per_s": n * its / t,
+           "ms_per_iteration": t / its * 1e3, **per_loop(st, 2 * its), "gen_s": tgen,
+           "fp32_lane_ops_per_s": lane_ops / (ms_assign / 1e3)}
+    # FP32 peak at the clock: 148 SMs x 128 lanes x 2 ops (FFMA2 packs 2) per cycle
+    out["frac_of_fp32_fma_peak_1965MHz"] = out["fp32_lane_ops_per_s"] / (148 * 128 * 2 * 1.965e9)
+    if check:
+        ok = np.array_equal(member, lab)
+        # closed form: centroids are the exact means of the generated clusters
+        s = np.zeros((k, d), dtype=np.float64)
+        for c0 in range(0, n, 1 << 24):
+            c1 = min(n, c0 + (1 << 24))
+            for j in range(d):
+                s[:, j] += np.bincount(lab[c0:c1], weights=x[c0:c1, j].astype(np.float64), minlength=k)
+        c = np.bincount(lab, minlength=k).astype(np.float64)
+        ok = ok and np.array_equal(cen, (s / c[:, None]).astype(np.float32))
+        out["parity"] = "closed-form labels+means" if ok else "MISMATCH"
+    return out
+
+
+def main():
+    p = argparse.ArgumentParser()
+    p.add_argument("--configs", default="c1,c2,c5,c3,c4")
+    p.add_argument("--partitions", default="1,2,4,8")
+    p.add_argument("--sweeps", type=int, default=100)
+    p.add_argument("--c5-sweeps", type=int, default=10)
+    p.add_argument("--gemm-n", type=int, default=32768)
+    p.add_argument("--gemm-reps", type=int, default=3)
+    p.add_argument("--kmeans-n", type=int, default=1 << 28)
+    p.add_argument("--kmeans-iters", type=int, default=20)
+    p.add_argument("--check", action="store_true", help="k-means closed-form check")
+    a = p.parse_args()
+    Ps = [int(x) for x in a.partitions.split(",")]
+    for cfg in a.configs.split(","):
+        for P in Ps:
+            try:
+                if cfg == "c1":
+                    if P in (1, 2):
+                        emit(jacobi_cfg("c1", 256, 10, P, True, True))
+                elif cfg == "c2":
+                    emit(jacobi_cfg("c2", 32768, a.sweeps, P, True, a.check and P == Ps[-1]))
+                elif cfg == "c5":
+                    emit(jacobi_cfg("c5", 32768, a.c5_sweeps, P, False, a.check and P == Ps[-1]))
+                elif cfg == "c3":
+                    emit(gemm_cfg(a.gemm_n, P, a.gemm_reps, a.check))
+                elif cfg == "c4":
+                    if a.kmeans_n * 16 * 4 * P > (100 << 30):
+                        emit({"config": cfg, "P": P, "skipped": "full-extent virtual replicas would exceed 100 GiB"})
+                        continue
+                    emit(kmeans_cfg(a.kmeans_n, a.kmeans_iters, P, a.check))
+            except Exception as e:  # report and continue with the next config
+                emit({"config": cfg, "P": P, "error": repr(e)})
+
+
+if __name__ == "__main__":
+    main()
