@@ -45,9 +45,13 @@ extern "C" {
 /* ---- configuration ------------------------------------------------------------------------ */
 /* exchange_mode */
 #define ACCMG_XCHG_AUTO     0  /* same-process partitions: device copies / direct scatter;
-                                  other processes: NCCL send/recv and all-reduce over NVLink */
+                                  other processes (P2P): peers' replicas are mapped through CUDA
+                                  IPC — pulls are copy-engine reads over NVLink, dirty runs are
+                                  pushed by one scatter kernel into every replica, reductions read
+                                  all partials; a device-side flag barrier closes each loop */
 #define ACCMG_XCHG_NCCL_ALL 1  /* every inter-partition move goes through NCCL, even between
                                   partitions of one process (self send/recv) — for testing */
+#define ACCMG_XCHG_NCCL     2  /* across processes: NCCL send/recv and all-reduce */
 
 typedef struct accmg_config {
     int32_t num_partitions;    /* P, the number of tasks groups every loop is divided into (L108);
@@ -66,8 +70,10 @@ typedef struct accmg_config {
                                   debug getters; costs extra device work */
     int32_t profile;           /* 1 = time body / compaction / exchange phases with CUDA events */
     int32_t reserved;
-    uint8_t nccl_unique_id[128]; /* world_size > 1: bytes from accmg_nccl_unique_id() on rank 0,
-                                    broadcast by the caller (e.g. torch.distributed) */
+    uint8_t nccl_unique_id[128]; /* world_size > 1: the job's id, made on rank 0 by
+                                    accmg_nccl_unique_id() (NCCL modes) or accmg_unique_id() (P2P),
+                                    broadcast by the caller (e.g. torch.distributed); P2P mode names
+                                    its single-node shared-memory bootstrap after it */
 } accmg_config;
 
 /* ---- regions (device arrays) --------------------------------------------------------------- */
@@ -136,7 +142,10 @@ typedef struct { int64_t M, N, K; } accmg_args_gemm;
 typedef struct { int64_t n; int32_t d, k, shift, pad; } accmg_args_kmeans;
 typedef struct { int64_t rows, cols, period; } accmg_args_sparse;
 
-/* ---- statistics (E5-style breakdown, L188; device memory User/System, L249) ------------------ */
+/* ---- statistics (E5-style breakdown, L188; device memory User/System, L249) ------------------
+ * Byte counters are this process's: pulls into its partitions (receiver-counted), packets its
+ * partitions sent (sender-counted, x (P-1) deliveries) and its V/P share of each reduction. With one
+ * process they are the whole job's; with several, the whole job's is the sum over ranks. */
 typedef struct accmg_stats {
     int64_t loops;                    /* loop launches */
     int64_t bytes_interpartition;     /* all bytes delivered between partitions (sum of the next 4) */
@@ -159,6 +168,9 @@ typedef struct accmg_stats {
 /* Writes a fresh NCCL unique id (128 bytes) for accmg_config.nccl_unique_id. Call on rank 0 only.
    Loads NCCL (libnccl.so.2) on first use. */
 int accmg_nccl_unique_id(uint8_t out[128]);
+
+/* Writes 128 random bytes (from /dev/urandom) usable as the P2P-mode job id. Rank 0 only. */
+int accmg_unique_id(uint8_t out[128]);
 
 /* Runtime start-up (L104 "control codes to initialize the devices"): selects the device, creates
    the process's stream and (world_size > 1) the NCCL communicator. ACCMG_ESTATE if initialised. */

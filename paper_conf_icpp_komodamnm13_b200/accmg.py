@@ -22,7 +22,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 
 # ---- constants (mirrors of include/accmg.h) --------------------------------------------------
 OK, EINVAL, ECUDA, ENCCL, ENOMEM, ESTATE, EUNSUPPORTED, ECONFLICT, EDATA = 0, -1, -2, -3, -4, -5, -6, -7, -8
-XCHG_AUTO, XCHG_NCCL_ALL = 0, 1
+XCHG_AUTO, XCHG_NCCL_ALL, XCHG_NCCL = 0, 1, 2
 R, W, RW, REDUCE_SUM = 1, 2, 3, 4
 BODY_JACOBI2D_5PT, BODY_GEMM_BF16_F32, BODY_KMEANS_ASSIGN, BODY_KMEANS_UPDATE = 1, 2, 3, 4
 BODY_TEST_SPARSE_WRITE = 100
@@ -76,6 +76,7 @@ _vp, _i32, _i64, _sz = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_s
 _p64 = ctypes.POINTER(ctypes.c_int64)
 _SIGS = {
     "accmg_nccl_unique_id": [_vp],
+    "accmg_unique_id": [_vp],
     "accmg_init": [ctypes.POINTER(accmg_config)],
     "accmg_finalize": [],
     "accmg_region_create": [_vp, _sz, _i64, ctypes.POINTER(_vp)],
@@ -143,6 +144,12 @@ class Region:
 def accmg_nccl_unique_id() -> bytes:
     buf = (ctypes.c_uint8 * 128)()
     _check(_lib.accmg_nccl_unique_id(buf), "accmg_nccl_unique_id")
+    return bytes(buf)
+
+
+def accmg_unique_id() -> bytes:
+    buf = (ctypes.c_uint8 * 128)()
+    _check(_lib.accmg_unique_id(buf), "accmg_unique_id")
     return bytes(buf)
 
 

@@ -188,15 +188,24 @@ write_k(uint32_t* __restrict__ l1, int64_t nwords, const int64_t* __restrict__ t
         int64_t ks = os + is - ps, ke = oe + ie - pe;
         for (uint32_t m = sm; m; m &= m - 1) run_start[ks++] = gw * 32 + (__ffs(m) - 1);
         for (uint32_t m = em; m; m &= m - 1) run_end[ke++] = gw * 32 + __ffs(m);
-        const int64_t myel = oel + iel - pel;
-        // payload: word by word, lanes = element bits (coalesced gather and store)
-        for (int q = 0; q < 32; ++q) {
-            const uint32_t wq = __shfl_sync(dev::kFull, w, q);
-            if (wq == 0u) continue;
-            const int64_t base = __shfl_sync(dev::kFull, myel, q);
-            const int64_t gwq = __shfl_sync(dev::kFull, gw, q);
-            if ((wq >> lane) & 1u)
-                payload[base + __popc(wq & ((1u << lane) - 1u))] = values[gwq * 32 + lane];
+        const int rel_el = iel - pel;  // this lane's word: first payload slot relative to oel
+        // payload: word by word, lanes = element bits; 16 words per batch so 16 coalesced loads are
+        // in flight before the stores (the gather is latency-bound otherwise)
+        const int64_t gbase = w0 + wb + g * 32;
+#pragma unroll 1
+        for (int q0 = 0; q0 < 32; q0 += 16) {
+            uint32_t wq[16];
+            int bq[16];
+            T v[16];
+#pragma unroll
+            for (int u = 0; u < 16; ++u) {
+                wq[u] = __shfl_sync(dev::kFull, w, q0 + u);
+                bq[u] = __shfl_sync(dev::kFull, rel_el, q0 + u);
+                v[u] = ((wq[u] >> lane) & 1u) ? values[(gbase + q0 + u) * 32 + lane] : T(0);
+            }
+#pragma unroll
+            for (int u = 0; u < 16; ++u)
+                if ((wq[u] >> lane) & 1u) payload[oel + bq[u] + __popc(wq[u] & ((1u << lane) - 1u))] = v[u];
         }
         os += __shfl_sync(dev::kFull, is, 31);
         oe += __shfl_sync(dev::kFull, ie, 31);
@@ -268,9 +277,22 @@ scatter_k(const uint8_t* __restrict__ packed, int64_t n_runs, const PtrList dsts
         const int nr = (int)((hi - base) < kThreads ? (hi - base) : kThreads);
         for (int q = warp; q < nr; q += kThreads / 32) {
             const int64_t st = s_start[q], ln = s_len[q], of = s_off[q];
-            for (int64_t x = lane; x < ln; x += 32) {
-                const T v = payload[of + x];
-                for (int d = 0; d < dsts.n; ++d) static_cast<T*>(dsts.p[d])[st + x] = v;
+            // 8 independent loads per lane in flight, then the stores to every destination
+            for (int64_t x0 = 0; x0 < ln; x0 += 32 * 8) {
+                T v[8];
+#pragma unroll
+                for (int u = 0; u < 8; ++u) {
+                    const int64_t x = x0 + 32 * u + lane;
+                    v[u] = x < ln ? payload[of + x] : T(0);
+                }
+                for (int d = 0; d < dsts.n; ++d) {
+                    T* dp = static_cast<T*>(dsts.p[d]) + st;
+#pragma unroll
+                    for (int u = 0; u < 8; ++u) {
+                        const int64_t x = x0 + 32 * u + lane;
+                        if (x < ln) dp[x] = v[u];
+                    }
+                }
             }
         }
         __syncthreads();

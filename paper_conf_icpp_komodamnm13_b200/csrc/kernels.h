@@ -76,6 +76,10 @@ cudaError_t scatter_packed(const uint8_t* packed, int64_t n_runs, const PtrList&
 cudaError_t reduce_sum_i64(int64_t* acc, const PtrList& srcs, int64_t n, cudaStream_t s, int64_t* launches);
 cudaError_t apply_add_i64(const PtrList& dsts, const int64_t* acc, int64_t n, cudaStream_t s, int64_t* launches);
 
+// Cross-process device barrier (p2p.cu): peer_sigs.p[q] = rank q's sig array (mapped via IPC).
+cudaError_t device_barrier(const PtrList& peer_sigs, uint64_t* my_sig, int rank, int W, uint64_t epoch,
+                           cudaStream_t s, int64_t* launches);
+
 // Device-side bitwise AND test of two bitmaps (debug_checks): *flag |= any(a & b).
 cudaError_t bitmap_overlap(const uint32_t* a, const uint32_t* b, int64_t nwords, int* flag, cudaStream_t s,
                            int64_t* launches);

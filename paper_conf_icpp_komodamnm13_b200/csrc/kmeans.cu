@@ -11,9 +11,9 @@
 // FP32-pipe bound (2*k*d flops per point, no tensor-core form preserves the exact fmaf order that
 // the bit-exact argmin needs). Two points share each packed __fadd2_rn / __ffma2_rn
 // (Blackwell FADD2/FFMA2: two fp32 lanes per instruction, each rounded exactly like the scalar op),
-// so the per-distance operation order is the scalar one; each thread owns 4 points; centroids
+// so the per-distance operation order is the scalar one; each thread owns 8 points; centroids
 // are staged in shared memory pre-negated and duplicated as float2 (-c, -c) so one LDS.128 feeds
-// two dims of two packed operations.
+// two dims of four packed pairs (8 packed operations).
 #include <cuda_fp16.h>
 
 #include "kernels.h"
@@ -24,7 +24,7 @@ namespace k {
 namespace {
 
 constexpr int kThreads = 256;
-constexpr int kPPT = 4;  // points per thread (2 packed pairs)
+constexpr int kPPT = 8;  // points per thread (4 packed pairs: one LDS.128 feeds 8 packed ops)
 
 __device__ __forceinline__ int64_t fixed_of(float x, float scale, int* err) {
     const float v = x * scale;  // exact: power-of-two scaling
@@ -43,7 +43,7 @@ __device__ __forceinline__ void flush_block(unsigned long long* s_sum, unsigned 
 }
 
 template <int D>
-__global__ void __launch_bounds__(kThreads)
+__global__ void __launch_bounds__(kThreads, 1)
 assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __restrict__ member,
          int64_t* __restrict__ sums, int64_t* __restrict__ counts, int64_t p0, int64_t p1, int kc, int shift,
          int* err) {
@@ -58,60 +58,68 @@ assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __
     }
     for (int i = threadIdx.x; i < kc; i += kThreads) s_cnt[i] = 0ull;
     __syncthreads();
+    constexpr int NP = kPPT / 2;  // packed point pairs per thread
     const float scale = (float)(1 << shift);
     const int64_t n = p1 - p0;
     const int64_t ngroups = (n + kPPT - 1) / kPPT;
     for (int64_t grp = (int64_t)blockIdx.x * kThreads + threadIdx.x; grp < ngroups;
          grp += (int64_t)gridDim.x * kThreads) {
         const int64_t pb = p0 + grp * kPPT;
-        float2 xa[D], xb[D];  // (point0, point1), (point2, point3)
-        bool ok[kPPT];
+        float2 xp[NP][D];  // pair h = points (pb + 2h, pb + 2h + 1)
 #pragma unroll
-        for (int q = 0; q < kPPT; ++q) ok[q] = pb + q < p1;
+        for (int h = 0; h < NP; ++h) {
+            const bool ok0 = pb + 2 * h < p1, ok1 = pb + 2 * h + 1 < p1;
 #pragma unroll
-        for (int j = 0; j < D; j += 4) {
-            float4 v[kPPT];
-#pragma unroll
-            for (int q = 0; q < kPPT; ++q)
-                v[q] = ok[q] ? __ldg(reinterpret_cast<const float4*>(x + (pb + q) * D + j)) : make_float4(0.f, 0.f, 0.f, 0.f);
-            xa[j] = make_float2(v[0].x, v[1].x); xb[j] = make_float2(v[2].x, v[3].x);
-            xa[j + 1] = make_float2(v[0].y, v[1].y); xb[j + 1] = make_float2(v[2].y, v[3].y);
-            xa[j + 2] = make_float2(v[0].z, v[1].z); xb[j + 2] = make_float2(v[2].z, v[3].z);
-            xa[j + 3] = make_float2(v[0].w, v[1].w); xb[j + 3] = make_float2(v[2].w, v[3].w);
+            for (int j = 0; j < D; j += 4) {
+                const float4 a = ok0 ? __ldg(reinterpret_cast<const float4*>(x + (pb + 2 * h) * D + j))
+                                     : make_float4(0.f, 0.f, 0.f, 0.f);
+                const float4 b = ok1 ? __ldg(reinterpret_cast<const float4*>(x + (pb + 2 * h + 1) * D + j))
+                                     : make_float4(0.f, 0.f, 0.f, 0.f);
+                xp[h][j] = make_float2(a.x, b.x);
+                xp[h][j + 1] = make_float2(a.y, b.y);
+                xp[h][j + 2] = make_float2(a.z, b.z);
+                xp[h][j + 3] = make_float2(a.w, b.w);
+            }
         }
         float bd[kPPT];
         int bi[kPPT];
 #pragma unroll
         for (int q = 0; q < kPPT; ++q) { bd[q] = __int_as_float(0x7f800000); bi[q] = 0; }
-#pragma unroll 2
+#pragma unroll 1
         for (int c = 0; c < kc; ++c) {
-            float2 aa = make_float2(0.f, 0.f), ab = make_float2(0.f, 0.f);
+            float2 acc[NP];
+#pragma unroll
+            for (int h = 0; h < NP; ++h) acc[h] = make_float2(0.f, 0.f);
             const float4* nc4 = reinterpret_cast<const float4*>(s_nc + c * D);
 #pragma unroll
             for (int j = 0; j < D; j += 2) {
                 const float4 nc = nc4[j / 2];  // (-c_j, -c_j, -c_{j+1}, -c_{j+1})
                 const float2 n0 = make_float2(nc.x, nc.y), n1 = make_float2(nc.z, nc.w);
-                float2 da = __fadd2_rn(xa[j], n0), db = __fadd2_rn(xb[j], n0);
-                aa = __ffma2_rn(da, da, aa);
-                ab = __ffma2_rn(db, db, ab);
-                da = __fadd2_rn(xa[j + 1], n1);
-                db = __fadd2_rn(xb[j + 1], n1);
-                aa = __ffma2_rn(da, da, aa);
-                ab = __ffma2_rn(db, db, ab);
+#pragma unroll
+                for (int h = 0; h < NP; ++h) {
+                    const float2 d0 = __fadd2_rn(xp[h][j], n0);
+                    acc[h] = __ffma2_rn(d0, d0, acc[h]);
+                }
+#pragma unroll
+                for (int h = 0; h < NP; ++h) {
+                    const float2 d1 = __fadd2_rn(xp[h][j + 1], n1);
+                    acc[h] = __ffma2_rn(d1, d1, acc[h]);
+                }
             }
-            if (aa.x < bd[0]) { bd[0] = aa.x; bi[0] = c; }
-            if (aa.y < bd[1]) { bd[1] = aa.y; bi[1] = c; }
-            if (ab.x < bd[2]) { bd[2] = ab.x; bi[2] = c; }
-            if (ab.y < bd[3]) { bd[3] = ab.y; bi[3] = c; }
+#pragma unroll
+            for (int h = 0; h < NP; ++h) {
+                if (acc[h].x < bd[2 * h]) { bd[2 * h] = acc[h].x; bi[2 * h] = c; }
+                if (acc[h].y < bd[2 * h + 1]) { bd[2 * h + 1] = acc[h].y; bi[2 * h + 1] = c; }
+            }
         }
 #pragma unroll
         for (int q = 0; q < kPPT; ++q) {
-            if (!ok[q]) continue;
+            if (pb + q >= p1) continue;
             member[pb + q] = bi[q];
             atomicAdd(s_cnt + bi[q], 1ull);
 #pragma unroll
             for (int j = 0; j < D; ++j) {
-                const float xv = q == 0 ? xa[j].x : q == 1 ? xa[j].y : q == 2 ? xb[j].x : xb[j].y;
+                const float xv = (q & 1) ? xp[q / 2][j].y : xp[q / 2][j].x;
                 atomicAdd(s_sum + bi[q] * D + j, (unsigned long long)fixed_of(xv, scale, err));
             }
         }

@@ -27,6 +27,7 @@
 #include <string>
 #include <vector>
 
+#include "bootstrap.h"
 #include "intervals.h"
 #include "kernels.h"
 #include "nccl_dl.h"
@@ -63,6 +64,12 @@ struct accmg_region_s {
     IntervalSet host_valid;          // this process's host copy
     std::vector<Trk> trk;            // V
     std::vector<int64_t*> partial;   // V reduction partials (REDUCE_SUM)
+    // P2P mode (one process per GPU): this process's view of EVERY partition's replica / partial
+    // (local allocations, or peer allocations mapped through CUDA IPC)
+    std::vector<uint8_t*> gdev;      // P
+    std::vector<int64_t*> gpartial;  // P
+    int64_t* acc = nullptr;          // local reduction accumulator (P2P mode)
+    std::vector<void*> opened;       // IPC mappings to close
 };
 
 namespace {
@@ -76,7 +83,12 @@ struct State {
     bool init = false;
     accmg_config cfg{};
     int P = 1, W = 1, rank = 0, V = 1;
-    bool dry = false, nccl_all = false;
+    bool dry = false, nccl_all = false, p2p = false, use_nccl = false;
+    accmg::Bootstrap boot;
+    uint64_t* sig = nullptr;         // P2P barrier flags (W entries), mapped by every peer
+    std::vector<void*> peer_sig;     // W
+    std::vector<void*> sig_opened;
+    uint64_t epoch = 0;
     int64_t chunk_bytes = 1 << 20;
     cudaStream_t stream = nullptr;
     accmg::NcclApi* nccl = nullptr;
@@ -139,6 +151,44 @@ inline int rank_of(int g) { return g / S.V; }
 inline bool local(int g) { return rank_of(g) == S.rank; }
 inline int lidx(int g) { return g % S.V; }
 inline int first_local() { return S.rank * S.V; }
+
+// P2P mode: publish `mine` (this process's device allocations, one per local partition) and map
+// every peer's through CUDA IPC; out[g] = pointer usable here for partition g (collective).
+int exchange_ptrs(const std::vector<void*>& mine, std::vector<void*>& out, std::vector<void*>& opened) {
+    const int n = (int)mine.size();
+    if ((size_t)n * sizeof(cudaIpcMemHandle_t) > accmg::Bootstrap::kSlotBytes)
+        return fail(ACCMG_EUNSUPPORTED, "exchange_ptrs: too many handles", false);
+    auto* slot = static_cast<cudaIpcMemHandle_t*>(S.boot.slot(S.rank));
+    for (int i = 0; i < n; ++i) CUDA_TRY(cudaIpcGetMemHandle(&slot[i], mine[i]));
+    std::string err;
+    if (!S.boot.barrier(&err)) return fail(ACCMG_ESTATE, err, true);
+    out.assign((size_t)S.W * n, nullptr);
+    for (int q = 0; q < S.W; ++q) {
+        auto* qs = static_cast<cudaIpcMemHandle_t*>(S.boot.slot(q));
+        for (int i = 0; i < n; ++i) {
+            if (q == S.rank) {
+                out[(size_t)q * n + i] = mine[i];
+                continue;
+            }
+            void* p = nullptr;
+            CUDA_TRY(cudaIpcOpenMemHandle(&p, qs[i], cudaIpcMemLazyEnablePeerAccess));
+            out[(size_t)q * n + i] = p;
+            opened.push_back(p);
+        }
+    }
+    if (!S.boot.barrier(&err)) return fail(ACCMG_ESTATE, err, true);  // slots may be reused after this
+    return 0;
+}
+
+// P2P mode: the global barrier of L64 on the device (csrc/p2p.cu).
+int dev_barrier() {
+    if (!S.p2p) return 0;
+    k::PtrList pl{};
+    for (int q = 0; q < S.W; ++q) pl.p[pl.n++] = S.peer_sig[q];
+    ++S.epoch;
+    CUDA_TRY(k::device_barrier(pl, S.sig, S.rank, S.W, S.epoch, S.stream, &S.st.kernel_launches));
+    return 0;
+}
 
 void chunk_of(int64_t lo, int64_t hi, int P, int g, int64_t* a, int64_t* b) {
     // L108: "the tasks in the parallel loop are equally divided among the GPUs" (reading G6)
@@ -252,11 +302,12 @@ int run_xfers(const std::vector<Xfer>& xs) {
     // accounting (partition-to-partition bytes are whole-job totals, identical on every rank)
     for (auto& x : xs) {
         int64_t nb = (x.hi - x.lo) * x.r->esize;
+        if (!local(x.dst)) continue;  // bytes are counted by the receiving process
         if (x.src >= 0) {
             S.st.bytes_interpartition += nb;
             S.st.bytes_declared += nb;
             if (rank_of(x.src) != rank_of(x.dst)) S.st.bytes_remote += nb;
-        } else if (local(x.dst)) {
+        } else {
             S.st.bytes_h2d += nb;
             if (!x.r->host_valid.contains(IntervalSet(x.lo, x.hi)))
                 return fail(ACCMG_ESTATE, "data loader: range valid on no partition and not on the host copy", false);
@@ -275,6 +326,11 @@ int run_xfers(const std::vector<Xfer>& xs) {
         } else if (local(x.src) && local(x.dst) && !S.nccl_all) {
             CUDA_TRY(cudaMemcpyAsync(x.r->dev[lidx(x.dst)] + off, x.r->dev[lidx(x.src)] + off, nb,
                                      cudaMemcpyDeviceToDevice, S.stream));
+        } else if (S.p2p) {
+            // pull from the peer's replica, mapped through IPC: a copy-engine transfer over NVLink
+            if (local(x.dst))
+                CUDA_TRY(cudaMemcpyAsync(x.r->dev[lidx(x.dst)] + off, x.r->gdev[x.src] + off, nb, cudaMemcpyDefault,
+                                         S.stream));
         } else if (local(x.src) || local(x.dst)) {
             any_nccl = true;
         }
@@ -536,7 +592,7 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
         }
     // 3. sizes of every partition's packet (all-gather across processes when needed)
     std::vector<int64_t> runs(S.P * regs.size()), elems(S.P * regs.size()), chunks(S.P * regs.size());
-    const bool multi = S.W > 1 || S.nccl_all;
+    const bool multi = S.use_nccl;  // packets travel through NCCL (sizes must be all-gathered)
     if (multi) {
         // layout per rank: [region][local] x {runs, elems, chunks, pad}
         const int64_t per = (int64_t)regs.size() * S.V * 4;
@@ -564,31 +620,43 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
     } else {
         for (size_t ri = 0; ri < regs.size(); ++ri)
             for (int li = 0; li < S.V; ++li) {
-                runs[ri * S.P + li] = regs[ri]->trk[li].n_runs;
-                elems[ri * S.P + li] = regs[ri]->trk[li].n_elems;
-                chunks[ri * S.P + li] = regs[ri]->trk[li].dirty_chunks;
+                const int g = first_local() + li;
+                runs[ri * S.P + g] = regs[ri]->trk[li].n_runs;
+                elems[ri * S.P + g] = regs[ri]->trk[li].n_elems;
+                chunks[ri * S.P + g] = regs[ri]->trk[li].dirty_chunks;
             }
     }
-    // accounting: every packet is delivered to the P-1 other partitions (reading W8)
+    // accounting (by the sending process): every packet is delivered to the P-1 other partitions
+    // (reading W8)
     for (size_t ri = 0; ri < regs.size(); ++ri) {
         const int64_t es = regs[ri]->esize, ce = chunk_elems(regs[ri]);
         for (int g = 0; g < S.P; ++g) {
+            if (!local(g)) continue;
             const int64_t hdr = 16 + 16 * runs[ri * S.P + g], pay = es * elems[ri * S.P + g];
             S.st.bytes_undeclared_headers += (S.P - 1) * hdr;
             S.st.bytes_undeclared_payload += (S.P - 1) * pay;
             S.st.bytes_interpartition += (S.P - 1) * (hdr + pay);
             S.st.bytes_paper_protocol += (S.P - 1) * chunks[ri * S.P + g] * (ce * es + ce / 8);
             if (multi) S.st.bytes_remote += (int64_t)(S.W - 1 + (S.nccl_all ? 1 : 0)) * (hdr + pay);
+            if (S.p2p) S.st.bytes_remote += (int64_t)(S.P - S.V) * (hdr + pay);
         }
     }
     // 4. exchange + scatter
     ProfScope ps(2);
     if (!multi) {
+        // sender-side push: one scatter kernel writes the runs into every other replica — the
+        // local ones and (P2P mode) the peers' replicas through their IPC mappings over NVLink
         for (auto* r : regs)
             for (int li = 0; li < S.V; ++li) {
+                const int g = first_local() + li;
                 k::PtrList dl{};
-                for (int h = 0; h < S.V; ++h)
-                    if (h != li) dl.p[dl.n++] = r->dev[h];
+                if (S.p2p) {
+                    for (int h = 0; h < S.P; ++h)
+                        if (h != g) dl.p[dl.n++] = r->gdev[h];
+                } else {
+                    for (int h = 0; h < S.V; ++h)
+                        if (h != li) dl.p[dl.n++] = r->dev[h];
+                }
                 CUDA_TRY(k::scatter_packed(r->trk[li].packed, r->trk[li].n_runs, dl, (int)r->esize, S.scratch, S.stream,
                                            &S.st.kernel_launches));
             }
@@ -634,10 +702,25 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
 // ---- reductiontoarray merge (L112: block -> GPU -> across GPUs) ------------------------------------
 int merge_reduce(accmg_region_s* r) {
     ProfScope ps(2);
+    if (S.p2p) {
+        // every rank sums all P partials (its own and its peers', read over NVLink) after a
+        // barrier, applies the total to its replicas, and a second barrier keeps the partials
+        // alive until every rank has read them
+        TRY(dev_barrier());
+        CUDA_TRY(cudaMemsetAsync(r->acc, 0, r->extent * 8, S.stream));
+        k::PtrList src{};
+        for (int g = 0; g < S.P; ++g) src.p[src.n++] = r->gpartial[g];
+        CUDA_TRY(k::reduce_sum_i64(r->acc, src, r->extent, S.stream, &S.st.kernel_launches));
+        k::PtrList dl{};
+        for (int li = 0; li < S.V; ++li) dl.p[dl.n++] = r->dev[li];
+        CUDA_TRY(k::apply_add_i64(dl, r->acc, r->extent, S.stream, &S.st.kernel_launches));
+        TRY(dev_barrier());
+        return 0;
+    }
     k::PtrList src{};
     for (int li = 1; li < S.V; ++li) src.p[src.n++] = r->partial[li];
     CUDA_TRY(k::reduce_sum_i64(r->partial[0], src, r->extent, S.stream, &S.st.kernel_launches));
-    if (S.W > 1 || S.nccl_all)
+    if (S.use_nccl)
         NCCL_TRY(S.nccl->AllReduce(r->partial[0], r->partial[0], (size_t)r->extent, ncclInt64, ncclSum, S.comm, S.stream));
     k::PtrList dl{};
     for (int li = 0; li < S.V; ++li) dl.p[dl.n++] = r->dev[li];
@@ -660,6 +743,12 @@ int check_data_flag() {
 void free_region(accmg_region_s* r) {
     if (!S.dry) {
         cudaStreamSynchronize(S.stream);
+        for (auto p : r->opened) cudaIpcCloseMemHandle(p);
+        r->opened.clear();
+        if (S.p2p) {  // nobody frees memory a peer may still have mapped
+            std::string err;
+            S.boot.barrier(&err);
+        }
         for (auto p : r->dev) dfree(p, r->extent * r->esize, false);
         for (auto& t : r->trk) {
             dfree(t.l1, t.nwords * 4, true);
@@ -673,6 +762,7 @@ void free_region(accmg_region_s* r) {
             dfree(t.snap_l2, t.nl2 * 4, true);
         }
         for (auto p : r->partial) dfree(p, r->extent * 8, true);
+        dfree(r->acc, r->extent * 8, true);
     }
     delete r;
 }
@@ -705,7 +795,8 @@ int accmg_init(const accmg_config* cfg) {
     if (c.num_partitions > 64) return fail(ACCMG_EUNSUPPORTED, "init: at most 64 partitions", false);
     int64_t cb = c.dirty_chunk_bytes ? c.dirty_chunk_bytes : (1 << 20);
     if (cb < 256 || (cb & (cb - 1))) return fail(ACCMG_EINVAL, "init: dirty_chunk_bytes must be a power of two >= 256", false);
-    if (c.exchange_mode != ACCMG_XCHG_AUTO && c.exchange_mode != ACCMG_XCHG_NCCL_ALL)
+    if (c.exchange_mode != ACCMG_XCHG_AUTO && c.exchange_mode != ACCMG_XCHG_NCCL_ALL &&
+        c.exchange_mode != ACCMG_XCHG_NCCL)
         return fail(ACCMG_EINVAL, "init: bad exchange_mode", false);
     S = State();
     S.cfg = c;
@@ -715,6 +806,8 @@ int accmg_init(const accmg_config* cfg) {
     S.V = S.P / S.W;
     S.dry = c.device < 0;
     S.nccl_all = c.exchange_mode == ACCMG_XCHG_NCCL_ALL;
+    S.p2p = !S.dry && S.W > 1 && c.exchange_mode == ACCMG_XCHG_AUTO;
+    S.use_nccl = !S.dry && (S.nccl_all || (S.W > 1 && c.exchange_mode == ACCMG_XCHG_NCCL));
     S.chunk_bytes = cb;
     if (S.dry) {
         S.init = true;
@@ -727,7 +820,16 @@ int accmg_init(const accmg_config* cfg) {
     TRY(dmalloc((void**)&S.d_flag, 16, true));
     CUDA_TRY(cudaHostAlloc((void**)&S.h_pin, (size_t)4 * 8 * 16 * S.P * (S.W + 1) + 64, cudaHostAllocDefault));
     CUDA_TRY(cudaMemsetAsync(S.d_flag, 0, 16, S.stream));
-    if (S.W > 1 || S.nccl_all) {
+    if (S.p2p) {
+        std::string err;
+        if (!S.boot.open(c.nccl_unique_id, S.rank, S.W, &err)) return fail(ACCMG_ESTATE, err, true);
+        TRY(dmalloc((void**)&S.sig, 8 * 64, true));
+        CUDA_TRY(cudaMemset(S.sig, 0, 8 * 64));
+        CUDA_TRY(cudaDeviceSynchronize());
+        std::vector<void*> mine{S.sig};
+        TRY(exchange_ptrs(mine, S.peer_sig, S.sig_opened));
+    }
+    if (S.use_nccl) {
         const char* why = nullptr;
         S.nccl = accmg::nccl_api(&why);
         if (!S.nccl) return fail(ACCMG_ENCCL, why ? why : "NCCL unavailable", true);
@@ -748,6 +850,13 @@ int accmg_finalize(void) {
     }
     for (auto* r : S.regions) free_region(r);
     S.regions.clear();
+    if (S.p2p) {
+        for (auto p : S.sig_opened) cudaIpcCloseMemHandle(p);
+        std::string err;
+        S.boot.barrier(&err);
+        dfree(S.sig, 0, true);
+        S.boot.close();
+    }
     if (!S.dry) {
         dfree(S.scratch, 0, true);
         dfree(S.d_sizes, 0, true);
@@ -785,6 +894,16 @@ int accmg_region_create(void* host_array, size_t elem_size, int64_t extent, accm
                 free_region(r);
                 return rc;
             }
+        }
+        if (S.p2p) {
+            std::vector<void*> mine(r->dev.begin(), r->dev.end()), all;
+            int rc = exchange_ptrs(mine, all, r->opened);
+            if (rc) {
+                free_region(r);
+                return rc;
+            }
+            r->gdev.resize(S.P);
+            for (int g = 0; g < S.P; ++g) r->gdev[g] = static_cast<uint8_t*>(all[g]);
         }
     }
     S.regions.push_back(r);
@@ -865,9 +984,17 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
         for (int i = 0; i < n_descs; ++i)
             if (descs[i].mode == ACCMG_REDUCE_SUM) {
                 accmg_region_s* r = descs[i].region;
+                const bool fresh = !r->partial[0];
                 for (int li = 0; li < S.V; ++li) {
                     if (!r->partial[li]) TRY(dmalloc((void**)&r->partial[li], r->extent * 8, true));
                     CUDA_TRY(cudaMemsetAsync(r->partial[li], 0, r->extent * 8, S.stream));
+                }
+                if (S.p2p && fresh) {  // same loop on every rank: publish the partials
+                    TRY(dmalloc((void**)&r->acc, r->extent * 8, true));
+                    std::vector<void*> mine(r->partial.begin(), r->partial.end()), all;
+                    TRY(exchange_ptrs(mine, all, r->opened));
+                    r->gpartial.resize(S.P);
+                    for (int g = 0; g < S.P; ++g) r->gpartial[g] = static_cast<int64_t*>(all[g]);
                 }
             }
         // 4. bodies on this process's partitions
@@ -882,12 +1009,17 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
         if (!tracked_regs.empty()) TRY(propagate_dirty(tracked_regs));
         for (int i = 0; i < n_descs; ++i)
             if (descs[i].mode == ACCMG_REDUCE_SUM) TRY(merge_reduce(descs[i].region));
+        // 6. global barrier (L64): no process starts the next loop before every peer finished
+        // this one (its body, its pushes and its pulls from the others' replicas)
+        TRY(dev_barrier());
     }
     for (int i = 0; i < n_descs; ++i) {
         accmg_region_s* r = descs[i].region;
         if (descs[i].mode == ACCMG_REDUCE_SUM) {
-            S.st.bytes_reduce += 2 * (int64_t)(S.P - 1) * r->extent * 8;
-            S.st.bytes_interpartition += 2 * (int64_t)(S.P - 1) * r->extent * 8;
+            // this process's V/P share of the ring all-reduce volume 2(P-1)*extent*8 (reading W8)
+            const int64_t nb = 2 * (int64_t)(S.P - 1) * r->extent * 8 * S.V / S.P;
+            S.st.bytes_reduce += nb;
+            S.st.bytes_interpartition += nb;
             r->host_valid.clear();
         } else if (descs[i].mode & ACCMG_W) {
             if (descs[i].declared) {
@@ -924,6 +1056,7 @@ static int sync_host_impl(accmg_region r, bool owned) {
         plan_pulls(r, need, xs);
         TRY(run_xfers(xs));
         for (int g = 0; g < S.P; ++g) r->valid[g].add(need[g]);
+        TRY(dev_barrier());
     }
     TRY(check_data_flag());
     IntervalSet todo(0, r->extent);
@@ -1057,3 +1190,14 @@ int accmg_debug_valid(accmg_region r, int partition, int64_t* out_pairs, int64_t
 }
 
 }  // extern "C"
+
+extern "C" int accmg_unique_id(uint8_t out[128]) {
+    if (!out) return fail(ACCMG_EINVAL, "unique_id: null", false);
+    FILE* f = std::fopen("/dev/urandom", "rb");
+    if (!f || std::fread(out, 1, 128, f) != 128) {
+        if (f) std::fclose(f);
+        return fail(ACCMG_ESTATE, "unique_id: cannot read /dev/urandom", false);
+    }
+    std::fclose(f);
+    return 0;
+}

@@ -83,5 +83,63 @@ __device__ __forceinline__ void track_warp(uint32_t* __restrict__ l1, uint32_t* 
     }
 }
 
+// Row-marching variant: a warp that writes the same lane/element mask on many rows (a fixed
+// column strip) builds the span pattern once; each row then costs one shift, plain stores for
+// the words it owns outright and atomicOr only on shared edge words, plus a cached L2 check.
+// Precondition: the elements a warp writes in one row form one contiguous range that no other
+// warp writes in the same loop (true for the row-strip bodies).
+template <int VEC>
+struct WarpTracker {
+    uint32_t lo = 0u, hi = 0u;  // this lane's relative words rel[lane], rel[lane-1]
+    int first = -1, last = -1;  // first/last written element offset within the span
+    int64_t l2_cache = -1;
+
+    __device__ __forceinline__ void init(unsigned nib) {
+        const int lane = threadIdx.x & 31;
+        uint32_t rel[VEC];
+        if constexpr (VEC == 4) {
+            uint32_t b0 = __ballot_sync(kFull, nib & 1u), b1 = __ballot_sync(kFull, nib & 2u);
+            uint32_t b2 = __ballot_sync(kFull, nib & 4u), b3 = __ballot_sync(kFull, nib & 8u);
+#pragma unroll
+            for (int q = 0; q < VEC; ++q) {
+                const int sh = 8 * q;
+                rel[q] = spread4(b0 >> sh) | (spread4(b1 >> sh) << 1) | (spread4(b2 >> sh) << 2) |
+                         (spread4(b3 >> sh) << 3);
+            }
+        } else {
+            rel[0] = __ballot_sync(kFull, nib & 1u);
+        }
+#pragma unroll
+        for (int q = 0; q < VEC; ++q) {
+            lo = (q == lane) ? rel[q] : lo;
+            hi = (q == lane - 1) ? rel[q] : hi;
+            if (rel[q]) {
+                if (first < 0) first = 32 * q + __ffs(rel[q]) - 1;
+                last = 32 * q + 31 - __clz(rel[q]);
+            }
+        }
+    }
+
+    __device__ __forceinline__ void mark(uint32_t* __restrict__ l1, uint32_t* __restrict__ l2, int l2_shift,
+                                         int64_t E0) {
+        if (first < 0) return;  // warp-uniform: nothing written by this warp
+        const int lane = threadIdx.x & 31;
+        const int s = (int)(E0 & 31);
+        if (lane <= VEC) {
+            const uint32_t v = (lo << s) | (s ? (hi >> (32 - s)) : 0u);
+            const int64_t w = (E0 >> 5) + lane;
+            // A word lying entirely inside this warp's written range holds only elements this warp
+            // writes (the range is contiguous and no other warp writes them in this loop, L62), and
+            // compaction left it zero: a plain store is exact. Edge words may be shared: atomicOr.
+            const bool inner = w * 32 >= E0 + first && w * 32 + 31 <= E0 + last;
+            if (v) {
+                if (inner) l1[w] = v;
+                else atomicOr(l1 + w, v);
+            }
+        }
+        if (lane == 0) track_l2(l2, l2_shift, E0 + first, E0 + last, l2_cache);
+    }
+};
+
 }  // namespace dev
 }  // namespace accmg

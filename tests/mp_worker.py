@@ -1,0 +1,51 @@
+"""One rank of a multi-process (one process per GPU) run, used by tests/test_gpu_multiproc.py.
+
+usage: python tests/mp_worker.py RANK WORLD V UID_HEX WORKLOAD OUTDIR [EXCHANGE_MODE]
+Runs the workload through the C ABI with world_size = WORLD, num_partitions = WORLD * V, and
+saves its host arrays (after sync_to_host) and its stats under OUTDIR/rank<R>_*.npy/.json.
+"""
+import json
+import os
+import sys
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+import gen  # noqa: E402
+from paper_conf_icpp_komodamnm13_b200 import accmg as A  # noqa: E402
+from paper_conf_icpp_komodamnm13_b200 import workloads as WL  # noqa: E402
+
+
+def main():
+    rank, world, V = int(sys.argv[1]), int(sys.argv[2]), int(sys.argv[3])
+    uid = bytes.fromhex(sys.argv[4])
+    work, out = sys.argv[5], sys.argv[6]
+    mode = int(sys.argv[7]) if len(sys.argv) > 7 else A.XCHG_AUTO
+    A.accmg_init(num_partitions=world * V, world_size=world, rank=rank, device=0, nccl_unique_id=uid,
+                 exchange_mode=mode, dirty_chunk_bytes=8192)
+    res = {}
+    if work in ("jacobi_decl", "jacobi_undecl"):
+        N, S = 300, 6
+        Ah = gen.jacobi_field(5, N)
+        Bh = Ah.copy()
+        per = WL.jacobi_run(Ah, Bh, S, declared=(work == "jacobi_decl"), per_loop_stats=True)
+        res = {"A": Ah, "B": Bh}
+        loops = {k: sum(p[k] for p in per) for k in per[0]}
+    elif work == "kmeans":
+        x = gen.kmeans_points(5, 20000, 16, 32, gen.KM_OVERLAP)
+        cen, mem = WL.kmeans_run(x, 32, 5)
+        res = {"cen": cen, "mem": mem}
+    st = A.accmg_get_stats()
+    if work.startswith("jacobi"):
+        st = {"total": st, **loops}
+    A.accmg_finalize()
+    for k, v in res.items():
+        np.save(os.path.join(out, f"rank{rank}_{k}.npy"), v)
+    with open(os.path.join(out, f"rank{rank}_stats.json"), "w") as f:
+        json.dump(st, f)
+
+
+if __name__ == "__main__":
+    main()

@@ -1,0 +1,64 @@
+"""One process per GPU (SPMD) through the C ABI: two processes share the one B200 available
+in-round (each its own CUDA context), exchanging through CUDA IPC mappings (P2P mode) and a
+device-side flag barrier — the same code path as one process per GPU on an NVSwitch box. Results
+must equal the oracle bit for bit on every rank, and the per-rank byte counters must sum to the
+single-process totals."""
+import json
+import os
+import subprocess
+import sys
+
+import numpy as np
+import pytest
+
+import gen
+import oracle
+from tests.gpu_util import need_gpu
+
+pytestmark = pytest.mark.gpu
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(autouse=True)
+def _gpu():
+    need_gpu()
+
+
+def _launch(world, V, work, tmp_path, mode=0):
+    uid = os.urandom(128).hex()
+    procs = [subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "mp_worker.py"), str(r), str(world), str(V),
+                               uid, work, str(tmp_path), str(mode)], cwd=ROOT)
+             for r in range(world)]
+    for p in procs:
+        assert p.wait(timeout=600) == 0
+    stats = [json.load(open(tmp_path / f"rank{r}_stats.json")) for r in range(world)]
+    return stats
+
+
+@pytest.mark.parametrize("work,V", [("jacobi_decl", 1), ("jacobi_decl", 2), ("jacobi_undecl", 1), ("jacobi_undecl", 2)])
+def test_jacobi_two_processes(tmp_path, work, V):
+    N, S = 300, 6
+    A0 = gen.jacobi_field(5, N)
+    oA, oB = A0.copy(), A0.copy()
+    oracle.jacobi_run(oA, oB, S)
+    stats = _launch(2, V, work, tmp_path)
+    for r in range(2):
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_A.npy"), oA)
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_B.npy"), oB)
+    P = 2 * V
+    tot = sum(s["bytes_interpartition"] for s in stats)
+    if work == "jacobi_decl":
+        assert sum(s["bytes_declared"] for s in stats) == (S - 1) * 2 * (P - 1) * 4 * N
+    else:
+        assert tot == S * (P - 1) * (16 * P + 16 * (N - 2) + 4 * (N - 2) ** 2)
+    assert sum(s["bytes_remote"] for s in stats) > 0
+
+
+def test_kmeans_two_processes(tmp_path):
+    x = gen.kmeans_points(5, 20000, 16, 32, gen.KM_OVERLAP)
+    ocen, omem = oracle.kmeans_run(x, 32, 5)
+    stats = _launch(2, 2, "kmeans", tmp_path)
+    for r in range(2):
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_cen.npy"), ocen)
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_mem.npy"), omem)
+    assert sum(s["bytes_reduce"] for s in stats) == 5 * 2 * 3 * (32 * 16 + 32) * 8
