@@ -190,3 +190,17 @@ def test_kmeans_thread_invariance():
     c1, m1 = oracle.kmeans_run(x, 64, 3, nthreads=1)
     c2, m2 = oracle.kmeans_run(x, 64, 3, nthreads=4)
     assert np.array_equal(c1, c2) and np.array_equal(m1, m2)
+
+
+def test_dependence_cone_window_reproduces_full_field():
+    """Pins the sampled full-size parity method of tests/test_gpu_fullsize.py: after S sweeps a
+    point depends only on the initial field within distance S, so sweeping the sub-grid of radius
+    S+1 around it (true boundaries kept) reproduces the full-field value bit for bit."""
+    from tests.test_gpu_fullsize import _oracle_point_window
+    N, S = 200, 7
+    A = gen.jacobi_field(2, N)
+    B = A.copy()
+    oracle.jacobi_run(A, B, S)
+    for (i, j) in [(1, 1), (N - 2, N - 2), (50, 100), (1, N - 2), (100, 1), (8, 8)]:
+        F, G, i0, j0 = _oracle_point_window(2, N, S, i, j)
+        assert A[i, j] == F[i - i0, j - j0] and B[i, j] == G[i - i0, j - j0]
