@@ -11,10 +11,12 @@
 // FP32-pipe bound (2*k*d flops per point, no tensor-core form preserves the exact fmaf order that
 // the bit-exact argmin needs). Two points share each packed __fadd2_rn / __ffma2_rn
 // (Blackwell FADD2/FFMA2: two fp32 lanes per instruction, each rounded exactly like the scalar op),
-// so the per-distance operation order is the scalar one; each thread owns 8 points; centroids
+// so the per-distance operation order is the scalar one; each thread owns 4 points; centroids
 // are staged in shared memory pre-negated and duplicated as float2 (-c, -c) so one LDS.128 feeds
-// two dims of four packed pairs (8 packed operations).
-#include <cuda_fp16.h>
+// two dims of two packed pairs, and the next centroid is prefetched while the current one is
+// consumed. Packed ops halve the issue slots but not the FP32 lane rate (128 lanes/clk/SM,
+// measured with scripts/fp32_micro.cu), which is the roofline of this kernel.
+#include <cstdlib>
 
 #include "kernels.h"
 #include "track.cuh"
@@ -24,12 +26,40 @@ namespace k {
 namespace {
 
 constexpr int kThreads = 256;
-constexpr int kPPT = 8;  // points per thread (4 packed pairs: one LDS.128 feeds 8 packed ops)
 
 __device__ __forceinline__ int64_t fixed_of(float x, float scale, int* err) {
     const float v = x * scale;  // exact: power-of-two scaling
     if (!(v == rintf(v) && fabsf(v) < 2147483648.0f)) atomicOr(err, 1);
     return (int64_t)v;
+}
+
+// Packed fp32x2 arithmetic on 64-bit registers (PTX add/fma .f32x2, sm_100): each lane is
+// rounded exactly like the scalar add.rn / fma.rn. Holding the pairs as .b64 values keeps them in
+// aligned register pairs (the float2 builtins let ptxas re-pair scalars with MOVs every use).
+__device__ __forceinline__ uint64_t pk2(float a, float b) {
+    uint64_t r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+    return r;
+}
+// Materialises a pair in an aligned register pair: x + (-0) == x for every x (also +-0), done
+// by a real FADD2 so the allocator keeps the pair instead of re-pairing scalars on every use.
+__device__ __forceinline__ uint64_t pk2m(float a, float b) {
+    uint64_t r;
+    asm volatile("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(pk2(a, b)), "l"(0x8000000080000000ull));
+    return r;
+}
+__device__ __forceinline__ void upk2(uint64_t v, float& a, float& b) {
+    asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(v));
+}
+__device__ __forceinline__ uint64_t add2(uint64_t a, uint64_t b) {
+    uint64_t d;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+}
+__device__ __forceinline__ uint64_t fma2sq(uint64_t d, uint64_t acc) {  // d*d + acc
+    uint64_t r;
+    asm("fma.rn.f32x2 %0, %1, %1, %2;" : "=l"(r) : "l"(d), "l"(acc));
+    return r;
 }
 
 // Block-level accumulation into shared memory, then flush to the partition's partial (global).
@@ -42,8 +72,11 @@ __device__ __forceinline__ void flush_block(unsigned long long* s_sum, unsigned 
         if (s_cnt[i]) atomicAdd(reinterpret_cast<unsigned long long*>(counts) + i, s_cnt[i]);
 }
 
-template <int D>
-__global__ void __launch_bounds__(kThreads, 1)
+// D dims, NP packed point pairs per thread (2*NP points), CU centroids per step (NP*CU
+// independent FFMA2 chains per thread hide the packed-op latency; one LDS.128 of a centroid's
+// duplicated pair of dims feeds 4*NP packed operations).
+template <int D, int NP, int CU, int NT, int MINB>
+__global__ void __launch_bounds__(NT, MINB)
 assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __restrict__ member,
          int64_t* __restrict__ sums, int64_t* __restrict__ counts, int64_t p0, int64_t p1, int kc, int shift,
          int* err) {
@@ -51,21 +84,21 @@ assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __
     float2* s_nc = reinterpret_cast<float2*>(smem);                                  // kc*D  (-c,-c)
     unsigned long long* s_sum = reinterpret_cast<unsigned long long*>(s_nc + kc * D);  // kc*D
     unsigned long long* s_cnt = s_sum + kc * D;                                      // kc
-    for (int i = threadIdx.x; i < kc * D; i += kThreads) {
+    for (int i = threadIdx.x; i < kc * D; i += NT) {
         const float c = -cen[i];
         s_nc[i] = make_float2(c, c);
         s_sum[i] = 0ull;
     }
-    for (int i = threadIdx.x; i < kc; i += kThreads) s_cnt[i] = 0ull;
+    for (int i = threadIdx.x; i < kc; i += NT) s_cnt[i] = 0ull;
     __syncthreads();
-    constexpr int NP = kPPT / 2;  // packed point pairs per thread
+    constexpr int PPT = 2 * NP;
     const float scale = (float)(1 << shift);
     const int64_t n = p1 - p0;
-    const int64_t ngroups = (n + kPPT - 1) / kPPT;
-    for (int64_t grp = (int64_t)blockIdx.x * kThreads + threadIdx.x; grp < ngroups;
-         grp += (int64_t)gridDim.x * kThreads) {
-        const int64_t pb = p0 + grp * kPPT;
-        float2 xp[NP][D];  // pair h = points (pb + 2h, pb + 2h + 1)
+    const int64_t ngroups = (n + PPT - 1) / PPT;
+    const float4* nc4 = reinterpret_cast<const float4*>(s_nc);
+    for (int64_t grp = (int64_t)blockIdx.x * NT + threadIdx.x; grp < ngroups; grp += (int64_t)gridDim.x * NT) {
+        const int64_t pb = p0 + grp * PPT;
+        uint64_t xp[NP][D];  // pair h = (x[pb+2h][j], x[pb+2h+1][j])
 #pragma unroll
         for (int h = 0; h < NP; ++h) {
             const bool ok0 = pb + 2 * h < p1, ok1 = pb + 2 * h + 1 < p1;
@@ -75,56 +108,99 @@ assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __
                                      : make_float4(0.f, 0.f, 0.f, 0.f);
                 const float4 b = ok1 ? __ldg(reinterpret_cast<const float4*>(x + (pb + 2 * h + 1) * D + j))
                                      : make_float4(0.f, 0.f, 0.f, 0.f);
-                xp[h][j] = make_float2(a.x, b.x);
-                xp[h][j + 1] = make_float2(a.y, b.y);
-                xp[h][j + 2] = make_float2(a.z, b.z);
-                xp[h][j + 3] = make_float2(a.w, b.w);
+                xp[h][j] = pk2m(a.x, b.x);
+                xp[h][j + 1] = pk2m(a.y, b.y);
+                xp[h][j + 2] = pk2m(a.z, b.z);
+                xp[h][j + 3] = pk2m(a.w, b.w);
             }
         }
-        float bd[kPPT];
-        int bi[kPPT];
+        float bd[PPT];
+        int bi[PPT];
 #pragma unroll
-        for (int q = 0; q < kPPT; ++q) { bd[q] = __int_as_float(0x7f800000); bi[q] = 0; }
+        for (int q = 0; q < PPT; ++q) { bd[q] = __int_as_float(0x7f800000); bi[q] = 0; }
+        const ulonglong2* nc2 = reinterpret_cast<const ulonglong2*>(s_nc);
+        // the next centroid group's values are loaded while the current one is consumed (the
+        // shared-memory latency is off the critical path)
+        ulonglong2 ncur[CU][D / 2];
+#pragma unroll
+        for (int u = 0; u < CU; ++u)
+#pragma unroll
+            for (int jj = 0; jj < D / 2; ++jj) ncur[u][jj] = nc2[(u * D) / 2 + jj];
 #pragma unroll 1
-        for (int c = 0; c < kc; ++c) {
-            float2 acc[NP];
+        for (int c = 0; c < kc; c += CU) {
+            ulonglong2 nnext[CU][D / 2];
+            const int cn = (c + CU < kc) ? c + CU : c;
 #pragma unroll
-            for (int h = 0; h < NP; ++h) acc[h] = make_float2(0.f, 0.f);
-            const float4* nc4 = reinterpret_cast<const float4*>(s_nc + c * D);
+            for (int u = 0; u < CU; ++u)
+#pragma unroll
+                for (int jj = 0; jj < D / 2; ++jj) nnext[u][jj] = nc2[((cn + u) * D) / 2 + jj];
+            uint64_t acc[CU][NP];
+#pragma unroll
+            for (int u = 0; u < CU; ++u)
+#pragma unroll
+                for (int h = 0; h < NP; ++h) acc[u][h] = 0ull;
 #pragma unroll
             for (int j = 0; j < D; j += 2) {
-                const float4 nc = nc4[j / 2];  // (-c_j, -c_j, -c_{j+1}, -c_{j+1})
-                const float2 n0 = make_float2(nc.x, nc.y), n1 = make_float2(nc.z, nc.w);
+#pragma unroll
+                for (int u = 0; u < CU; ++u)
+#pragma unroll
+                    for (int h = 0; h < NP; ++h) acc[u][h] = fma2sq(add2(xp[h][j], ncur[u][j / 2].x), acc[u][h]);
+#pragma unroll
+                for (int u = 0; u < CU; ++u)
+#pragma unroll
+                    for (int h = 0; h < NP; ++h) acc[u][h] = fma2sq(add2(xp[h][j + 1], ncur[u][j / 2].y), acc[u][h]);
+            }
+            // centroids in ascending order: strict < keeps the lowest index on ties
+#pragma unroll
+            for (int u = 0; u < CU; ++u)
 #pragma unroll
                 for (int h = 0; h < NP; ++h) {
-                    const float2 d0 = __fadd2_rn(xp[h][j], n0);
-                    acc[h] = __ffma2_rn(d0, d0, acc[h]);
+                    float d0, d1;
+                    upk2(acc[u][h], d0, d1);
+                    if (d0 < bd[2 * h]) { bd[2 * h] = d0; bi[2 * h] = c + u; }
+                    if (d1 < bd[2 * h + 1]) { bd[2 * h + 1] = d1; bi[2 * h + 1] = c + u; }
                 }
 #pragma unroll
-                for (int h = 0; h < NP; ++h) {
-                    const float2 d1 = __fadd2_rn(xp[h][j + 1], n1);
-                    acc[h] = __ffma2_rn(d1, d1, acc[h]);
-                }
-            }
+            for (int u = 0; u < CU; ++u)
 #pragma unroll
-            for (int h = 0; h < NP; ++h) {
-                if (acc[h].x < bd[2 * h]) { bd[2 * h] = acc[h].x; bi[2 * h] = c; }
-                if (acc[h].y < bd[2 * h + 1]) { bd[2 * h + 1] = acc[h].y; bi[2 * h + 1] = c; }
-            }
+                for (int jj = 0; jj < D / 2; ++jj) ncur[u][jj] = nnext[u][jj];
         }
 #pragma unroll
-        for (int q = 0; q < kPPT; ++q) {
+        for (int q = 0; q < PPT; ++q) {
             if (pb + q >= p1) continue;
             member[pb + q] = bi[q];
             atomicAdd(s_cnt + bi[q], 1ull);
 #pragma unroll
             for (int j = 0; j < D; ++j) {
-                const float xv = (q & 1) ? xp[q / 2][j].y : xp[q / 2][j].x;
+                float xa, xb;
+                upk2(xp[q / 2][j], xa, xb);
+                const float xv = (q & 1) ? xb : xa;
                 atomicAdd(s_sum + bi[q] * D + j, (unsigned long long)fixed_of(xv, scale, err));
             }
         }
     }
     flush_block(s_sum, s_cnt, sums, counts, kc, D);
+}
+
+template <int NP, int CU, int NT, int MINB = 1>
+cudaError_t launch_assign16(const float* x, const float* cen, int32_t* member, int64_t* sums, int64_t* counts,
+                            int64_t p0, int64_t p1, int kc, int shift, int* err, cudaStream_t s, int sms) {
+    auto kern = assign_d<16, NP, CU, NT, MINB>;
+    const size_t smem = (size_t)kc * 16 * 8 + (size_t)kc * 16 * 8 + (size_t)kc * 8;
+    if (smem > 200 * 1024) return cudaErrorNotSupported;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    // all of the unified L1/shared capacity as shared memory, so several blocks fit per SM
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem);
+    const int64_t groups = (p1 - p0 + 2 * NP - 1) / (2 * NP);
+    int64_t blocks = (groups + NT - 1) / NT;
+    const int64_t cap = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
+    if (blocks > cap) blocks = cap;
+    kern<<<(unsigned)blocks, NT, smem, s>>>(x, cen, member, sums, counts, p0, p1, kc, shift, err);
+    return cudaGetLastError();
 }
 
 // Generic d (any d <= 32): one point per thread, scalar fmaf chain in the same order.
@@ -223,17 +299,27 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
     if (p1 <= p0) return cudaSuccess;
     const int sms = sm_count();
     if (d == 16 && (reinterpret_cast<uintptr_t>(x) % 16) == 0) {
-        const size_t smem = (size_t)kc * 16 * 8 + (size_t)kc * 16 * 8 + (size_t)kc * 8;
-        if (smem > 200 * 1024) return cudaErrorNotSupported;
-        cudaError_t e = cudaFuncSetAttribute(assign_d<16>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        // variant (tuning knob, default chosen from measurements in profiles/)
+        static int variant = -1;
+        if (variant < 0) {
+            const char* v = getenv("ACCMG_KMEANS_VARIANT");
+            variant = v ? atoi(v) : 0;
+        }
+        cudaError_t e;
+        const bool cu2 = kc % 2 == 0;
+        switch (variant) {
+            case 1: e = launch_assign16<2, 1, 256, 1>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 2: e = launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 3: e = launch_assign16<2, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 4: e = launch_assign16<4, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 5: e = launch_assign16<4, 1, 256, 1>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 6: e = cu2 ? launch_assign16<2, 2, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                            : launch_assign16<2, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 7: e = launch_assign16<1, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            // default: measured fastest on B200 (profiles/r01/kmeans_variants.txt)
+            default: e = launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+        }
         if (e != cudaSuccess) return e;
-        int per_sm = 0;
-        cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, assign_d<16>, kThreads, smem);
-        const int64_t groups = (p1 - p0 + kPPT - 1) / kPPT;
-        int64_t blocks = (groups + kThreads - 1) / kThreads;
-        const int64_t cap = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
-        if (blocks > cap) blocks = cap;
-        assign_d<16><<<(unsigned)blocks, kThreads, smem, s>>>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag);
     } else {
         const size_t smem = (((size_t)kc * d * 4 + 15) / 16) * 16 + (size_t)kc * d * 8 + (size_t)kc * 8;
         if (smem > 200 * 1024) return cudaErrorNotSupported;
