@@ -95,41 +95,54 @@ count_k(const uint32_t* __restrict__ l1, const uint32_t* __restrict__ l2, int64_
     }
 }
 
+// One block: exclusive scan of the per-tile triples {starts, ends, elems}, 1024 tiles per step
+// (coalesced loads, warp-shuffle scans, one carry per step), then the L2 popcount + clear.
 __global__ void __launch_bounds__(1024)
 scan_k(const int64_t* __restrict__ tile_counts, int64_t ntiles, int64_t* __restrict__ tile_offs,
        int64_t* __restrict__ totals, uint32_t* __restrict__ l2, int64_t nl2words) {
-    __shared__ int64_t sh[3][1024];
-    const int tid = threadIdx.x;
-    const int64_t per = (ntiles + 1023) / 1024;
-    const int64_t b = tid * per, e = (b + per < ntiles) ? b + per : ntiles;
-    int64_t s[3] = {0, 0, 0};
-    for (int64_t t = b; t < e; ++t)
-        for (int q = 0; q < 3; ++q) s[q] += tile_counts[3 * t + q];
-    for (int q = 0; q < 3; ++q) sh[q][tid] = s[q];
+    __shared__ int64_t wsum[3][32];
+    __shared__ int64_t carry[3];
+    __shared__ unsigned long long nchunks;
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid < 3) carry[tid] = 0;
+    if (tid == 0) nchunks = 0ull;
     __syncthreads();
-    // Hillis-Steele inclusive scan over 1024 thread sums
-    for (int o = 1; o < 1024; o <<= 1) {
-        int64_t v[3];
-        for (int q = 0; q < 3; ++q) v[q] = tid >= o ? sh[q][tid - o] : 0;
+    for (int64_t base = 0; base < ntiles; base += 1024) {
+        const int64_t t = base + tid;
+        int64_t v[3], inc[3];
+#pragma unroll
+        for (int q = 0; q < 3; ++q) {
+            v[q] = t < ntiles ? tile_counts[3 * t + q] : 0;
+            inc[q] = warp_incl_scan(v[q]);
+            if (lane == 31) wsum[q][warp] = inc[q];
+        }
         __syncthreads();
-        for (int q = 0; q < 3; ++q) sh[q][tid] += v[q];
+        if (warp == 0) {
+#pragma unroll
+            for (int q = 0; q < 3; ++q) {
+                const int64_t x = wsum[q][lane];
+                const int64_t xi = warp_incl_scan(x);
+                wsum[q][lane] = xi - x;  // exclusive warp offsets
+            }
+        }
+        __syncthreads();
+#pragma unroll
+        for (int q = 0; q < 3; ++q)
+            if (t < ntiles) tile_offs[3 * t + q] = carry[q] + wsum[q][warp] + inc[q] - v[q];
+        __syncthreads();
+        if (tid == 1023) {
+#pragma unroll
+            for (int q = 0; q < 3; ++q) carry[q] += wsum[q][31] + inc[q];
+        }
         __syncthreads();
     }
-    int64_t run[3];
-    for (int q = 0; q < 3; ++q) run[q] = sh[q][tid] - s[q];
-    for (int64_t t = b; t < e; ++t)
-        for (int q = 0; q < 3; ++q) { tile_offs[3 * t + q] = run[q]; run[q] += tile_counts[3 * t + q]; }
-    // L2 popcount + clear
-    __shared__ int64_t nchunks;
-    if (tid == 0) nchunks = 0;
-    __syncthreads();
-    int64_t pc = 0;
+    unsigned long long pc = 0;
     for (int64_t w = tid; w < nl2words; w += 1024) { pc += __popc(l2[w]); l2[w] = 0u; }
-    atomicAdd(reinterpret_cast<unsigned long long*>(&nchunks), (unsigned long long)pc);
+    pc = warp_sum(pc);
+    if (lane == 0) atomicAdd(&nchunks, pc);
     __syncthreads();
     if (tid == 0) {
-        const int64_t n_runs = sh[0][1023], n_elems = sh[2][1023];
-        totals[0] = n_runs; totals[1] = n_elems; totals[2] = nchunks; totals[3] = sh[1][1023];
+        totals[0] = carry[0]; totals[1] = carry[2]; totals[2] = (int64_t)nchunks; totals[3] = carry[1];
     }
 }
 
@@ -189,22 +202,23 @@ write_k(uint32_t* __restrict__ l1, int64_t nwords, const int64_t* __restrict__ t
         for (uint32_t m = sm; m; m &= m - 1) run_start[ks++] = gw * 32 + (__ffs(m) - 1);
         for (uint32_t m = em; m; m &= m - 1) run_end[ke++] = gw * 32 + __ffs(m);
         const int rel_el = iel - pel;  // this lane's word: first payload slot relative to oel
-        // payload: word by word, lanes = element bits; 16 words per batch so 16 coalesced loads are
-        // in flight before the stores (the gather is latency-bound otherwise)
+        // payload: word by word, lanes = element bits; all 32 words of the group are loaded before
+        // any is stored (32 coalesced 128-byte loads in flight per warp: the gather is
+        // latency-bound otherwise)
         const int64_t gbase = w0 + wb + g * 32;
 #pragma unroll 1
-        for (int q0 = 0; q0 < 32; q0 += 16) {
-            uint32_t wq[16];
-            int bq[16];
-            T v[16];
+        for (int q0 = 0; q0 < 32; q0 += 32) {
+            uint32_t wq[32];
+            int bq[32];
+            T v[32];
 #pragma unroll
-            for (int u = 0; u < 16; ++u) {
+            for (int u = 0; u < 32; ++u) {
                 wq[u] = __shfl_sync(dev::kFull, w, q0 + u);
                 bq[u] = __shfl_sync(dev::kFull, rel_el, q0 + u);
                 v[u] = ((wq[u] >> lane) & 1u) ? values[(gbase + q0 + u) * 32 + lane] : T(0);
             }
 #pragma unroll
-            for (int u = 0; u < 16; ++u)
+            for (int u = 0; u < 32; ++u)
                 if ((wq[u] >> lane) & 1u) payload[oel + bq[u] + __popc(wq[u] & ((1u << lane) - 1u))] = v[u];
         }
         os += __shfl_sync(dev::kFull, is, 31);

@@ -24,7 +24,7 @@ namespace {
 constexpr int kWarps = 8;          // warps per CTA (8 adjacent column strips)
 constexpr int kRowsPerSeg = 128;   // rows one warp marches through (2 halo rows re-read per segment)
 constexpr int kUnrollPlain = 4;    // rows loaded ahead (untracked body: 0.97 of copy peak)
-constexpr int kUnrollTrack = 8;    // tracked body: more loads in flight to hide the extra epilogue work
+constexpr int kUnrollTrack = 4;    // tracked body: same pipeline, tracking done after the row loop
 
 template <int VEC>
 struct Row {
@@ -111,11 +111,12 @@ jacobi_rows(const float* __restrict__ src, float* __restrict__ dst, int64_t cols
             } else {
                 if (nib) q[0] = o[0];
             }
-            if constexpr (TRACK) trk.mark(t.l1, t.l2, t.l2_shift, r * cols + cw);
         }
         rb[0] = rb[kUnroll];
         rb[1] = rb[kUnroll + 1];
     }
+    // fused dirty tracking of every element this warp wrote (rows [rs, re) of its strip)
+    if constexpr (TRACK) trk.mark_rows(t.l1, t.l2, t.l2_shift, rs, re, cols, cw, t.dbg);
 }
 
 template <int VEC>

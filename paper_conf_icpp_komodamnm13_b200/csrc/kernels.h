@@ -14,6 +14,7 @@ struct Track {
     uint32_t* l1;
     uint32_t* l2;
     int l2_shift;
+    int dbg;  // experiment knob (ACCMG_TRACK_DBG): bit0 skip L1 writes, bit1 skip L2 atomics
 };
 
 // Up to 64 device pointers passed by value in the kernel parameter block (no staging copy).

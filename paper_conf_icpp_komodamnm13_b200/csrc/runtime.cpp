@@ -23,6 +23,7 @@
 
 #include <algorithm>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <string>
 #include <vector>
@@ -405,7 +406,12 @@ int ensure_recv(int64_t bytes) {
 }
 
 k::Track track_of(accmg_region_s* r, int li, bool on) {
-    k::Track t{nullptr, nullptr, 0};
+    static int dbg = -1;
+    if (dbg < 0) {
+        const char* e = std::getenv("ACCMG_TRACK_DBG");
+        dbg = e ? std::atoi(e) : 0;
+    }
+    k::Track t{nullptr, nullptr, 0, dbg};
     if (!on) return t;
     t.l1 = r->trk[li].l1;
     t.l2 = r->trk[li].l2;

@@ -25,12 +25,22 @@ __device__ __forceinline__ uint32_t spread4(uint32_t x) {
     return x;
 }
 
+// Sets chunk bit c. Thousands of warps write into one chunk and all of them would hit the same
+// L2 word with an atomic, serialising at that L2 slice (measured: it doubled the tracked sweep);
+// reading the word first (L2-cached load) skips the atomic once some warp has set the bit.
+// A stale 0 only costs one redundant atomicOr; bits are cleared only by the compaction kernels,
+// which are stream-ordered after this kernel.
+__device__ __forceinline__ void set_chunk_bit(uint32_t* l2, int64_t c) {
+    const uint32_t bit = 1u << (c & 31);
+    if (!(__ldcg(l2 + (c >> 5)) & bit)) atomicOr(l2 + (c >> 5), bit);
+}
+
 // Sets the L2 (chunk) bits of elements [first, last] (inclusive, all written). `cache` holds the
 // last chunk this warp marked so steady marching re-issues nothing.
 __device__ __forceinline__ void track_l2(uint32_t* l2, int l2_shift, int64_t first, int64_t last, int64_t& cache) {
     int64_t c0 = first >> l2_shift, c1 = last >> l2_shift;
     if (c0 == c1 && c0 == cache) return;
-    for (int64_t c = c0; c <= c1; ++c) atomicOr(l2 + (c >> 5), 1u << (c & 31));
+    for (int64_t c = c0; c <= c1; ++c) set_chunk_bit(l2, c);
     cache = c1;
 }
 
@@ -116,6 +126,42 @@ struct WarpTracker {
             if (rel[q]) {
                 if (first < 0) first = 32 * q + __ffs(rel[q]) - 1;
                 last = 32 * q + 31 - __clz(rel[q]);
+            }
+        }
+    }
+
+    // All rows [rs, re) of a strip at once, after the stencil loop (keeps the tracking work out of
+    // the load pipeline): lane i handles (row, word) pair i, 32 at a time; each row's chunk range is
+    // marked once unless the previous row already marked it.
+    __device__ __forceinline__ void mark_rows(uint32_t* __restrict__ l1, uint32_t* __restrict__ l2, int l2_shift,
+                                              int64_t rs, int64_t re, int64_t cols, int64_t cw, int dbg = 0) {
+        if (first < 0) return;
+        const int lane = threadIdx.x & 31;
+        constexpr int NW = VEC + 1;
+        const int64_t n = (re - rs) * NW;
+        for (int64_t base = 0; base < n; base += 32) {  // warp-uniform trip count (shuffles)
+            const int64_t i = base + lane;
+            const bool ok = i < n;
+            const int64_t r = rs + i / NW;
+            const int q = (int)(i % NW);
+            // lane k (< VEC) holds rel[k] in `lo`; lane VEC holds 0
+            const uint32_t lo_q = __shfl_sync(kFull, lo, q);
+            const uint32_t hi_q = __shfl_sync(kFull, lo, q == 0 ? 31 : q - 1);  // lane 31 holds 0
+            if (!ok) continue;
+            const int64_t E0 = r * cols + cw;
+            const int s = (int)(E0 & 31);
+            const uint32_t v = (lo_q << s) | (s ? (hi_q >> (32 - s)) : 0u);
+            const int64_t w = (E0 >> 5) + q;
+            const bool inner = w * 32 >= E0 + first && w * 32 + 31 <= E0 + last;
+            if (v && !(dbg & 1)) {
+                if (inner) l1[w] = v;
+                else atomicOr(l1 + w, v);
+            }
+            if (q == 0 && !(dbg & 2)) {
+                const int64_t c0 = (E0 + first) >> l2_shift, c1 = (E0 + last) >> l2_shift;
+                const int64_t cp = r > rs ? (E0 - cols + last) >> l2_shift : -1;
+                for (int64_t c = c0; c <= c1; ++c)
+                    if (c != cp) set_chunk_bit(l2, c);
             }
         }
     }
