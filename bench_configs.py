@@ -156,6 +156,28 @@ def kmeans_cfg(n, iters, P, check):
     return out
 
 
+def scatter_cfg(n, P, reps):
+    """§8 row f1: irregular writes dst[idx[i]] = src[i] (idx a random permutation) to a distributed
+    array; (P-1)/P of the writes miss the writer's window and go through the system buffers."""
+    src = gen.jacobi_field(3, 16384, 0, 16384).reshape(-1)[:n].copy()
+    idx = gen.permutation(11, n)
+    dst = np.zeros(n, np.float32)
+    A.accmg_init(num_partitions=P, device=0, profile=1)
+    try:
+        regs = [A.accmg_region_create(a) for a in (src, idx, dst)]
+        WL.scatter_loop(*regs, n, n)
+        A.accmg_barrier()
+        A.accmg_reset_stats()
+        t = wall(lambda: [WL.scatter_loop(*regs, n, n) for _ in range(reps)])
+        st = A.accmg_get_stats()
+    finally:
+        A.accmg_finalize()
+    out = {"config": "f1_scatter", "P": P, "n": n, "reps": reps, "iters_per_s": n * reps / t,
+           "ms_per_loop": t / reps * 1e3, **per_loop(st, reps),
+           "write_misses_per_loop": st["write_misses"] / reps, "bytes_write_miss_per_loop": st["bytes_write_miss"] / reps}
+    return out
+
+
 def main():
     p = argparse.ArgumentParser()
     p.add_argument("--configs", default="c1,c2,c5,c3,c4")
@@ -181,6 +203,8 @@ def main():
                     emit(jacobi_cfg("c5", 32768, a.c5_sweeps, P, False, a.check and P == Ps[-1]))
                 elif cfg == "c3":
                     emit(gemm_cfg(a.gemm_n, P, a.gemm_reps, a.check))
+                elif cfg == "f1":
+                    emit(scatter_cfg(1 << 26, P, 5))
                 elif cfg == "c4":
                     if a.kmeans_n * 16 * 4 * P > (100 << 30):
                         emit({"config": cfg, "P": P, "skipped": "full-extent virtual replicas would exceed 100 GiB"})

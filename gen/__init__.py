@@ -44,6 +44,7 @@ def lib() -> ctypes.CDLL:
         L.accgen_bf16_matrix.argtypes = [u64, i64, i64, i64, i64, i32, vp, i32]
         L.accgen_kmeans_centres.argtypes = [u64, i32, i32, i32, vp]
         L.accgen_kmeans_points.argtypes = [u64, i64, i32, i32, i32, vp, i64, i64, vp, vp, i32]
+        L.accgen_permutation.argtypes = [u64, i64, vp]
         _LIB = L
     return _LIB
 
@@ -107,6 +108,13 @@ def kmeans_points(seed: int, n: int, d: int, k: int, mode: int, p0: int = 0, p1:
     lib().accgen_kmeans_points(seed, n, d, k, mode, cen.ctypes.data, p0, p1, _ptr(out),
                                lab.ctypes.data if labels else None, nthreads)
     return (out, lab, cen) if labels else out
+
+
+def permutation(seed: int, n: int) -> np.ndarray:
+    """Seeded random permutation of [0, n) as int32 (index array of the scatter workload)."""
+    out = np.empty(n, dtype=np.int32)
+    lib().accgen_permutation(seed, n, out.ctypes.data)
+    return out
 
 
 def bf16_to_f32(a: np.ndarray) -> np.ndarray:

@@ -121,3 +121,13 @@ void accgen_kmeans_points(uint64_t seed, int64_t n, int d, int k, int mode, cons
         }
     }
 }
+
+/* Random permutation of [0, n) (Fisher-Yates, swap i with u(seed, i) % (i + 1), i = n-1 .. 1):
+ * the index array of the irregular-write (scatter) workload. */
+void accgen_permutation(uint64_t seed, int64_t n, int32_t* out) {
+    for (int64_t i = 0; i < n; ++i) out[i] = (int32_t)i;
+    for (int64_t i = n - 1; i > 0; --i) {
+        int64_t j = (int64_t)(accgen_u(seed, (uint64_t)i) % (uint64_t)(i + 1));
+        int32_t t = out[i]; out[i] = out[j]; out[j] = t;
+    }
+}

@@ -128,6 +128,13 @@ typedef struct accmg_access {
  *   descs [sums RW (int64 k*d), counts RW (int64 k), centroids W (fp32 k*d)];
  *   if counts[c] > 0: cen[c][j] = (float)(((double)sums[c][j] * 2^-shift) / (double)counts[c]);
  *   then sums[c][*] = 0, counts[c] = 0.
+ * ACCMG_BODY_SCATTER: bounds ndim=1 [0,n); descs [src R (fp32 n, declared stride=1), idx R (int32 n,
+ *   declared stride=1), dst W (fp32 m, declared stride=1)]; dst[idx[i]] = src[i] (irregular writes,
+ *   the BFS class: idx[i] may fall outside the writer's window). Every write is checked against the
+ *   partition's write window (L137 §IV.D.2); a miss appends (index, value) to the partition's
+ *   system buffer, and after the kernel the buffered writes are completed in the owner's replica
+ *   (the partition whose window holds the index) — L137, L163. Indices must be distinct (L62) and
+ *   lie in some partition's window of dst.
  * ACCMG_BODY_TEST_SPARSE_WRITE: bounds ndim=1 rows [0,R); descs [in R (fp32 R*C), out W (fp32 R*C)];
  *   rows i with i % period == 0: out[i][j] = in[i][j] + 1.0f for all j (exercises L2 chunk skipping).
  */
@@ -135,12 +142,14 @@ typedef struct accmg_access {
 #define ACCMG_BODY_GEMM_BF16_F32     2
 #define ACCMG_BODY_KMEANS_ASSIGN     3
 #define ACCMG_BODY_KMEANS_UPDATE     4
+#define ACCMG_BODY_SCATTER           5
 #define ACCMG_BODY_TEST_SPARSE_WRITE 100
 
 typedef struct { int64_t rows, cols; } accmg_args_jacobi2d;
 typedef struct { int64_t M, N, K; } accmg_args_gemm;
 typedef struct { int64_t n; int32_t d, k, shift, pad; } accmg_args_kmeans;
 typedef struct { int64_t rows, cols, period; } accmg_args_sparse;
+typedef struct { int64_t n, m; } accmg_args_scatter;
 
 /* ---- statistics (E5-style breakdown, L188; device memory User/System, L249) ------------------
  * Byte counters are this process's: pulls into its partitions (receiver-counted), packets its
@@ -161,6 +170,8 @@ typedef struct accmg_stats {
     int64_t device_bytes_user;        /* replicas on this process's GPU */
     int64_t device_bytes_system;      /* bitmaps, packed/receive buffers, partials (L249-252) */
     double  ms_body, ms_compact, ms_exchange; /* profile=1: summed CUDA-event times */
+    int64_t write_misses;             /* distributed-array writes outside the writer's window (L137) */
+    int64_t bytes_write_miss;         /* (index, value) records delivered to owners: 8 + esize each */
 } accmg_stats;
 
 /* ---- entry points ------------------------------------------------------------------------- */

@@ -43,6 +43,7 @@ def lib() -> ctypes.CDLL:
         L.orc_kmeans_assign.argtypes = [vp, i64, i32, i32, vp, vp, i32]
         L.orc_kmeans_update.argtypes = [vp, i64, i32, i32, vp, vp, vp, vp]
         L.orc_kmeans_run.argtypes = [vp, i64, i32, i32, i32, vp, vp, i32]
+        L.orc_scatter.argtypes = [vp, vp, vp, i64, i64, i32, vp]
         _LIB = L
     return _LIB
 
@@ -167,3 +168,10 @@ def kmeans_run(x: np.ndarray, k: int, iters: int, nthreads: int = 0):
     m = np.empty(n, dtype=np.int32)
     lib().orc_kmeans_run(x.ctypes.data, n, d, k, iters, cen.ctypes.data, m.ctypes.data, nthreads)
     return cen, m
+
+
+def scatter(src: np.ndarray, idx: np.ndarray, dst: np.ndarray, P: int = 0):
+    """dst[idx[i]] = src[i] in place; returns per-partition write-miss counts if P > 0."""
+    miss = np.zeros(max(P, 1), dtype=np.int64)
+    lib().orc_scatter(src.ctypes.data, idx.ctypes.data, dst.ctypes.data, 0, src.size, P, miss.ctypes.data)
+    return miss[:P] if P > 0 else None

@@ -257,3 +257,22 @@ void orc_kmeans_run(const float* x, int64_t n, int d, int k, int iters, float* c
         orc_kmeans_update(x, n, d, k, member, cen, NULL, NULL);
     }
 }
+
+/* ------------------------------------------------------------------------------------ */
+/* Irregular writes to a distributed array (L137 §IV.D.2; §8 row f1; the BFS class of L173):
+ * loop i in [lo, hi): dst[idx[i]] = src[i], sequential. If P > 0, miss[g] = the number of writes by
+ * partition g's iterations whose index lies outside g's declared write window [a_g, b_g) (stride 1,
+ * the window of iterations [a_g, b_g) of the same loop bounds). pin: tests — identity and reversal
+ * permutations, scatter-then-inverse-scatter identity, brute-force miss counts. */
+void orc_scatter(const float* src, const int32_t* idx, float* dst, int64_t lo, int64_t hi, int P, int64_t* miss) {
+    for (int64_t i = lo; i < hi; ++i) dst[idx[i]] = src[i];
+    if (miss && P > 0) {
+        for (int g = 0; g < P; ++g) {
+            int64_t a, b;
+            orc_partition(lo, hi, P, g, &a, &b);
+            miss[g] = 0;
+            for (int64_t i = a; i < b; ++i)
+                if (idx[i] < a || idx[i] >= b) miss[g]++;
+        }
+    }
+}

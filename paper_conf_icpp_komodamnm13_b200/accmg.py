@@ -25,6 +25,7 @@ OK, EINVAL, ECUDA, ENCCL, ENOMEM, ESTATE, EUNSUPPORTED, ECONFLICT, EDATA = 0, -1
 XCHG_AUTO, XCHG_NCCL_ALL, XCHG_NCCL = 0, 1, 2
 R, W, RW, REDUCE_SUM = 1, 2, 3, 4
 BODY_JACOBI2D_5PT, BODY_GEMM_BF16_F32, BODY_KMEANS_ASSIGN, BODY_KMEANS_UPDATE = 1, 2, 3, 4
+BODY_SCATTER = 5
 BODY_TEST_SPARSE_WRITE = 100
 
 
@@ -62,6 +63,10 @@ class accmg_args_sparse(ctypes.Structure):
     _fields_ = [("rows", ctypes.c_int64), ("cols", ctypes.c_int64), ("period", ctypes.c_int64)]
 
 
+class accmg_args_scatter(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64), ("m", ctypes.c_int64)]
+
+
 _STAT_FIELDS = ["loops", "bytes_interpartition", "bytes_declared", "bytes_undeclared_payload",
                 "bytes_undeclared_headers", "bytes_reduce", "bytes_paper_protocol", "bytes_remote", "bytes_h2d",
                 "bytes_d2h", "body_launches", "kernel_launches", "device_bytes_user", "device_bytes_system"]
@@ -69,7 +74,8 @@ _STAT_FIELDS = ["loops", "bytes_interpartition", "bytes_declared", "bytes_undecl
 
 class accmg_stats(ctypes.Structure):
     _fields_ = [(f, ctypes.c_int64) for f in _STAT_FIELDS] + [
-        ("ms_body", ctypes.c_double), ("ms_compact", ctypes.c_double), ("ms_exchange", ctypes.c_double)]
+        ("ms_body", ctypes.c_double), ("ms_compact", ctypes.c_double), ("ms_exchange", ctypes.c_double),
+        ("write_misses", ctypes.c_int64), ("bytes_write_miss", ctypes.c_int64)]
 
 
 _vp, _i32, _i64, _sz = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_size_t

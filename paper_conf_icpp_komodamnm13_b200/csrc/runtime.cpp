@@ -105,6 +105,12 @@ struct State {
     int* d_flag = nullptr;
     uint8_t* recv = nullptr;
     int64_t recv_cap = 0;
+    // write-miss system buffers (L137): per local partition {index, value} records + counters
+    std::vector<uint64_t*> miss_recs;
+    int64_t miss_base = 0;
+    int64_t miss_cap = 0;
+    int64_t* d_miss = nullptr;       // [V] per-loop counters, [V] unused, [64] window bounds, total
+    int64_t* d_miss_total = nullptr;
     std::vector<Prof> prof;
     std::vector<cudaEvent_t> ev_free;
 };
@@ -442,6 +448,7 @@ bool body_spec(int id, BodySpec* b) {
             *b = {3, {ACCMG_RW, ACCMG_RW, ACCMG_W}, {8, 8, 4}, 1, sizeof(accmg_args_kmeans)};
             return true;
         case ACCMG_BODY_TEST_SPARSE_WRITE: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 1, sizeof(accmg_args_sparse)}; return true;
+        case ACCMG_BODY_SCATTER: *b = {3, {ACCMG_R, ACCMG_R, ACCMG_W}, {4, 4, 4}, 1, sizeof(accmg_args_scatter)}; return true;
         default: return false;
     }
 }
@@ -465,6 +472,17 @@ int validate_body(const accmg_bounds* bd, int body, const accmg_access* d, const
             if (ext(0) != a->rows * a->cols || ext(1) != a->rows * a->cols) return bad("sparse: extent != rows*cols");
             if (bd->lo[0] < 0 || bd->hi[0] > a->rows) return bad("sparse: bounds outside [0,rows)");
             if (d[0].region == d[1].region) return bad("sparse: in and out must differ");
+            return 0;
+        }
+        case ACCMG_BODY_SCATTER: {
+            auto a = static_cast<const accmg_args_scatter*>(args);
+            if (a->n < 1 || a->m < 1) return bad("scatter: n, m >= 1");
+            if (ext(0) != a->n || ext(1) != a->n || ext(2) != a->m) return bad("scatter: extents");
+            if (bd->lo[0] < 0 || bd->hi[0] > a->n) return bad("scatter: bounds outside [0,n)");
+            if (!d[2].declared)
+                return fail(ACCMG_EUNSUPPORTED, "scatter: dst must be a distributed (declared) array", false);
+            if (S.use_nccl && S.W > 1)
+                return fail(ACCMG_EUNSUPPORTED, "scatter: write misses need the P2P transport", false);
             return 0;
         }
         case ACCMG_BODY_GEMM_BF16_F32: {
@@ -514,6 +532,13 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
         case ACCMG_BODY_TEST_SPARSE_WRITE: {
             auto x = static_cast<const accmg_args_sparse*>(args);
             e = k::sparse_rows((const float*)P(0), (float*)P(1), x->rows, x->cols, a, b, x->period, T(1), S.stream, L);
+            break;
+        }
+        case ACCMG_BODY_SCATTER: {
+            IntervalSet w = window(d[2], a, b, d[2].region->extent);
+            const int64_t wlo = w.empty() ? 0 : w.items()[0].lo, whi = w.empty() ? 0 : w.items()[0].hi;
+            e = k::scatter_body((const float*)P(0), (const int32_t*)P(1), (float*)P(2), a, b, wlo, whi,
+                                S.miss_recs[li], S.d_miss + li, S.stream, L);
             break;
         }
         case ACCMG_BODY_GEMM_BF16_F32: {
@@ -824,6 +849,9 @@ int accmg_init(const accmg_config* cfg) {
     TRY(dmalloc((void**)&S.scratch, 2 * k::kScatterBlocks * 8, true));
     TRY(dmalloc((void**)&S.d_sizes, (size_t)4 * 8 * 16 * S.P * (S.W + 1), true));
     TRY(dmalloc((void**)&S.d_flag, 16, true));
+    TRY(dmalloc((void**)&S.d_miss, sizeof(int64_t) * 4 * 64, true));
+    S.d_miss_total = S.d_miss + 3 * 64;
+    CUDA_TRY(cudaMemsetAsync(S.d_miss, 0, sizeof(int64_t) * 4 * 64, S.stream));
     CUDA_TRY(cudaHostAlloc((void**)&S.h_pin, (size_t)4 * 8 * 16 * S.P * (S.W + 1) + 64, cudaHostAllocDefault));
     CUDA_TRY(cudaMemsetAsync(S.d_flag, 0, 16, S.stream));
     if (S.p2p) {
@@ -867,6 +895,8 @@ int accmg_finalize(void) {
         dfree(S.scratch, 0, true);
         dfree(S.d_sizes, 0, true);
         dfree(S.d_flag, 0, true);
+        dfree(S.d_miss, 0, true);
+        for (auto p : S.miss_recs) dfree(p, 0, true);
         dfree(S.recv, 0, true);
         if (S.h_pin) cudaFreeHost(S.h_pin);
         for (auto& p : S.prof) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
@@ -1003,6 +1033,18 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
                     for (int g = 0; g < S.P; ++g) r->gpartial[g] = static_cast<int64_t*>(all[g]);
                 }
             }
+        if (body_id == ACCMG_BODY_SCATTER) {
+            int64_t cap = 1;
+            for (int g = 0; g < S.P; ++g) cap = std::max(cap, cb[g] - ca[g]);
+            if (cap > S.miss_cap) {
+                CUDA_TRY(cudaStreamSynchronize(S.stream));
+                for (auto p : S.miss_recs) dfree(p, S.miss_cap * 16, true);
+                S.miss_recs.assign(S.V, nullptr);
+                for (int li = 0; li < S.V; ++li) TRY(dmalloc((void**)&S.miss_recs[li], cap * 16, true));
+                S.miss_cap = cap;
+            }
+            CUDA_TRY(cudaMemsetAsync(S.d_miss, 0, sizeof(int64_t) * S.V, S.stream));
+        }
         // 4. bodies on this process's partitions
         {
             ProfScope ps(0);
@@ -1012,6 +1054,26 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
             }
         }
         // 5. coherence
+        if (body_id == ACCMG_BODY_SCATTER) {
+            // complete the buffered write misses in the owners' replicas (L137, L163): owner =
+            // the partition whose declared write window holds the index
+            ProfScope ps(2);
+            accmg_region_s* r = descs[2].region;
+            std::vector<int64_t> starts(S.P, 0);
+            int nb = 0;
+            k::PtrList dl{};
+            for (int g = 0; g < S.P; ++g) {
+                IntervalSet w = window(descs[2], ca[g], cb[g], r->extent);
+                if (w.empty()) continue;
+                starts[nb++] = w.items()[0].lo;
+                dl.p[dl.n++] = S.p2p ? (void*)r->gdev[g] : (void*)r->dev[lidx(g)];
+            }
+            CUDA_TRY(cudaMemcpyAsync(S.d_miss + 2 * 64, starts.data(), sizeof(int64_t) * nb, cudaMemcpyHostToDevice,
+                                     S.stream));
+            for (int li = 0; li < S.V; ++li)
+                CUDA_TRY(k::apply_misses(S.miss_recs[li], S.d_miss + li, S.miss_cap, dl, S.d_miss + 2 * 64, nb,
+                                         S.d_miss_total, S.stream, &S.st.kernel_launches));
+        }
         if (!tracked_regs.empty()) TRY(propagate_dirty(tracked_regs));
         for (int i = 0; i < n_descs; ++i)
             if (descs[i].mode == ACCMG_REDUCE_SUM) TRY(merge_reduce(descs[i].region));
@@ -1102,14 +1164,22 @@ int accmg_get_stats(accmg_stats* out) {
     if (!S.dry) {
         TRY(collect_prof());
         TRY(check_data_flag());
+        int64_t misses = 0;
+        CUDA_TRY(cudaMemcpy(&misses, S.d_miss_total, sizeof(int64_t), cudaMemcpyDeviceToHost));
+        S.st.write_misses = misses - S.miss_base;
+        S.st.bytes_write_miss = S.st.write_misses * 12;  // int64 index + fp32 value delivered
     }
     *out = S.st;
+    out->bytes_interpartition += out->bytes_write_miss;
     return 0;
 }
 
 int accmg_reset_stats(void) {
     GUARD();
-    if (!S.dry) TRY(collect_prof());
+    if (!S.dry) {
+        TRY(collect_prof());
+        CUDA_TRY(cudaMemcpy(&S.miss_base, S.d_miss_total, sizeof(int64_t), cudaMemcpyDeviceToHost));
+    }
     const int64_t u = S.st.device_bytes_user, sy = S.st.device_bytes_system;
     S.st = accmg_stats{};
     S.st.device_bytes_user = u;

@@ -83,3 +83,11 @@ def gemm_descs(rA, rB, rC, M: int, N: int, K: int):
 def gemm_loop(rA, rB, rC, M: int, N: int, K: int) -> None:
     A.accmg_loop_launch(A.bounds([0, 0], [M, N]), A.BODY_GEMM_BF16_F32, gemm_descs(rA, rB, rC, M, N, K),
                         A.accmg_args_gemm(M, N, K))
+
+
+def scatter_loop(rsrc, ridx, rdst, n: int, m: int) -> None:
+    """One irregular-write loop dst[idx[i]] = src[i]: src and idx distributed by iteration
+    (stride 1), dst distributed by owner window (stride 1); misses go through the system buffers."""
+    A.accmg_loop_launch(A.bounds([0], [n]), A.BODY_SCATTER,
+                        [A.access(rsrc, A.R, True, 1, 0, 0), A.access(ridx, A.R, True, 1, 0, 0),
+                         A.access(rdst, A.W, True, 1, 0, 0)], A.accmg_args_scatter(n, m))

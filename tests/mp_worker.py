@@ -37,6 +37,15 @@ def main():
         x = gen.kmeans_points(5, 20000, 16, 32, gen.KM_OVERLAP)
         cen, mem = WL.kmeans_run(x, 32, 5)
         res = {"cen": cen, "mem": mem}
+    if work == "scatter":
+        n = 50000
+        src = gen.jacobi_field(3, 317, 0, 317).reshape(-1)[:n].copy()
+        idx = gen.permutation(11, n)
+        dst = np.zeros(n, np.float32)
+        regs = [A.accmg_region_create(a) for a in (src, idx, dst)]
+        WL.scatter_loop(*regs, n, n)
+        A.accmg_sync_to_host(regs[2])
+        res = {"dst": dst}
     st = A.accmg_get_stats()
     if work.startswith("jacobi"):
         st = {"total": st, **loops}

@@ -172,3 +172,16 @@ def test_state_errors():
     with pytest.raises(A.AccmgError) as e:
         A.accmg_init(num_partitions=1, device=-1, dirty_chunk_bytes=1000)
     assert e.value.code == A.EINVAL
+
+
+def test_scatter_requires_declared_dst(dry):
+    dry(2)
+    n = 64
+    regs = [A.accmg_region_create(a) for a in (np.zeros(n, np.float32), np.zeros(n, np.int32), np.zeros(n, np.float32))]
+    with pytest.raises(A.AccmgError) as e:
+        A.accmg_loop_launch(A.bounds([0], [n]), A.BODY_SCATTER,
+                            [A.access(regs[0], A.R, True, 1), A.access(regs[1], A.R, True, 1), A.access(regs[2], A.W)],
+                            A.accmg_args_scatter(n, n))
+    assert e.value.code == A.EUNSUPPORTED
+    from paper_conf_icpp_komodamnm13_b200 import workloads as WL
+    WL.scatter_loop(*regs, n, n)   # declared: accepted (dry run: planning only)

@@ -62,3 +62,16 @@ def test_kmeans_two_processes(tmp_path):
         assert np.array_equal(np.load(tmp_path / f"rank{r}_cen.npy"), ocen)
         assert np.array_equal(np.load(tmp_path / f"rank{r}_mem.npy"), omem)
     assert sum(s["bytes_reduce"] for s in stats) == 5 * 2 * 3 * (32 * 16 + 32) * 8
+
+
+def test_scatter_two_processes(tmp_path):
+    """Write misses completed directly in a peer process's replica through its IPC mapping."""
+    n = 50000
+    src = gen.jacobi_field(3, 317, 0, 317).reshape(-1)[:n].copy()
+    idx = gen.permutation(11, n)
+    exp = np.zeros(n, np.float32)
+    miss = oracle.scatter(src, idx, exp, P=4)
+    stats = _launch(2, 2, "scatter", tmp_path)
+    for r in range(2):
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_dst.npy"), exp)
+    assert sum(s["write_misses"] for s in stats) == int(miss.sum())

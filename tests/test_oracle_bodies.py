@@ -204,3 +204,31 @@ def test_dependence_cone_window_reproduces_full_field():
     for (i, j) in [(1, 1), (N - 2, N - 2), (50, 100), (1, N - 2), (100, 1), (8, 8)]:
         F, G, i0, j0 = _oracle_point_window(2, N, S, i, j)
         assert A[i, j] == F[i - i0, j - j0] and B[i, j] == G[i - i0, j - j0]
+
+
+# ---- irregular writes (write misses, L137) ------------------------------------------------------
+def test_scatter_pins():
+    n = 1000
+    src = np.arange(n, dtype=np.float32) * np.float32(0.5)
+    ident = np.arange(n, dtype=np.int32)
+    dst = np.zeros(n, np.float32)
+    miss = oracle.scatter(src, ident, dst, P=4)
+    assert np.array_equal(dst, src) and miss.tolist() == [0, 0, 0, 0]   # no write leaves its window
+    rev = ident[::-1].copy()
+    dst2 = np.zeros(n, np.float32)
+    miss2 = oracle.scatter(src, rev, dst2, P=2)
+    assert np.array_equal(dst2, src[::-1]) and miss2.tolist() == [500, 500]  # every write crosses
+    perm = gen.permutation(9, n)
+    assert np.array_equal(np.sort(perm), ident)                           # a permutation
+    d3 = np.zeros(n, np.float32)
+    oracle.scatter(src, perm, d3)
+    inv = np.empty(n, np.int32)
+    inv[perm] = ident                                                      # inverse permutation
+    back = np.zeros(n, np.float32)
+    oracle.scatter(d3, inv, back)
+    assert np.array_equal(back, src)
+    # brute-force miss counts at P=3
+    m3 = oracle.scatter(src, perm, np.zeros(n, np.float32), P=3)
+    for g in range(3):
+        a, b = oracle.partition(0, n, 3, g)
+        assert m3[g] == sum(1 for i in range(a, b) if not (a <= perm[i] < b))
