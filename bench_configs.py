@@ -156,6 +156,30 @@ def kmeans_cfg(n, iters, P, check):
     return out
 
 
+def jacobi3d_cfg(n, sweeps, P, declared=True):
+    """§8 row f2: 3-D 7-point Jacobi on n^3 fp32, plane-block partition, TMA-staged tiles."""
+    Ah = gen.field3d(6, n, n, n)
+    Bh = Ah.copy()
+    A.accmg_init(num_partitions=P, device=0, profile=1)
+    try:
+        rA, rB = A.accmg_region_create(Ah), A.accmg_region_create(Bh)
+        for s in range(2):
+            WL.jacobi3d_sweep(rA, rB, s, n, n, n, declared)
+        A.accmg_barrier()
+        A.accmg_reset_stats()
+        t = wall(lambda: [WL.jacobi3d_sweep(rA, rB, s, n, n, n, declared) for s in range(2, 2 + sweeps)])
+        st = A.accmg_get_stats()
+    finally:
+        A.accmg_finalize()
+    pts = (n - 2) ** 3
+    ms_launch = st["ms_body"] / max(st["body_launches"], 1)
+    out = {"config": "f2_jacobi3d", "P": P, "n": n, "sweeps": sweeps, "declared": declared,
+           "iters_per_s": pts * sweeps / t, "ms_per_loop": t / sweeps * 1e3, **per_loop(st, sweeps),
+           "body_GBs": 8 * pts / P / (ms_launch / 1e3) / 1e9}
+    out["body_frac_of_measured_hbm"] = out["body_GBs"] / peaks()["hbm_gbs"]
+    return out
+
+
 def scatter_cfg(n, P, reps):
     """§8 row f1: irregular writes dst[idx[i]] = src[i] (idx a random permutation) to a distributed
     array; (P-1)/P of the writes miss the writer's window and go through the system buffers."""
@@ -203,6 +227,8 @@ def main():
                     emit(jacobi_cfg("c5", 32768, a.c5_sweeps, P, False, a.check and P == Ps[-1]))
                 elif cfg == "c3":
                     emit(gemm_cfg(a.gemm_n, P, a.gemm_reps, a.check))
+                elif cfg == "f2":
+                    emit(jacobi3d_cfg(1024, 20, P))
                 elif cfg == "f1":
                     emit(scatter_cfg(1 << 26, P, 5))
                 elif cfg == "c4":

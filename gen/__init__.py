@@ -45,6 +45,7 @@ def lib() -> ctypes.CDLL:
         L.accgen_kmeans_centres.argtypes = [u64, i32, i32, i32, vp]
         L.accgen_kmeans_points.argtypes = [u64, i64, i32, i32, i32, vp, i64, i64, vp, vp, i32]
         L.accgen_permutation.argtypes = [u64, i64, vp]
+        L.accgen_field3d.argtypes = [u64, i64, i64, i64, i64, i64, vp, i32]
         _LIB = L
     return _LIB
 
@@ -108,6 +109,16 @@ def kmeans_points(seed: int, n: int, d: int, k: int, mode: int, p0: int = 0, p1:
     lib().accgen_kmeans_points(seed, n, d, k, mode, cen.ctypes.data, p0, p1, _ptr(out),
                                lab.ctypes.data if labels else None, nthreads)
     return (out, lab, cen) if labels else out
+
+
+def field3d(seed: int, n0: int, n1: int, n2: int, i0: int = 0, i1: int | None = None, out=None,
+            nthreads: int = 0):
+    """Planes [i0, i1) of the 3-D Jacobi field (plane 0 = 1, other faces 0, interior U[0,1))."""
+    i1 = n0 if i1 is None else i1
+    if out is None:
+        out = np.empty((i1 - i0, n1, n2), dtype=np.float32)
+    lib().accgen_field3d(seed, n0, n1, n2, i0, i1, _ptr(out), nthreads)
+    return out
 
 
 def permutation(seed: int, n: int) -> np.ndarray:

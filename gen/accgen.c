@@ -131,3 +131,20 @@ void accgen_permutation(uint64_t seed, int64_t n, int32_t* out) {
         int32_t t = out[i]; out[i] = out[j]; out[j] = t;
     }
 }
+
+/* 3-D Jacobi field (row f2): n0 x n1 x n2 fp32, planes [i0, i1) written to out. Plane 0 = 1.0; the
+ * other boundary faces 0; interior (i,j,k) = (u(seed, (i*n1+j)*n2+k) >> 40) * 2^-24. */
+void accgen_field3d(uint64_t seed, int64_t n0, int64_t n1, int64_t n2, int64_t i0, int64_t i1, float* out,
+                    int nthreads) {
+    #pragma omp parallel for schedule(static) num_threads(nthr(nthreads))
+    for (int64_t i = i0; i < i1; ++i)
+        for (int64_t j = 0; j < n1; ++j)
+            for (int64_t k = 0; k < n2; ++k) {
+                const int64_t x = (i * n1 + j) * n2 + k;
+                float v;
+                if (i == 0) v = 1.0f;
+                else if (i == n0 - 1 || j == 0 || j == n1 - 1 || k == 0 || k == n2 - 1) v = 0.0f;
+                else v = unit24(accgen_u(seed, (uint64_t)x));
+                out[x - i0 * n1 * n2] = v;
+            }
+}

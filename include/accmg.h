@@ -128,6 +128,11 @@ typedef struct accmg_access {
  *   descs [sums RW (int64 k*d), counts RW (int64 k), centroids W (fp32 k*d)];
  *   if counts[c] > 0: cen[c][j] = (float)(((double)sums[c][j] * 2^-shift) / (double)counts[c]);
  *   then sums[c][*] = 0, counts[c] = 0.
+ * ACCMG_BODY_JACOBI3D_7PT: bounds ndim=3 [1,n0-1) x [1,n1-1) x [1,n2-1) (or a sub-box); descs
+ *   [src R (fp32 n0*n1*n2), dst W (fp32 n0*n1*n2)]; n2 % 4 == 0;
+ *   dst[i][j][k] = ((((u+d) + (n+s)) + ((w+e) + (c+c))) * 0.125f with u/d = src[i-1/i+1][j][k],
+ *   n/s = src[i][j-1/j+1][k], w/e = src[i][j][k-1/k+1], c = src[i][j][k] (multi-dimensional
+ *   stencil of L256; planes are partitioned: declared src stride=n1*n2 left=right=n1*n2).
  * ACCMG_BODY_SCATTER: bounds ndim=1 [0,n); descs [src R (fp32 n, declared stride=1), idx R (int32 n,
  *   declared stride=1), dst W (fp32 m, declared stride=1)]; dst[idx[i]] = src[i] (irregular writes,
  *   the BFS class: idx[i] may fall outside the writer's window). Every write is checked against the
@@ -143,6 +148,7 @@ typedef struct accmg_access {
 #define ACCMG_BODY_KMEANS_ASSIGN     3
 #define ACCMG_BODY_KMEANS_UPDATE     4
 #define ACCMG_BODY_SCATTER           5
+#define ACCMG_BODY_JACOBI3D_7PT      6
 #define ACCMG_BODY_TEST_SPARSE_WRITE 100
 
 typedef struct { int64_t rows, cols; } accmg_args_jacobi2d;
@@ -150,6 +156,7 @@ typedef struct { int64_t M, N, K; } accmg_args_gemm;
 typedef struct { int64_t n; int32_t d, k, shift, pad; } accmg_args_kmeans;
 typedef struct { int64_t rows, cols, period; } accmg_args_sparse;
 typedef struct { int64_t n, m; } accmg_args_scatter;
+typedef struct { int64_t n0, n1, n2; } accmg_args_jacobi3d;
 
 /* ---- statistics (E5-style breakdown, L188; device memory User/System, L249) ------------------
  * Byte counters are this process's: pulls into its partitions (receiver-counted), packets its

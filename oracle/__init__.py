@@ -44,6 +44,8 @@ def lib() -> ctypes.CDLL:
         L.orc_kmeans_update.argtypes = [vp, i64, i32, i32, vp, vp, vp, vp]
         L.orc_kmeans_run.argtypes = [vp, i64, i32, i32, i32, vp, vp, i32]
         L.orc_scatter.argtypes = [vp, vp, vp, i64, i64, i32, vp]
+        L.orc_jacobi3d_sweep.argtypes = [vp, vp, i64, i64, i64, i32, vp, i32]
+        L.orc_jacobi3d_run.argtypes = [vp, vp, i64, i64, i64, i32, i32]
         _LIB = L
     return _LIB
 
@@ -175,3 +177,15 @@ def scatter(src: np.ndarray, idx: np.ndarray, dst: np.ndarray, P: int = 0):
     miss = np.zeros(max(P, 1), dtype=np.int64)
     lib().orc_scatter(src.ctypes.data, idx.ctypes.data, dst.ctypes.data, 0, src.size, P, miss.ctypes.data)
     return miss[:P] if P > 0 else None
+
+
+def jacobi3d_sweep(src: np.ndarray, dst: np.ndarray, P: int = 1, track: bool = False, nthreads: int = 0):
+    n0, n1, n2 = src.shape
+    bms = np.zeros((P, nwords(src.size)), dtype=np.uint32) if track else None
+    lib().orc_jacobi3d_sweep(src.ctypes.data, dst.ctypes.data, n0, n1, n2, P, _p(bms), nthreads)
+    return bms
+
+
+def jacobi3d_run(A: np.ndarray, B: np.ndarray, S: int, nthreads: int = 0) -> None:
+    n0, n1, n2 = A.shape
+    lib().orc_jacobi3d_run(A.ctypes.data, B.ctypes.data, n0, n1, n2, S, nthreads)

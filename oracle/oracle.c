@@ -276,3 +276,39 @@ void orc_scatter(const float* src, const int32_t* idx, float* dst, int64_t lo, i
         }
     }
 }
+
+/* ------------------------------------------------------------------------------------ */
+/* 3-D 7-point Jacobi sweep (§8 row f2; multi-dimensional stencils, L256; reading in DESIGN.md):
+ * for i in [1,n0-1) (partitioned), j in [1,n1-1), k in [1,n2-1):
+ *   dst = ((((u + d) + (n + s)) + ((w + e) + (c + c))) * 0.125f
+ * u/d = src[i-1/i+1][j][k], n/s = src[i][j-1/j+1][k], w/e = src[i][j][k-1/k+1], c = src[i][j][k].
+ * Bitmaps as for the 2-D sweep (plane i belongs to partition orc_owner(1, n0-1, P, i)).
+ * pin: tests — constant and integer-linear fixed points, axis reflections, dyadic exact rationals. */
+void orc_jacobi3d_sweep(const float* src, float* dst, int64_t n0, int64_t n1, int64_t n2, int P, uint32_t* bitmaps,
+                        int nthreads) {
+    int64_t E = n0 * n1 * n2, nwords = (E + 31) / 32, pl = n1 * n2;
+    #pragma omp parallel for schedule(static) num_threads(nthr(nthreads))
+    for (int64_t i = 1; i < n0 - 1; ++i)
+        for (int64_t j = 1; j < n1 - 1; ++j)
+            for (int64_t k = 1; k < n2 - 1; ++k) {
+                int64_t x = i * pl + j * n2 + k;
+                float ud = src[x - pl] + src[x + pl];
+                float ns = src[x - n2] + src[x + n2];
+                float we = src[x - 1] + src[x + 1];
+                float cc = src[x] + src[x];
+                dst[x] = ((ud + ns) + (we + cc)) * 0.125f;
+            }
+    if (bitmaps)
+        for (int64_t i = 1; i < n0 - 1; ++i) {
+            int g = orc_owner(1, n0 - 1, P, i);
+            for (int64_t j = 1; j < n1 - 1; ++j)
+                for (int64_t k = 1; k < n2 - 1; ++k) set_bit(bitmaps + (int64_t)g * nwords, i * pl + j * n2 + k);
+        }
+}
+
+void orc_jacobi3d_run(float* A, float* B, int64_t n0, int64_t n1, int64_t n2, int S, int nthreads) {
+    for (int s = 0; s < S; ++s) {
+        if (s % 2 == 0) orc_jacobi3d_sweep(A, B, n0, n1, n2, 1, NULL, nthreads);
+        else orc_jacobi3d_sweep(B, A, n0, n1, n2, 1, NULL, nthreads);
+    }
+}

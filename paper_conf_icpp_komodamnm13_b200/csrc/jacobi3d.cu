@@ -1,0 +1,152 @@
+// Loop body: 3-D 7-point Jacobi sweep (§8 row f2: the multi-dimensional stencils of L256, with
+// plane-block partitioning — declared windows stride = n1*n2, left = right = n1*n2).
+//
+//   dst[i][j][k] = ((((u + d) + (n + s)) + ((w + e) + (c + c))) * 0.125f
+//   u/d = src[i-1/i+1][j][k], n/s = src[i][j-1/j+1][k], w/e = src[i][j][k-1/k+1], c = src[i][j][k]
+//   (damped Jacobi of the 3-D Laplacian; reading in DESIGN.md), interior points only.
+//
+// TMA-staged shared-memory tiles (B200): each CTA owns a 16 (j) x 128 (k) column of the domain and
+// marches down a segment of planes i. One thread issues cp.async.bulk.tensor.3d loads of
+// 18 x 136-float tiles (the tile plus its j and k halo) of successive planes into a 4-stage ring
+// completed on mbarriers, so three planes are resident while the fourth streams in; every input
+// element crosses HBM once (+ the 2 halo rows / 2 halo planes per segment, L2-resident). Threads
+// read the 7 operands from shared memory (horizontal neighbours by warp shuffle), use explicit
+// round-to-nearest adds in the stated order, and store 128-bit vectors of interior points. The
+// optional fused epilogue sets the two-level dirty bits (L133-135).
+#include "kernels.h"
+#include "tma_dev.cuh"
+#include "tma_host.h"
+#include "track.cuh"
+
+namespace accmg {
+namespace k {
+namespace {
+
+constexpr int TK = 128;          // k columns per CTA (32 lanes x float4)
+constexpr int TJ = 16;           // j rows per CTA (8 warps x 2 rows)
+constexpr int BOXK = TK + 8;     // k halo: 4 on each side (keeps 16-byte alignment)
+constexpr int BOXJ = TJ + 2;     // j halo: 1 on each side
+constexpr int kStages = 4;
+constexpr int kPlaneSeg = 32;    // planes per CTA
+constexpr int kTileFloats = BOXK * BOXJ;
+constexpr uint32_t kTileBytes = kTileFloats * 4;
+constexpr int kStageFloats = ((kTileBytes + 127) / 128) * 32;  // TMA destinations are 128-byte aligned
+
+__device__ __forceinline__ float s7(float u, float d, float n, float s, float w, float e, float c) {
+    const float ud = __fadd_rn(u, d), ns = __fadd_rn(n, s), we = __fadd_rn(w, e), cc = __fadd_rn(c, c);
+    return __fmul_rn(__fadd_rn(__fadd_rn(ud, ns), __fadd_rn(we, cc)), 0.125f);
+}
+
+template <bool TRACK>
+__global__ void __launch_bounds__(256)
+jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, int64_t n1, int64_t n2, int64_t i0,
+             int64_t i1, int64_t jl, int64_t jh, int64_t kl, int64_t kh, int64_t kbase, Track t) {
+    __shared__ __align__(128) float tile[kStages][kStageFloats];
+    __shared__ __align__(8) uint64_t bar[kStages];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int64_t k0 = kbase + (int64_t)blockIdx.x * TK;
+    const int64_t j0 = jl + (int64_t)blockIdx.y * TJ;
+    const int64_t ps = i0 + (int64_t)blockIdx.z * kPlaneSeg;
+    const int64_t pe = ps + kPlaneSeg < i1 ? ps + kPlaneSeg : i1;
+    const int count = (int)(pe - ps + 2);  // planes ps-1 .. pe
+    if (tid == 0) {
+        for (int s = 0; s < kStages; ++s) dev::mbar_init(&bar[s], 1);
+        dev::mbar_fence_init();
+        dev::tma_prefetch_desc(&map);
+        for (int q = 0; q < kStages && q < count; ++q) {  // all stages free at the start
+            dev::mbar_expect_tx(&bar[q], kTileBytes);
+            dev::tma_load_3d(&map, &bar[q], tile[q], (int)(k0 - 4), (int)(j0 - 1), (int)(ps - 1 + q));
+        }
+    }
+    __syncthreads();
+    // this thread's columns and rows
+    const int64_t k = k0 + 4 * lane;
+    unsigned nib = 0;
+#pragma unroll
+    for (int c = 0; c < 4; ++c) nib |= (k + c >= kl && k + c < kh) ? (1u << c) : 0u;
+    const bool full = nib == 0xFu;
+    const int col = 4 + 4 * lane;  // tile column of k
+    dev::WarpTracker<4> trk;
+    if constexpr (TRACK) trk.init(nib);
+    dev::mbar_wait(&bar[0], 0);
+    dev::mbar_wait(&bar[1], 0);
+    for (int64_t i = ps; i < pe; ++i) {
+        const int q = (int)(i - ps) + 2;  // plane i+1
+        dev::mbar_wait(&bar[q % kStages], (uint32_t)((q / kStages) & 1));
+        const float* P0 = tile[(q - 2) % kStages];
+        const float* P1 = tile[(q - 1) % kStages];
+        const float* P2 = tile[q % kStages];
+#pragma unroll
+        for (int r = 0; r < 2; ++r) {
+            const int tr = 2 * warp + r + 1;  // tile row of j
+            const int64_t j = j0 + tr - 1;
+            const float4 C = *reinterpret_cast<const float4*>(P1 + tr * BOXK + col);
+            const float4 N = *reinterpret_cast<const float4*>(P1 + (tr - 1) * BOXK + col);
+            const float4 S = *reinterpret_cast<const float4*>(P1 + (tr + 1) * BOXK + col);
+            const float4 U = *reinterpret_cast<const float4*>(P0 + tr * BOXK + col);
+            const float4 D = *reinterpret_cast<const float4*>(P2 + tr * BOXK + col);
+            float w = __shfl_up_sync(dev::kFull, C.w, 1);
+            float e = __shfl_down_sync(dev::kFull, C.x, 1);
+            if (lane == 0) w = P1[tr * BOXK + col - 1];
+            if (lane == 31) e = P1[tr * BOXK + col + 4];
+            const bool rowok = j < jh;  // warp-uniform
+            if (rowok) {
+                float o[4];
+                o[0] = s7(U.x, D.x, N.x, S.x, w, C.y, C.x);
+                o[1] = s7(U.y, D.y, N.y, S.y, C.x, C.z, C.y);
+                o[2] = s7(U.z, D.z, N.z, S.z, C.y, C.w, C.z);
+                o[3] = s7(U.w, D.w, N.w, S.w, C.z, e, C.w);
+                float* out = dst + (i * n1 + j) * n2 + k;
+                if (full) {
+                    *reinterpret_cast<float4*>(out) = make_float4(o[0], o[1], o[2], o[3]);
+                } else {
+#pragma unroll
+                    for (int c = 0; c < 4; ++c)
+                        if (nib & (1u << c)) out[c] = o[c];
+                }
+                if constexpr (TRACK) trk.mark(t.l1, t.l2, t.l2_shift, (i * n1 + j) * n2 + k0);
+            }
+        }
+        __syncthreads();  // every thread is done with plane i-1 (stage (q-2) % kStages)
+        if (tid == 0 && q + 2 < count) {
+            const int qn = q + 2;
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            dev::mbar_expect_tx(&bar[qn % kStages], kTileBytes);
+            dev::tma_load_3d(&map, &bar[qn % kStages], tile[qn % kStages], (int)(k0 - 4), (int)(j0 - 1),
+                             (int)(ps - 1 + qn));
+        }
+    }
+}
+
+}  // namespace
+
+cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64_t n2, int64_t i0, int64_t i1,
+                     int64_t jl, int64_t jh, int64_t kl, int64_t kh, Track t, cudaStream_t s, int64_t* launches) {
+    if (i1 <= i0 || jh <= jl || kh <= kl) return cudaSuccess;
+    if (n2 % 4 != 0 || (reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) % 16 != 0 ||
+        n0 >= (1ll << 31) || n1 >= (1ll << 31) || n2 >= (1ll << 31))
+        return cudaErrorNotSupported;
+    auto fn = tma_encode_fn();
+    if (!fn) return cudaErrorNotSupported;
+    CUtensorMap map;
+    cuuint64_t dims[3] = {(cuuint64_t)n2, (cuuint64_t)n1, (cuuint64_t)n0};
+    cuuint64_t strides[2] = {(cuuint64_t)n2 * 4, (cuuint64_t)n1 * n2 * 4};
+    cuuint32_t box[3] = {BOXK, BOXJ, 1};
+    cuuint32_t es[3] = {1, 1, 1};
+    if (fn(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(src), dims, strides, box, es,
+           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+        return cudaErrorNotSupported;
+    const int64_t kbase = (kl / 4) * 4;
+    dim3 grid((unsigned)((kh - kbase + TK - 1) / TK), (unsigned)((jh - jl + TJ - 1) / TJ),
+              (unsigned)((i1 - i0 + kPlaneSeg - 1) / kPlaneSeg));
+    if (t.l1)
+        jacobi3d_tma<true><<<grid, 256, 0, s>>>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, kbase, t);
+    else
+        jacobi3d_tma<false><<<grid, 256, 0, s>>>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, kbase, t);
+    if (launches) *launches += 1;
+    return cudaGetLastError();
+}
+
+}  // namespace k
+}  // namespace accmg

@@ -30,6 +30,11 @@ struct PtrList {
 cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
                      int64_t c0, int64_t c1, Track t, int impl, cudaStream_t s, int64_t* launches);
 
+// 3-D 7-point Jacobi (TMA-staged tiles) on planes [i0, i1) x rows [jl, jh) x cols [kl, kh) of an
+// n0 x n1 x n2 fp32 array; needs n2 % 4 == 0 (else cudaErrorNotSupported).
+cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64_t n2, int64_t i0, int64_t i1,
+                     int64_t jl, int64_t jh, int64_t kl, int64_t kh, Track t, cudaStream_t s, int64_t* launches);
+
 // Test body: rows i in [r0, r1) with i % period == 0: out[i][:] = in[i][:] + 1.0f.
 cudaError_t sparse_rows(const float* in, float* out, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
                         int64_t period, Track t, cudaStream_t s, int64_t* launches);

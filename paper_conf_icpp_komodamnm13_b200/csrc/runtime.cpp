@@ -449,6 +449,7 @@ bool body_spec(int id, BodySpec* b) {
             return true;
         case ACCMG_BODY_TEST_SPARSE_WRITE: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 1, sizeof(accmg_args_sparse)}; return true;
         case ACCMG_BODY_SCATTER: *b = {3, {ACCMG_R, ACCMG_R, ACCMG_W}, {4, 4, 4}, 1, sizeof(accmg_args_scatter)}; return true;
+        case ACCMG_BODY_JACOBI3D_7PT: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 3, sizeof(accmg_args_jacobi3d)}; return true;
         default: return false;
     }
 }
@@ -472,6 +473,18 @@ int validate_body(const accmg_bounds* bd, int body, const accmg_access* d, const
             if (ext(0) != a->rows * a->cols || ext(1) != a->rows * a->cols) return bad("sparse: extent != rows*cols");
             if (bd->lo[0] < 0 || bd->hi[0] > a->rows) return bad("sparse: bounds outside [0,rows)");
             if (d[0].region == d[1].region) return bad("sparse: in and out must differ");
+            return 0;
+        }
+        case ACCMG_BODY_JACOBI3D_7PT: {
+            auto a = static_cast<const accmg_args_jacobi3d*>(args);
+            if (a->n0 < 3 || a->n1 < 3 || a->n2 < 3) return bad("jacobi3d: n0, n1, n2 >= 3");
+            const int64_t E = a->n0 * a->n1 * a->n2;
+            if (ext(0) != E || ext(1) != E) return bad("jacobi3d: region extent != n0*n1*n2");
+            if (bd->lo[0] < 1 || bd->hi[0] > a->n0 - 1 || bd->lo[1] < 1 || bd->hi[1] > a->n1 - 1 || bd->lo[2] < 1 ||
+                bd->hi[2] > a->n2 - 1)
+                return bad("jacobi3d: bounds must lie in the interior");
+            if (d[0].region == d[1].region) return bad("jacobi3d: src and dst must differ");
+            if (a->n2 % 4 != 0) return fail(ACCMG_EUNSUPPORTED, "jacobi3d: needs n2 % 4 == 0", false);
             return 0;
         }
         case ACCMG_BODY_SCATTER: {
@@ -532,6 +545,12 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
         case ACCMG_BODY_TEST_SPARSE_WRITE: {
             auto x = static_cast<const accmg_args_sparse*>(args);
             e = k::sparse_rows((const float*)P(0), (float*)P(1), x->rows, x->cols, a, b, x->period, T(1), S.stream, L);
+            break;
+        }
+        case ACCMG_BODY_JACOBI3D_7PT: {
+            auto x = static_cast<const accmg_args_jacobi3d*>(args);
+            e = k::jacobi3d((const float*)P(0), (float*)P(1), x->n0, x->n1, x->n2, a, b, bd->lo[1], bd->hi[1],
+                            bd->lo[2], bd->hi[2], T(1), S.stream, L);
             break;
         }
         case ACCMG_BODY_SCATTER: {

@@ -91,3 +91,26 @@ def scatter_loop(rsrc, ridx, rdst, n: int, m: int) -> None:
     A.accmg_loop_launch(A.bounds([0], [n]), A.BODY_SCATTER,
                         [A.access(rsrc, A.R, True, 1, 0, 0), A.access(ridx, A.R, True, 1, 0, 0),
                          A.access(rdst, A.W, True, 1, 0, 0)], A.accmg_args_scatter(n, m))
+
+
+def jacobi3d_sweep(rA, rB, s: int, n0: int, n1: int, n2: int, declared: bool) -> None:
+    """One 3-D 7-point sweep; planes are the partitioned outer loop: iteration i reads planes
+    i-1..i+1 (stride n1*n2, left = right = n1*n2) and writes plane i (L87 on the flattened array)."""
+    src, dst = (rA, rB) if s % 2 == 0 else (rB, rA)
+    pl = n1 * n2
+    A.accmg_loop_launch(A.bounds([1, 1, 1], [n0 - 1, n1 - 1, n2 - 1]), A.BODY_JACOBI3D_7PT,
+                        [A.access(src, A.R, declared, pl, pl, pl), A.access(dst, A.W, declared, pl, 0, 0)],
+                        A.accmg_args_jacobi3d(n0, n1, n2))
+
+
+def jacobi3d_run(Ahost, Bhost, sweeps: int, declared: bool = True):
+    n0, n1, n2 = Ahost.shape
+    rA, rB = A.accmg_region_create(Ahost), A.accmg_region_create(Bhost)
+    try:
+        for s in range(sweeps):
+            jacobi3d_sweep(rA, rB, s, n0, n1, n2, declared)
+        A.accmg_sync_to_host(rA)
+        A.accmg_sync_to_host(rB)
+    finally:
+        A.accmg_region_destroy(rA)
+        A.accmg_region_destroy(rB)

@@ -232,3 +232,40 @@ def test_scatter_pins():
     for g in range(3):
         a, b = oracle.partition(0, n, 3, g)
         assert m3[g] == sum(1 for i in range(a, b) if not (a <= perm[i] < b))
+
+
+# ---- 3-D 7-point Jacobi (row f2) ------------------------------------------------------------------
+def _sweeps3(A, S):
+    A = A.copy()
+    B = A.copy()
+    oracle.jacobi3d_run(A, B, S)
+    return A if S % 2 == 0 else B
+
+
+def test_jacobi3d_fixed_points_and_reflections():
+    c = np.full((9, 10, 12), 3.0, np.float32)
+    assert np.array_equal(_sweeps3(c, 6), c)                       # constant field
+    i, j, k = np.meshgrid(np.arange(9), np.arange(10), np.arange(12), indexing="ij")
+    lin = (2 * i - 3 * j + 5 * k + 7).astype(np.float32)           # harmonic, integer sums exact
+    assert np.array_equal(_sweeps3(lin, 6), lin)
+    rng = np.random.default_rng(1)
+    A = rng.random((8, 9, 12), dtype=np.float32)
+    out = _sweeps3(A, 5)
+    for ax in range(3):                                            # each pair (a+b) is commutative
+        assert np.array_equal(_sweeps3(np.ascontiguousarray(np.flip(A, ax)), 5), np.flip(out, ax))
+
+
+def test_jacobi3d_dyadic_exact_rationals():
+    rng = np.random.default_rng(2)
+    A = (rng.integers(0, 16, (6, 5, 7)) / 8.0).astype(np.float32)
+    F = A.astype(object)
+    F = np.vectorize(lambda v: Fraction(float(v)))(A)
+    for s in range(3):
+        G = F.copy()
+        for i in range(1, 5):
+            for j in range(1, 4):
+                for k in range(1, 6):
+                    G[i, j, k] = (F[i - 1, j, k] + F[i + 1, j, k] + F[i, j - 1, k] + F[i, j + 1, k] +
+                                  F[i, j, k - 1] + F[i, j, k + 1] + 2 * F[i, j, k]) / 8
+        F = G
+        assert np.array_equal(_sweeps3(A, s + 1).astype(np.float64), F.astype(np.float64))
