@@ -180,6 +180,29 @@ def jacobi3d_cfg(n, sweeps, P, declared=True):
     return out
 
 
+def footprint_cfg(P):
+    """§8 row f4 / Fig. 9 (L249-252): device memory per configuration — User (replicas) and
+    System (bitmaps, packed buffers, partials, miss buffers) — normalised to the P=1 User total."""
+    rows = []
+    N = 32768
+    for declared in (True, False):
+        Ah = gen.jacobi_field(2, N)
+        Bh = Ah.copy()
+        A.accmg_init(num_partitions=P, device=0)
+        try:
+            rA, rB = A.accmg_region_create(Ah), A.accmg_region_create(Bh)
+            for s in range(2):
+                WL.jacobi_sweep(rA, rB, s, N, declared)
+            st = A.accmg_get_stats()
+        finally:
+            A.accmg_finalize()
+        one = 2 * N * N * 4
+        rows.append({"config": "f4_footprint", "workload": "c2" if declared else "c5", "P": P,
+                     "user_bytes": st["device_bytes_user"], "system_bytes": st["device_bytes_system"],
+                     "user_rel_1gpu": st["device_bytes_user"] / one, "system_rel_1gpu": st["device_bytes_system"] / one})
+    return rows
+
+
 def scatter_cfg(n, P, reps):
     """§8 row f1: irregular writes dst[idx[i]] = src[i] (idx a random permutation) to a distributed
     array; (P-1)/P of the writes miss the writer's window and go through the system buffers."""
@@ -229,6 +252,9 @@ def main():
                     emit(gemm_cfg(a.gemm_n, P, a.gemm_reps, a.check))
                 elif cfg == "f2":
                     emit(jacobi3d_cfg(1024, 20, P))
+                elif cfg == "f4":
+                    for row in footprint_cfg(P):
+                        emit(row)
                 elif cfg == "f1":
                     emit(scatter_cfg(1 << 26, P, 5))
                 elif cfg == "c4":

@@ -199,9 +199,12 @@ int accmg_finalize(void);
 
 /* Data-region entry (copyin semantics, L119 §IV.C). Registers `extent` elements of `elem_size`
    bytes at `host_array` (caller-owned, borrowed until accmg_region_destroy; must stay valid and
-   unchanged). Device replicas are allocated now (full extent per local partition, so global
-   indices need no rewriting, L110) but filled lazily: before each loop the data loader copies in
-   only what each partition may read and does not yet hold (L119, L125). elem_size in {1,2,4,8}. */
+   unchanged). Device replicas are allocated lazily and only as large as each partition needs: the
+   hull of its declared windows for distributed arrays (L121-123 "only the sub-array actually
+   accessed by the GPU is loaded"), the whole array for replicated ones; kernels still use global
+   indices (the replica pointer is offset, so the index rewriting of L110 is the identity). Before
+   each loop the data loader copies in only what each partition may read and does not yet hold
+   (L119, L125). elem_size in {1,2,4,8}. */
 int accmg_region_create(void* host_array, size_t elem_size, int64_t extent, accmg_region* out);
 
 /* Data-region exit without copy-out (OpenACC `delete`); frees the region's device memory. */
@@ -252,8 +255,9 @@ int accmg_debug_chunk_bits(accmg_region r, int partition, uint32_t* out_words, i
    uint64 n_runs, uint64 n_elems, int64 run_start[n_runs], int64 run_end[n_runs] (exclusive),
    payload (elem_size * n_elems bytes). *used = its size; copies min(cap, size) bytes. */
 int accmg_debug_packed(accmg_region r, int partition, void* out, int64_t cap, int64_t* used);
-/* Copies `partition`'s whole replica (extent * elem_size bytes) to out; only its valid ranges
-   (accmg_debug_valid) hold defined values. Blocks. */
+/* Copies `partition`'s replica into out (an extent * elem_size buffer) at the same offsets; only
+   the allocated hull is written and only the valid ranges (accmg_debug_valid) hold defined values.
+   Blocks. */
 int accmg_debug_replica(accmg_region r, int partition, void* out);
 /* Valid intervals [lo, hi) of `partition`'s replica (any partition; host-side table):
    out_pairs receives up to cap pairs, *n the total count. partition = -1: this process's host copy. */

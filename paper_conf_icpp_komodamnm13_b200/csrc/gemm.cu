@@ -88,7 +88,7 @@ __device__ __forceinline__ void tile_coords(int64_t t, int num_m, int num_n, int
 
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ CUtensorMap map_b,
-            float* __restrict__ C, int64_t N, int64_t K, int64_t m0, int64_t m1) {
+            float* __restrict__ C, int64_t N, int64_t K, int64_t m0, int64_t m1, int64_t row_lo) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages * kStageBytes);
@@ -134,7 +134,7 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
                     unsigned char* sa = smem + stage * kStageBytes;
                     unsigned char* sb = sa + kABytes;
                     mbar_expect_tx(&full[stage], kStageBytes);
-                    tma_load_2d(&map_a, &full[stage], sa, kb * BK, row);
+                    tma_load_2d(&map_a, &full[stage], sa, kb * BK, row - (int)row_lo);
 #pragma unroll
                     for (int j = 0; j < BN / 64; ++j) tma_load_2d(&map_b, &full[stage], sb + j * (BK * 128), col + 64 * j, kb * BK);
                     if (++stage == kStages) { stage = 0; phase ^= 1; }
@@ -236,13 +236,18 @@ bool make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, 
 }  // namespace
 
 cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M, int64_t N, int64_t K, int64_t m0,
-                      int64_t m1, cudaStream_t s, int64_t* launches) {
+                      int64_t m1, int64_t a_lo, cudaStream_t s, int64_t* launches) {
     (void)M;
     if (m1 <= m0) return cudaSuccess;
     if (N % BN != 0 || K % BK != 0 || K >= (1ll << 31) || N >= (1ll << 31) || m1 >= (1ll << 31))
         return cudaErrorNotSupported;
+    // A's map starts at the first whole row of its allocation, so the TMA unit never addresses
+    // rows outside it (row coordinates are relative to row_lo)
+    const int64_t row_lo = (a_lo + K - 1) / K;
+    if (m0 < row_lo) return cudaErrorInvalidValue;
     CUtensorMap ma, mb;
-    if (!make_map(&ma, A, (uint64_t)K, (uint64_t)m1, (uint64_t)K * 2, BK, BM)) return cudaErrorNotSupported;
+    if (!make_map(&ma, A + row_lo * K, (uint64_t)K, (uint64_t)(m1 - row_lo), (uint64_t)K * 2, BK, BM))
+        return cudaErrorNotSupported;
     if (!make_map(&mb, B, (uint64_t)N, (uint64_t)K, (uint64_t)N * 2, 64, BK)) return cudaErrorNotSupported;
     static int sms = 0;
     if (!sms) {
@@ -255,7 +260,7 @@ cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M,
     if (e != cudaSuccess) return e;
     const int64_t tiles = ((m1 - m0 + BM - 1) / BM) * (N / BN);
     const int grid = (int)(tiles < sms ? tiles : sms);
-    gemm_kernel<<<grid, kThreads, smem, s>>>(ma, mb, C, N, K, m0, m1);
+    gemm_kernel<<<grid, kThreads, smem, s>>>(ma, mb, C, N, K, m0, m1, row_lo);
     if (launches) *launches += 1;
     return cudaGetLastError();
 }

@@ -40,7 +40,7 @@ __device__ __forceinline__ float s7(float u, float d, float n, float s, float w,
 template <bool TRACK>
 __global__ void __launch_bounds__(256)
 jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, int64_t n1, int64_t n2, int64_t i0,
-             int64_t i1, int64_t jl, int64_t jh, int64_t kl, int64_t kh, int64_t kbase, Track t) {
+             int64_t i1, int64_t jl, int64_t jh, int64_t kl, int64_t kh, int64_t kbase, int64_t plane_lo, Track t) {
     __shared__ __align__(128) float tile[kStages][kStageFloats];
     __shared__ __align__(8) uint64_t bar[kStages];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
@@ -55,7 +55,7 @@ jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, i
         dev::tma_prefetch_desc(&map);
         for (int q = 0; q < kStages && q < count; ++q) {  // all stages free at the start
             dev::mbar_expect_tx(&bar[q], kTileBytes);
-            dev::tma_load_3d(&map, &bar[q], tile[q], (int)(k0 - 4), (int)(j0 - 1), (int)(ps - 1 + q));
+            dev::tma_load_3d(&map, &bar[q], tile[q], (int)(k0 - 4), (int)(j0 - 1), (int)(ps - 1 + q - plane_lo));
         }
     }
     __syncthreads();
@@ -113,7 +113,7 @@ jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, i
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             dev::mbar_expect_tx(&bar[qn % kStages], kTileBytes);
             dev::tma_load_3d(&map, &bar[qn % kStages], tile[qn % kStages], (int)(k0 - 4), (int)(j0 - 1),
-                             (int)(ps - 1 + qn));
+                             (int)(ps - 1 + qn - plane_lo));
         }
     }
 }
@@ -121,19 +121,25 @@ jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, i
 }  // namespace
 
 cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64_t n2, int64_t i0, int64_t i1,
-                     int64_t jl, int64_t jh, int64_t kl, int64_t kh, Track t, cudaStream_t s, int64_t* launches) {
+                     int64_t jl, int64_t jh, int64_t kl, int64_t kh, int64_t src_lo, int64_t src_hi, Track t,
+                     cudaStream_t s, int64_t* launches) {
     if (i1 <= i0 || jh <= jl || kh <= kl) return cudaSuccess;
     if (n2 % 4 != 0 || (reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) % 16 != 0 ||
         n0 >= (1ll << 31) || n1 >= (1ll << 31) || n2 >= (1ll << 31))
         return cudaErrorNotSupported;
     auto fn = tma_encode_fn();
     if (!fn) return cudaErrorNotSupported;
+    // the tensor map covers only the planes of src's allocation ([src_lo, src_hi) elements), so
+    // the TMA unit never addresses memory outside it; plane coordinates are relative to plane_lo
+    const int64_t pl = n1 * n2;
+    const int64_t plane_lo = (src_lo + pl - 1) / pl, plane_hi = src_hi / pl;
+    if (i0 - 1 < plane_lo || i1 + 1 > plane_hi) return cudaErrorInvalidValue;
     CUtensorMap map;
-    cuuint64_t dims[3] = {(cuuint64_t)n2, (cuuint64_t)n1, (cuuint64_t)n0};
+    cuuint64_t dims[3] = {(cuuint64_t)n2, (cuuint64_t)n1, (cuuint64_t)(plane_hi - plane_lo)};
     cuuint64_t strides[2] = {(cuuint64_t)n2 * 4, (cuuint64_t)n1 * n2 * 4};
     cuuint32_t box[3] = {BOXK, BOXJ, 1};
     cuuint32_t es[3] = {1, 1, 1};
-    if (fn(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(src), dims, strides, box, es,
+    if (fn(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(src) + plane_lo * pl, dims, strides, box, es,
            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
         return cudaErrorNotSupported;
@@ -141,9 +147,9 @@ cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64
     dim3 grid((unsigned)((kh - kbase + TK - 1) / TK), (unsigned)((jh - jl + TJ - 1) / TJ),
               (unsigned)((i1 - i0 + kPlaneSeg - 1) / kPlaneSeg));
     if (t.l1)
-        jacobi3d_tma<true><<<grid, 256, 0, s>>>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, kbase, t);
+        jacobi3d_tma<true><<<grid, 256, 0, s>>>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, kbase, plane_lo, t);
     else
-        jacobi3d_tma<false><<<grid, 256, 0, s>>>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, kbase, t);
+        jacobi3d_tma<false><<<grid, 256, 0, s>>>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, kbase, plane_lo, t);
     if (launches) *launches += 1;
     return cudaGetLastError();
 }

@@ -32,8 +32,10 @@ cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, i
 
 // 3-D 7-point Jacobi (TMA-staged tiles) on planes [i0, i1) x rows [jl, jh) x cols [kl, kh) of an
 // n0 x n1 x n2 fp32 array; needs n2 % 4 == 0 (else cudaErrorNotSupported).
+// [src_lo, src_hi): the element range allocated behind src (the TMA map is limited to it).
 cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64_t n2, int64_t i0, int64_t i1,
-                     int64_t jl, int64_t jh, int64_t kl, int64_t kh, Track t, cudaStream_t s, int64_t* launches);
+                     int64_t jl, int64_t jh, int64_t kl, int64_t kh, int64_t src_lo, int64_t src_hi, Track t,
+                     cudaStream_t s, int64_t* launches);
 
 // Test body: rows i in [r0, r1) with i % period == 0: out[i][:] = in[i][:] + 1.0f.
 cudaError_t sparse_rows(const float* in, float* out, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
@@ -51,8 +53,9 @@ cudaError_t kmeans_update(int64_t* sums, int64_t* counts, float* cen, int64_t c0
 
 // bf16 x bf16 -> fp32 GEMM of rows [m0, m1) of C = A.B (A [M][K], B [K][N], C [M][N], row-major),
 // tcgen05.mma with TMEM accumulators and TMA operand staging.
+// a_lo: first element of A's allocation (the A tensor map starts at its first whole row).
 cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M, int64_t N, int64_t K,
-                      int64_t m0, int64_t m1, cudaStream_t s, int64_t* launches);
+                      int64_t m0, int64_t m1, int64_t a_lo, cudaStream_t s, int64_t* launches);
 
 // Irregular-write body (L137): dst[idx[i]] = src[i] for i in [i0, i1); writes whose index is outside
 // [wlo, whi) append {index, value bits} to recs (slot from *count, warp-aggregated).

@@ -60,7 +60,12 @@ struct accmg_region_s {
     int64_t id = 0;
     uint8_t* host = nullptr;
     int64_t esize = 0, extent = 0;
-    std::vector<uint8_t*> dev;       // V local replicas (full extent)
+    // Local replicas: dev[li] is the *global-index base* of partition li's replica — element e lives
+    // at dev[li] + e*esize — but only the hull of what the partition ever needs is allocated
+    // (window-sized allocations for distributed arrays, §8 row f4; full extent for replicated ones).
+    std::vector<uint8_t*> dev;       // V (virtual bases; nullptr = nothing allocated yet)
+    std::vector<uint8_t*> abase;     // V cudaMalloc'd pointers
+    std::vector<Ival> arange;        // P allocated element range of every partition (global table)
     std::vector<IntervalSet> valid;  // P partitions
     IntervalSet host_valid;          // this process's host copy
     std::vector<Trk> trk;            // V
@@ -161,12 +166,16 @@ inline int first_local() { return S.rank * S.V; }
 
 // P2P mode: publish `mine` (this process's device allocations, one per local partition) and map
 // every peer's through CUDA IPC; out[g] = pointer usable here for partition g (collective).
+// Null entries publish nothing (out = nullptr).
 int exchange_ptrs(const std::vector<void*>& mine, std::vector<void*>& out, std::vector<void*>& opened) {
     const int n = (int)mine.size();
     if ((size_t)n * sizeof(cudaIpcMemHandle_t) > accmg::Bootstrap::kSlotBytes)
         return fail(ACCMG_EUNSUPPORTED, "exchange_ptrs: too many handles", false);
     auto* slot = static_cast<cudaIpcMemHandle_t*>(S.boot.slot(S.rank));
-    for (int i = 0; i < n; ++i) CUDA_TRY(cudaIpcGetMemHandle(&slot[i], mine[i]));
+    for (int i = 0; i < n; ++i) {
+        if (mine[i]) CUDA_TRY(cudaIpcGetMemHandle(&slot[i], mine[i]));
+        else std::memset(&slot[i], 0, sizeof(cudaIpcMemHandle_t));
+    }
     std::string err;
     if (!S.boot.barrier(&err)) return fail(ACCMG_ESTATE, err, true);
     out.assign((size_t)S.W * n, nullptr);
@@ -177,6 +186,9 @@ int exchange_ptrs(const std::vector<void*>& mine, std::vector<void*>& out, std::
                 out[(size_t)q * n + i] = mine[i];
                 continue;
             }
+            cudaIpcMemHandle_t zero;
+            std::memset(&zero, 0, sizeof(zero));
+            if (std::memcmp(&qs[i], &zero, sizeof(zero)) == 0) continue;  // nothing allocated there
             void* p = nullptr;
             CUDA_TRY(cudaIpcOpenMemHandle(&p, qs[i], cudaIpcMemLazyEnablePeerAccess));
             out[(size_t)q * n + i] = p;
@@ -272,6 +284,59 @@ int collect_prof() {
         S.ev_free.push_back(p.b);
     }
     S.prof.clear();
+    return 0;
+}
+
+// ---- window-sized replicas (§8 row f4) -------------------------------------------------------------
+// Grows every partition's allocated hull to cover need[g] (the same decision on every rank: the
+// tables are global). Local growth: allocate the new hull, copy what is valid, free the old one
+// (after the P2P re-exchange, so no peer still maps it). P2P: re-publish the region's replicas.
+int ensure_alloc(accmg_region_s* r, const std::vector<IntervalSet>& need) {
+    if (S.dry) return 0;
+    bool changed = false;
+    std::vector<uint8_t*> to_free;
+    std::vector<int64_t> freed_bytes;
+    for (int g = 0; g < S.P; ++g) {
+        if (need[g].empty()) continue;
+        Ival& a = r->arange[g];
+        int64_t lo = need[g].items().front().lo, hi = need[g].items().back().hi;
+        if (a.hi > a.lo) {
+            lo = std::min(lo, a.lo);
+            hi = std::max(hi, a.hi);
+        }
+        if (a.hi > a.lo && lo == a.lo && hi == a.hi) continue;
+        changed = true;
+        const Ival old = a;
+        a = {lo, hi};
+        if (!local(g)) continue;
+        const int li = lidx(g);
+        uint8_t* nb = nullptr;
+        TRY(dmalloc((void**)&nb, (size_t)((hi - lo) * r->esize), false));
+        uint8_t* nbase = nb - lo * r->esize;
+        if (r->abase[li]) {
+            IntervalSet keep = r->valid[g].intersect(IntervalSet(old.lo, old.hi));
+            for (auto& iv : keep.items())
+                CUDA_TRY(cudaMemcpyAsync(nbase + iv.lo * r->esize, r->dev[li] + iv.lo * r->esize,
+                                         (size_t)((iv.hi - iv.lo) * r->esize), cudaMemcpyDeviceToDevice, S.stream));
+            to_free.push_back(r->abase[li]);
+            freed_bytes.push_back((old.hi - old.lo) * r->esize);
+        }
+        r->abase[li] = nb;
+        r->dev[li] = nbase;
+    }
+    if (changed && S.p2p) {
+        for (auto p : r->opened) cudaIpcCloseMemHandle(p);
+        r->opened.clear();
+        std::vector<void*> mine(r->abase.begin(), r->abase.end()), all;
+        TRY(exchange_ptrs(mine, all, r->opened));
+        r->gdev.assign(S.P, nullptr);
+        for (int g = 0; g < S.P; ++g)
+            if (all[g]) r->gdev[g] = static_cast<uint8_t*>(all[g]) - r->arange[g].lo * r->esize;
+    }
+    if (!to_free.empty()) {
+        CUDA_TRY(cudaStreamSynchronize(S.stream));
+        for (size_t i = 0; i < to_free.size(); ++i) dfree(to_free[i], freed_bytes[i], false);
+    }
     return 0;
 }
 
@@ -549,8 +614,9 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
         }
         case ACCMG_BODY_JACOBI3D_7PT: {
             auto x = static_cast<const accmg_args_jacobi3d*>(args);
+            const Ival al = d[0].region->arange[g];
             e = k::jacobi3d((const float*)P(0), (float*)P(1), x->n0, x->n1, x->n2, a, b, bd->lo[1], bd->hi[1],
-                            bd->lo[2], bd->hi[2], T(1), S.stream, L);
+                            bd->lo[2], bd->hi[2], al.lo, al.hi, T(1), S.stream, L);
             break;
         }
         case ACCMG_BODY_SCATTER: {
@@ -563,7 +629,7 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
         case ACCMG_BODY_GEMM_BF16_F32: {
             auto x = static_cast<const accmg_args_gemm*>(args);
             e = k::gemm_bf16((const uint16_t*)P(0), (const uint16_t*)P(1), (float*)P(2), x->M, x->N, x->K, a, b,
-                             S.stream, L);
+                             d[0].region->arange[g].lo, S.stream, L);
             break;
         }
         case ACCMG_BODY_KMEANS_ASSIGN: {
@@ -799,7 +865,11 @@ void free_region(accmg_region_s* r) {
             std::string err;
             S.boot.barrier(&err);
         }
-        for (auto p : r->dev) dfree(p, r->extent * r->esize, false);
+        for (int li = 0; li < (int)r->abase.size(); ++li)
+            if (r->abase[li]) {
+                const Ival& a = r->arange[first_local() + li];
+                dfree(r->abase[li], (a.hi - a.lo) * r->esize, false);
+            }
         for (auto& t : r->trk) {
             dfree(t.l1, t.nwords * 4, true);
             dfree(t.l2, t.nl2 * 4, true);
@@ -941,26 +1011,11 @@ int accmg_region_create(void* host_array, size_t elem_size, int64_t extent, accm
     r->host_valid = IntervalSet(0, extent);
     r->trk.assign(S.V, Trk());
     r->dev.assign(S.V, nullptr);
+    r->abase.assign(S.V, nullptr);
+    r->arange.assign(S.P, Ival{0, 0});
+    r->gdev.assign(S.P, nullptr);
     r->partial.assign(S.V, nullptr);
-    if (!S.dry) {
-        for (int li = 0; li < S.V; ++li) {
-            int rc = dmalloc((void**)&r->dev[li], (size_t)(extent * elem_size), false);
-            if (rc) {
-                free_region(r);
-                return rc;
-            }
-        }
-        if (S.p2p) {
-            std::vector<void*> mine(r->dev.begin(), r->dev.end()), all;
-            int rc = exchange_ptrs(mine, all, r->opened);
-            if (rc) {
-                free_region(r);
-                return rc;
-            }
-            r->gdev.resize(S.P);
-            for (int g = 0; g < S.P; ++g) r->gdev[g] = static_cast<uint8_t*>(all[g]);
-        }
-    }
+    // replicas are allocated on first use, sized to what each partition needs (ensure_alloc)
     S.regions.push_back(r);
     *out = r;
     return 0;
@@ -1019,6 +1074,8 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
                 for (int h = 0; h < g; ++h)
                     if (need[i][g].overlaps(need[i][h]))
                         return fail(ACCMG_ECONFLICT, "declared write windows of two partitions overlap (G14)", false);
+    // window-sized replicas: every partition's allocation covers what it needs (f4)
+    for (int i = 0; i < n_descs; ++i) TRY(ensure_alloc(descs[i].region, need[i]));
     // 3. data loader: plan all pulls from the pre-phase state, then run them
     std::vector<Xfer> xs;
     for (int i = 0; i < n_descs; ++i) plan_pulls(descs[i].region, need[i], xs);
@@ -1029,7 +1086,10 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
     std::vector<bool> tracked(n_descs, false);
     std::vector<accmg_region_s*> tracked_regs;
     for (int i = 0; i < n_descs; ++i)
-        if ((descs[i].mode & ACCMG_W) && descs[i].mode != ACCMG_REDUCE_SUM && !descs[i].declared) {
+        // with a single partition there is no other replica to keep coherent: no tracking
+        // (kept under debug_checks so the artefacts can still be inspected)
+        if ((descs[i].mode & ACCMG_W) && descs[i].mode != ACCMG_REDUCE_SUM && !descs[i].declared &&
+            (S.P > 1 || S.cfg.debug_checks)) {
             tracked[i] = true;
             tracked_regs.push_back(descs[i].region);
         }
@@ -1139,6 +1199,7 @@ static int sync_host_impl(accmg_region r, bool owned) {
             need[q * S.V].add(m);
             need[q * S.V].add(r->valid[q * S.V]);
         }
+        TRY(ensure_alloc(r, need));
         std::vector<Xfer> xs;
         plan_pulls(r, need, xs);
         TRY(run_xfers(xs));
@@ -1264,7 +1325,10 @@ int accmg_debug_replica(accmg_region r, int partition, void* out) {
     Trk* t;
     TRY(debug_region(r, partition, &t));
     if (!out) return fail(ACCMG_EINVAL, "debug: null", false);
-    CUDA_TRY(cudaMemcpyAsync(out, r->dev[lidx(partition)], (size_t)(r->extent * r->esize), cudaMemcpyDeviceToHost, S.stream));
+    const Ival a = r->arange[partition];
+    if (a.hi > a.lo)
+        CUDA_TRY(cudaMemcpyAsync(static_cast<uint8_t*>(out) + a.lo * r->esize, r->dev[lidx(partition)] + a.lo * r->esize,
+                                 (size_t)((a.hi - a.lo) * r->esize), cudaMemcpyDeviceToHost, S.stream));
     CUDA_TRY(cudaStreamSynchronize(S.stream));
     return 0;
 }
