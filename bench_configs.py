@@ -203,6 +203,42 @@ def footprint_cfg(P):
     return rows
 
 
+def chunk_sweep_cfg(P):
+    """§8 row f3 / E7 (L135: "we experimentally choose 1MB"): loop time and inter-partition bytes of
+    undeclared writes vs the second-level chunk size, for the paper's protocol (whole chunks +
+    bits) and for compacted runs; a sparse writer (every 100th row of 16384^2) and a dense one (C5)."""
+    rows = []
+    N = 16384
+    for body in ("sparse", "dense"):
+        for proto in (A.DIRTY_RUNS, A.DIRTY_CHUNKS):
+            for cb in (1 << 12, 1 << 14, 1 << 16, 1 << 18, 1 << 20, 1 << 22, 1 << 24):
+                src = gen.jacobi_field(7, N)
+                dst = src.copy()
+                A.accmg_init(num_partitions=P, device=0, profile=1, dirty_chunk_bytes=cb, dirty_protocol=proto)
+                try:
+                    rs, rd = A.accmg_region_create(src), A.accmg_region_create(dst)
+                    def loop(s):
+                        if body == "sparse":
+                            A.accmg_loop_launch(A.bounds([0], [N]), A.BODY_TEST_SPARSE_WRITE,
+                                                [A.access(rs, A.R), A.access(rd, A.W)], A.accmg_args_sparse(N, N, 100))
+                        else:
+                            WL.jacobi_sweep(rs, rd, s, N, False)
+                    loop(0)
+                    loop(1)
+                    A.accmg_barrier()
+                    A.accmg_reset_stats()
+                    reps = 5
+                    t = wall(lambda: [loop(s) for s in range(2, 2 + reps)])
+                    st = A.accmg_get_stats()
+                finally:
+                    A.accmg_finalize()
+                rows.append({"config": "f3_chunk_sweep", "body": body, "P": P,
+                             "protocol": "chunks" if proto == A.DIRTY_CHUNKS else "runs", "chunk_bytes": cb,
+                             "ms_per_loop": t / reps * 1e3, "bytes_per_loop": st["bytes_interpartition"] / reps,
+                             "ms_compact": st["ms_compact"] / reps, "ms_exchange": st["ms_exchange"] / reps})
+    return rows
+
+
 def scatter_cfg(n, P, reps):
     """§8 row f1: irregular writes dst[idx[i]] = src[i] (idx a random permutation) to a distributed
     array; (P-1)/P of the writes miss the writer's window and go through the system buffers."""
@@ -252,6 +288,9 @@ def main():
                     emit(gemm_cfg(a.gemm_n, P, a.gemm_reps, a.check))
                 elif cfg == "f2":
                     emit(jacobi3d_cfg(1024, 20, P))
+                elif cfg == "f3":
+                    for row in chunk_sweep_cfg(P):
+                        emit(row)
                 elif cfg == "f4":
                     for row in footprint_cfg(P):
                         emit(row)

@@ -53,6 +53,10 @@ extern "C" {
                                   partitions of one process (self send/recv) — for testing */
 #define ACCMG_XCHG_NCCL     2  /* across processes: NCCL send/recv and all-reduce */
 
+/* dirty_protocol */
+#define ACCMG_DIRTY_RUNS   0
+#define ACCMG_DIRTY_CHUNKS 1
+
 typedef struct accmg_config {
     int32_t num_partitions;    /* P, the number of tasks groups every loop is divided into (L108);
                                   1..64; a multiple of world_size. P / world_size partitions live on
@@ -69,7 +73,11 @@ typedef struct accmg_config {
                                   disjointness (L62), keep per-loop bitmap snapshots for the
                                   debug getters; costs extra device work */
     int32_t profile;           /* 1 = time body / compaction / exchange phases with CUDA events */
-    int32_t reserved;
+    int32_t dirty_protocol;    /* undeclared writes: ACCMG_DIRTY_RUNS (default: compacted maximal runs
+                                  in the canonical packed buffer, scattered into the peers) or
+                                  ACCMG_DIRTY_CHUNKS (the paper's protocol, L133-135: every dirty
+                                  chunk with its first-level bits, merged by the bits; same-node
+                                  transports only) */
     uint8_t nccl_unique_id[128]; /* world_size > 1: the job's id, made on rank 0 by
                                     accmg_nccl_unique_id() (NCCL modes) or accmg_unique_id() (P2P),
                                     broadcast by the caller (e.g. torch.distributed); P2P mode names

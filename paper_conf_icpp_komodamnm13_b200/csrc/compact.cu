@@ -313,6 +313,32 @@ scatter_k(const uint8_t* __restrict__ packed, int64_t n_runs, const PtrList dsts
     }
 }
 
+// The paper's protocol (L133-135): for every chunk whose second-level bit is set, the whole chunk's
+// first-level bits decide which elements overwrite the peers' copies ("merged by the dirty bits").
+// One block per dirty chunk; lanes = bits of one word; clears the chunk's L1 words afterwards.
+template <typename T>
+__global__ void __launch_bounds__(kThreads)
+chunk_merge_k(uint32_t* __restrict__ l1, const uint32_t* __restrict__ l2, int64_t nwords, int cw_log2,
+              const T* __restrict__ src, const PtrList dsts) {
+    const int64_t cwords = (int64_t)1 << cw_log2;
+    const int64_t nchunks = (nwords + cwords - 1) / cwords;
+    const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+    for (int64_t c = blockIdx.x; c < nchunks; c += gridDim.x) {
+        if (!((l2[c >> 5] >> (c & 31)) & 1u)) continue;  // clean chunk: skipped (block-uniform)
+        const int64_t w0 = c * cwords, w1 = w0 + cwords < nwords ? w0 + cwords : nwords;
+        for (int64_t w = w0 + warp; w < w1; w += kThreads / 32) {
+            const uint32_t m = l1[w];
+            if ((m >> lane) & 1u) {
+                const T v = src[w * 32 + lane];
+                for (int d = 0; d < dsts.n; ++d) static_cast<T*>(dsts.p[d])[w * 32 + lane] = v;
+            }
+        }
+        __syncthreads();
+        for (int64_t w = w0 + threadIdx.x; w < w1; w += kThreads) l1[w] = 0u;
+        __syncthreads();
+    }
+}
+
 __global__ void reduce_sum_k(int64_t* __restrict__ acc, const PtrList srcs, int64_t n) {
     for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x) {
         int64_t a = acc[i];
@@ -385,6 +411,20 @@ cudaError_t scatter_packed(const uint8_t* packed, int64_t n_runs, const PtrList&
         default: return cudaErrorInvalidValue;
     }
     if (launches) *launches += 3;
+    return cudaGetLastError();
+}
+
+cudaError_t chunk_merge(uint32_t* l1, const uint32_t* l2, int64_t nwords, int chunk_words_log2, const void* values,
+                        int esize, const PtrList& dsts, cudaStream_t s, int64_t* launches) {
+    const unsigned g = 148 * 4;
+    switch (esize) {
+        case 1: chunk_merge_k<uint8_t><<<g, kThreads, 0, s>>>(l1, l2, nwords, chunk_words_log2, (const uint8_t*)values, dsts); break;
+        case 2: chunk_merge_k<uint16_t><<<g, kThreads, 0, s>>>(l1, l2, nwords, chunk_words_log2, (const uint16_t*)values, dsts); break;
+        case 4: chunk_merge_k<uint32_t><<<g, kThreads, 0, s>>>(l1, l2, nwords, chunk_words_log2, (const uint32_t*)values, dsts); break;
+        case 8: chunk_merge_k<uint64_t><<<g, kThreads, 0, s>>>(l1, l2, nwords, chunk_words_log2, (const uint64_t*)values, dsts); break;
+        default: return cudaErrorInvalidValue;
+    }
+    if (launches) *launches += 1;
     return cudaGetLastError();
 }
 

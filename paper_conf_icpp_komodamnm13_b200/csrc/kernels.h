@@ -89,6 +89,11 @@ constexpr int kScatterBlocks = 592;  // 4 x 148 SMs
 cudaError_t scatter_packed(const uint8_t* packed, int64_t n_runs, const PtrList& dsts, int esize,
                            int64_t* scratch, cudaStream_t s, int64_t* launches);
 
+// The paper's chunk protocol (L133-135): every dirty chunk's elements with a set L1 bit are copied
+// from `values` into each destination replica; clears those L1 words.
+cudaError_t chunk_merge(uint32_t* l1, const uint32_t* l2, int64_t nwords, int chunk_words_log2, const void* values,
+                        int esize, const PtrList& dsts, cudaStream_t s, int64_t* launches);
+
 // ---- reductions (reductiontoarray merge, L112) -------------------------------------------------
 // acc[i] += srcs.p[j][i] for every j, then dsts.p[j][i] += acc[i] for every j (int64 elements).
 cudaError_t reduce_sum_i64(int64_t* acc, const PtrList& srcs, int64_t n, cudaStream_t s, int64_t* launches);

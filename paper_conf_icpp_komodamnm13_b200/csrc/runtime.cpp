@@ -89,7 +89,7 @@ struct State {
     bool init = false;
     accmg_config cfg{};
     int P = 1, W = 1, rank = 0, V = 1;
-    bool dry = false, nccl_all = false, p2p = false, use_nccl = false;
+    bool dry = false, nccl_all = false, p2p = false, use_nccl = false, chunks = false;
     accmg::Bootstrap boot;
     uint64_t* sig = nullptr;         // P2P barrier flags (W entries), mapped by every peer
     std::vector<void*> peer_sig;     // W
@@ -668,6 +668,16 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
                 while ((1ll << cw) < chunk_elems(r) / 32) ++cw;
                 CUDA_TRY(k::compact_count(t.l1, t.l2, t.nwords, cw, t.ntiles, t.tile_counts, t.tile_edges, S.stream,
                                           &S.st.kernel_launches));
+                if (S.chunks) {
+                    // the paper's protocol: dirty chunks merged into every peer by their L1 bits
+                    ProfScope px(2);
+                    const int g = first_local() + li;
+                    k::PtrList dl{};
+                    for (int h = 0; h < S.P; ++h)
+                        if (h != g) dl.p[dl.n++] = S.p2p ? (void*)r->gdev[h] : (void*)r->dev[lidx(h)];
+                    CUDA_TRY(k::chunk_merge(t.l1, t.l2, t.nwords, cw, r->dev[li], (int)r->esize, dl, S.stream,
+                                            &S.st.kernel_launches));
+                }
                 CUDA_TRY(k::compact_scan(t.tile_counts, t.ntiles, t.tile_offs, t.totals, t.l2, t.nl2, S.stream,
                                          &S.st.kernel_launches));
             }
@@ -699,6 +709,7 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
             t.dirty_chunks = S.h_pin[4 * slot + 2];
             if (S.h_pin[4 * slot + 3] != t.n_runs) return fail(ACCMG_ECUDA, "compaction: run starts != run ends", true);
             t.packed_bytes = 16 + 16 * t.n_runs + r->esize * t.n_elems;
+            if (S.chunks) continue;  // merged already; nothing to pack
             TRY(ensure_packed(t, t.packed_bytes));
             CUDA_TRY(cudaMemcpyAsync(t.packed, t.totals, 16, cudaMemcpyDeviceToDevice, S.stream));
             ProfScope ps(1);
@@ -741,6 +752,21 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
                 elems[ri * S.P + g] = regs[ri]->trk[li].n_elems;
                 chunks[ri * S.P + g] = regs[ri]->trk[li].dirty_chunks;
             }
+    }
+    if (S.chunks) {
+        // accounting of the paper's protocol: every dirty chunk (data + its L1 bits) to P-1 peers
+        for (size_t ri = 0; ri < regs.size(); ++ri) {
+            const int64_t es = regs[ri]->esize, ce = chunk_elems(regs[ri]);
+            for (int li = 0; li < S.V; ++li) {
+                const int64_t nb = (S.P - 1) * regs[ri]->trk[li].dirty_chunks * (ce * es + ce / 8);
+                S.st.bytes_interpartition += nb;
+                S.st.bytes_paper_protocol += nb;
+                S.st.bytes_undeclared_payload += (S.P - 1) * regs[ri]->trk[li].dirty_chunks * ce * es;
+                S.st.bytes_undeclared_headers += (S.P - 1) * regs[ri]->trk[li].dirty_chunks * (ce / 8);
+                if (S.p2p) S.st.bytes_remote += (int64_t)(S.P - S.V) * regs[ri]->trk[li].dirty_chunks * (ce * es + ce / 8);
+            }
+        }
+        return 0;
     }
     // accounting (by the sending process): every packet is delivered to the P-1 other partitions
     // (reading W8)
@@ -929,6 +955,10 @@ int accmg_init(const accmg_config* cfg) {
     S.p2p = !S.dry && S.W > 1 && c.exchange_mode == ACCMG_XCHG_AUTO;
     S.use_nccl = !S.dry && (S.nccl_all || (S.W > 1 && c.exchange_mode == ACCMG_XCHG_NCCL));
     S.chunk_bytes = cb;
+    if (c.dirty_protocol != ACCMG_DIRTY_RUNS && c.dirty_protocol != ACCMG_DIRTY_CHUNKS)
+        return fail(ACCMG_EINVAL, "init: bad dirty_protocol", false);
+    S.chunks = c.dirty_protocol == ACCMG_DIRTY_CHUNKS;
+    if (S.chunks && S.use_nccl) return fail(ACCMG_EUNSUPPORTED, "init: the chunk protocol needs a same-node transport", false);
     if (S.dry) {
         S.init = true;
         return 0;

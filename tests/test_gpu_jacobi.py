@@ -149,3 +149,42 @@ def test_sparse_writes_skip_clean_chunks():
         assert st["bytes_undeclared_payload"] == (P - 1) * nrows * N * 4
         paper = st["bytes_paper_protocol"]
         assert paper > st["bytes_interpartition"]   # whole chunks + bits vs compacted runs
+
+
+@pytest.mark.parametrize("P,chunk", [(2, 1 << 20), (3, 4096)])
+def test_paper_chunk_protocol_bitexact(P, chunk):
+    """§8 row f3: the paper's protocol — whole dirty chunks with their L1 bits, merged by the bits
+    (L133-135) — gives the same replicas; it moves (P-1) * chunks * (CH*esize + CH/8) bytes."""
+    from paper_conf_icpp_komodamnm13_b200 import accmg as Acc
+    N, S = 300, 5
+    A0 = gen.jacobi_field(5, N)
+    oA, oB = _oracle_run(A0, S)
+    A, B, per, st = _gpu_run(A0, S, P, declared=False, per_loop=True, dirty_chunk_bytes=chunk,
+                             dirty_protocol=Acc.DIRTY_CHUNKS)
+    assert np.array_equal(A, oA) and np.array_equal(B, oB)
+    ce = chunk // 4
+    for p in per:
+        chunks = 0
+        for g in range(P):
+            a, b = oracle.partition(1, N - 1, P, g)
+            chunks += len({e // ce for r in range(a, b) for e in (r * N + 1, r * N + N - 2)} |
+                          {c for r in range(a, b) for c in range((r * N + 1) // ce, (r * N + N - 2) // ce + 1)})
+        assert p["bytes_interpartition"] == (P - 1) * chunks * (ce * 4 + ce // 8)
+
+
+def test_paper_chunk_protocol_sparse_rows():
+    from paper_conf_icpp_komodamnm13_b200 import accmg as Acc
+    N, P, period, chunk = 1024, 3, 100, 4096
+    src = gen.jacobi_field(7, N)
+    out0 = gen.jacobi_field(8, N)
+    o_out = out0.copy()
+    oracle.sparse_rows(src, o_out, period)
+    out = out0.copy()
+    with runtime(num_partitions=P, dirty_chunk_bytes=chunk, dirty_protocol=Acc.DIRTY_CHUNKS) as acc:
+        rs, ro = acc.accmg_region_create(src.copy()), acc.accmg_region_create(out)
+        acc.accmg_loop_launch(acc.bounds([0], [N]), Acc.BODY_TEST_SPARSE_WRITE,
+                              [acc.access(rs, Acc.R), acc.access(ro, Acc.W)], Acc.accmg_args_sparse(N, N, period))
+        for g in range(P):
+            assert np.array_equal(acc.accmg_debug_replica(ro, g, np.float32).reshape(N, N), o_out)
+        acc.accmg_sync_to_host(ro)
+    assert np.array_equal(out, o_out)
