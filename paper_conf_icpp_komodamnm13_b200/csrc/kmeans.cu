@@ -81,12 +81,11 @@ assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __
          int64_t* __restrict__ sums, int64_t* __restrict__ counts, int64_t p0, int64_t p1, int kc, int shift,
          int* err) {
     extern __shared__ __align__(16) unsigned char smem[];
-    float2* s_nc = reinterpret_cast<float2*>(smem);                                  // kc*D  (-c,-c)
-    unsigned long long* s_sum = reinterpret_cast<unsigned long long*>(s_nc + kc * D);  // kc*D
+    unsigned long long* s_sum = reinterpret_cast<unsigned long long*>(smem);           // kc*D
     unsigned long long* s_cnt = s_sum + kc * D;                                      // kc
+    float* s_nc = reinterpret_cast<float*>(s_cnt + kc);                              // kc*D  (-c)
     for (int i = threadIdx.x; i < kc * D; i += NT) {
-        const float c = -cen[i];
-        s_nc[i] = make_float2(c, c);
+        s_nc[i] = -cen[i];
         s_sum[i] = 0ull;
     }
     for (int i = threadIdx.x; i < kc; i += NT) s_cnt[i] = 0ull;
@@ -118,37 +117,38 @@ assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __
         int bi[PPT];
 #pragma unroll
         for (int q = 0; q < PPT; ++q) { bd[q] = __int_as_float(0x7f800000); bi[q] = 0; }
-        const ulonglong2* nc2 = reinterpret_cast<const ulonglong2*>(s_nc);
+        const float4* nc4 = reinterpret_cast<const float4*>(s_nc);
         // the next centroid group's values are loaded while the current one is consumed (the
-        // shared-memory latency is off the critical path)
-        ulonglong2 ncur[CU][D / 2];
+        // shared-memory latency is off the critical path); one LDS.128 brings 4 dims, and FADD2
+        // takes each dim as a scalar operand broadcast to both lanes
+        float4 ncur[CU][D / 4];
 #pragma unroll
         for (int u = 0; u < CU; ++u)
 #pragma unroll
-            for (int jj = 0; jj < D / 2; ++jj) ncur[u][jj] = nc2[(u * D) / 2 + jj];
+            for (int jj = 0; jj < D / 4; ++jj) ncur[u][jj] = nc4[(u * D) / 4 + jj];
 #pragma unroll 1
         for (int c = 0; c < kc; c += CU) {
-            ulonglong2 nnext[CU][D / 2];
+            float4 nnext[CU][D / 4];
             const int cn = (c + CU < kc) ? c + CU : c;
 #pragma unroll
             for (int u = 0; u < CU; ++u)
 #pragma unroll
-                for (int jj = 0; jj < D / 2; ++jj) nnext[u][jj] = nc2[((cn + u) * D) / 2 + jj];
+                for (int jj = 0; jj < D / 4; ++jj) nnext[u][jj] = nc4[((cn + u) * D) / 4 + jj];
             uint64_t acc[CU][NP];
 #pragma unroll
             for (int u = 0; u < CU; ++u)
 #pragma unroll
                 for (int h = 0; h < NP; ++h) acc[u][h] = 0ull;
 #pragma unroll
-            for (int j = 0; j < D; j += 2) {
+            for (int j = 0; j < D; ++j) {
 #pragma unroll
-                for (int u = 0; u < CU; ++u)
+                for (int u = 0; u < CU; ++u) {
+                    const float4 q4 = ncur[u][j / 4];
+                    const float nj = (j % 4 == 0) ? q4.x : (j % 4 == 1) ? q4.y : (j % 4 == 2) ? q4.z : q4.w;
+                    const uint64_t n2 = pk2(nj, nj);
 #pragma unroll
-                    for (int h = 0; h < NP; ++h) acc[u][h] = fma2sq(add2(xp[h][j], ncur[u][j / 2].x), acc[u][h]);
-#pragma unroll
-                for (int u = 0; u < CU; ++u)
-#pragma unroll
-                    for (int h = 0; h < NP; ++h) acc[u][h] = fma2sq(add2(xp[h][j + 1], ncur[u][j / 2].y), acc[u][h]);
+                    for (int h = 0; h < NP; ++h) acc[u][h] = fma2sq(add2(xp[h][j], n2), acc[u][h]);
+                }
             }
             // centroids in ascending order: strict < keeps the lowest index on ties
 #pragma unroll
@@ -163,7 +163,7 @@ assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __
 #pragma unroll
             for (int u = 0; u < CU; ++u)
 #pragma unroll
-                for (int jj = 0; jj < D / 2; ++jj) ncur[u][jj] = nnext[u][jj];
+                for (int jj = 0; jj < D / 4; ++jj) ncur[u][jj] = nnext[u][jj];
         }
 #pragma unroll
         for (int q = 0; q < PPT; ++q) {
@@ -186,7 +186,7 @@ template <int NP, int CU, int NT, int MINB = 1>
 cudaError_t launch_assign16(const float* x, const float* cen, int32_t* member, int64_t* sums, int64_t* counts,
                             int64_t p0, int64_t p1, int kc, int shift, int* err, cudaStream_t s, int sms) {
     auto kern = assign_d<16, NP, CU, NT, MINB>;
-    const size_t smem = (size_t)kc * 16 * 8 + (size_t)kc * 16 * 8 + (size_t)kc * 8;
+    const size_t smem = (size_t)kc * 16 * 8 + (size_t)kc * 8 + (size_t)kc * 16 * 4;
     if (smem > 200 * 1024) return cudaErrorNotSupported;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
@@ -317,7 +317,8 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
                             : launch_assign16<2, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
             case 7: e = launch_assign16<1, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
             // default: measured fastest on B200 (profiles/r01/kmeans_variants.txt)
-            default: e = launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            default: e = cu2 ? launch_assign16<2, 2, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                             : launch_assign16<2, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
         }
         if (e != cudaSuccess) return e;
     } else {

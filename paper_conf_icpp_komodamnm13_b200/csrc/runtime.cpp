@@ -291,7 +291,9 @@ int collect_prof() {
 // Grows every partition's allocated hull to cover need[g] (the same decision on every rank: the
 // tables are global). Local growth: allocate the new hull, copy what is valid, free the old one
 // (after the P2P re-exchange, so no peer still maps it). P2P: re-publish the region's replicas.
-int ensure_alloc(accmg_region_s* r, const std::vector<IntervalSet>& need) {
+// `pad`: elements added on each side of a new or grown hull (one declared stride: a write window
+// that later loops read with a one-iteration halo then needs no reallocation).
+int ensure_alloc(accmg_region_s* r, const std::vector<IntervalSet>& need, int64_t pad = 0) {
     if (S.dry) return 0;
     bool changed = false;
     std::vector<uint8_t*> to_free;
@@ -300,11 +302,13 @@ int ensure_alloc(accmg_region_s* r, const std::vector<IntervalSet>& need) {
         if (need[g].empty()) continue;
         Ival& a = r->arange[g];
         int64_t lo = need[g].items().front().lo, hi = need[g].items().back().hi;
+        if (a.hi > a.lo && lo >= a.lo && hi <= a.hi) continue;  // covered
+        lo = std::max<int64_t>(lo - pad, 0);
+        hi = std::min<int64_t>(hi + pad, r->extent);
         if (a.hi > a.lo) {
             lo = std::min(lo, a.lo);
             hi = std::max(hi, a.hi);
         }
-        if (a.hi > a.lo && lo == a.lo && hi == a.hi) continue;
         changed = true;
         const Ival old = a;
         a = {lo, hi};
@@ -1105,7 +1109,7 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
                     if (need[i][g].overlaps(need[i][h]))
                         return fail(ACCMG_ECONFLICT, "declared write windows of two partitions overlap (G14)", false);
     // window-sized replicas: every partition's allocation covers what it needs (f4)
-    for (int i = 0; i < n_descs; ++i) TRY(ensure_alloc(descs[i].region, need[i]));
+    for (int i = 0; i < n_descs; ++i) TRY(ensure_alloc(descs[i].region, need[i], descs[i].declared ? descs[i].stride : 0));
     // 3. data loader: plan all pulls from the pre-phase state, then run them
     std::vector<Xfer> xs;
     for (int i = 0; i < n_descs; ++i) plan_pulls(descs[i].region, need[i], xs);
