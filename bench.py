@@ -38,7 +38,7 @@ def parse():
     p.add_argument("--impl", default="accmg", choices=["accmg", "reference"])
     p.add_argument("--size", type=int, default=32768, help="field size N (C2: 32768)")
     p.add_argument("--undeclared", action="store_true", help="C5: no access directives (dirty-bit path)")
-    p.add_argument("--e2e-steps", type=int, default=2, help="end-to-end steps (copy-in, 100 sweeps, copy-out)")
+    p.add_argument("--e2e-steps", type=int, default=3, help="end-to-end steps (copy-in, 100 sweeps, copy-out)")
     p.add_argument("--e2e-sweeps", type=int, default=100)
     p.add_argument("--no-e2e", action="store_true")
     p.add_argument("--no-cpu-baseline", action="store_true")
@@ -216,10 +216,10 @@ def run_accmg(args):
     alg_bytes = 8 * rows_g * (N - 2)
     achieved = alg_bytes / (body_ms / 1e3) / 1e9
     # the committed ncu capture is of the N=32768, one-partition launch; other shapes report none
-    traffic = ncu_traffic("jacobi_rows") if (N == 32768 and ws == 1) else None
+    traffic = ncu_traffic("jacobi2d_tma") if (N == 32768 and ws == 1) else None
     roof = {"bound": "hbm", "achieved": round(achieved, 1), "peak": peaks["hbm_gbs"], "unit": "GB/s",
             "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": traffic,
-            "peak_source": peak_src, "kernel": "jacobi_rows<4>", "algorithmic_bytes_per_launch": alg_bytes,
+            "peak_source": peak_src, "kernel": "jacobi2d_tma_k (TMA-staged tiles)", "algorithmic_bytes_per_launch": alg_bytes,
             "avg_launch_ms": round(body_ms, 4)}
     bytes_loop = float(tb[0]) / max(st["loops"], 1)
     launches = int(tb[1])

@@ -14,6 +14,8 @@
 // parenthesisation above, so results are bit-identical to the oracle for any partition count.
 // The optional fused epilogue (TRACK) sets the two-level dirty bits of every written element
 // (L133-135) with warp-aggregated atomics (track.cuh).
+#include <cstdlib>
+
 #include "kernels.h"
 #include "track.cuh"
 
@@ -153,9 +155,21 @@ sparse_rows_kernel(const float* __restrict__ in, float* __restrict__ out, int64_
 }  // namespace
 
 cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
-                     int64_t c0, int64_t c1, Track t, int impl, cudaStream_t s, int64_t* launches) {
+                     int64_t c0, int64_t c1, int64_t src_lo, int64_t src_hi, Track t, int impl, cudaStream_t s,
+                     int64_t* launches) {
     if (r1 <= r0 || c1 <= c0) return cudaSuccess;
-    (void)impl;
+    if (impl == 0) {
+        static int env = -1;
+        if (env < 0) {
+            const char* v = getenv("ACCMG_JACOBI_IMPL");
+            env = v ? atoi(v) : 2;  // TMA-staged tiles: measured faster (profiles/r01/jacobi_impl.log)
+        }
+        impl = env;
+    }
+    if (impl == 2) {
+        cudaError_t e = jacobi2d_tma(src, dst, rows, cols, r0, r1, c0, c1, src_lo, src_hi, t, s, launches);
+        if (e != cudaErrorNotSupported) return e;  // shapes the TMA variant does not take fall through
+    }
     const bool vec4 = (cols % 4 == 0) && ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) % 16 == 0);
     cudaError_t e = vec4 ? launch_rows<4>(src, dst, rows, cols, r0, r1, c0, c1, t, s)
                          : launch_rows<1>(src, dst, rows, cols, r0, r1, c0, c1, t, s);

@@ -1,0 +1,142 @@
+// Loop body variant: 2-D 5-point Jacobi with TMA-staged shared-memory tiles (impl = 2).
+//
+// Same operation and rounding as jacobi.cu. Each CTA owns a 128-column strip and a segment of
+// kTiles x 32 rows; one thread streams (32 + 2) x 136-float tiles (rows with their halo rows,
+// columns with 4 halo columns each side) through a 4-stage ring with cp.async.bulk.tensor.2d
+// completing on mbarriers; 8 warps compute 4 rows x 4 columns per lane from shared memory
+// (horizontal neighbours by shuffle) and store 128-bit vectors of interior points. The halo rows
+// of a tile are the previous / next tile's edge rows, so their second read hits L2.
+// Kept beside the register-marching kernel (impl = 1, the default) to compare the two designs on
+// the same shapes: see profiles/ and DESIGN.md.
+#include "kernels.h"
+#include "tma_dev.cuh"
+#include "tma_host.h"
+#include "track.cuh"
+
+namespace accmg {
+namespace k {
+namespace {
+
+constexpr int TK = 128;
+constexpr int RB = 32;             // rows computed per tile
+constexpr int BOXK = TK + 8;
+constexpr int BOXR = RB + 2;
+constexpr int kStages = 4;
+constexpr int kTiles = 8;          // tiles per CTA (256 rows)
+constexpr uint32_t kTileBytes = BOXK * BOXR * 4;
+constexpr int kStageFloats = ((kTileBytes + 127) / 128) * 32;  // 128-byte aligned stages
+
+__device__ __forceinline__ float st5(float n, float s, float w, float e) {
+    return __fmul_rn(__fadd_rn(__fadd_rn(n, s), __fadd_rn(w, e)), 0.25f);
+}
+
+template <bool TRACK>
+__global__ void __launch_bounds__(256)
+jacobi2d_tma_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, int64_t cols, int64_t r0, int64_t r1,
+               int64_t c0, int64_t c1, int64_t cbase, int64_t row_lo, Track t) {
+    extern __shared__ __align__(128) unsigned char smem_raw[];
+    float* tiles = reinterpret_cast<float*>(smem_raw);
+    __shared__ __align__(8) uint64_t bar[kStages];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int64_t k0 = cbase + (int64_t)blockIdx.x * TK;
+    const int64_t rs = r0 + (int64_t)blockIdx.y * (RB * kTiles);
+    if (rs >= r1) return;
+    const int ntiles = (int)((((r1 - rs) < RB * kTiles ? (r1 - rs) : RB * kTiles) + RB - 1) / RB);
+    if (tid == 0) {
+        for (int s = 0; s < kStages; ++s) dev::mbar_init(&bar[s], 1);
+        dev::mbar_fence_init();
+        dev::tma_prefetch_desc(&map);
+        for (int m = 0; m < kStages && m < ntiles; ++m) {
+            dev::mbar_expect_tx(&bar[m], kTileBytes);
+            dev::tma_load_2d(&map, &bar[m], tiles + m * kStageFloats, (int)(k0 - 4), (int)(rs + RB * m - 1 - row_lo));
+        }
+    }
+    __syncthreads();
+    const int64_t k = k0 + 4 * lane;
+    unsigned nib = 0;
+#pragma unroll
+    for (int c = 0; c < 4; ++c) nib |= (k + c >= c0 && k + c < c1) ? (1u << c) : 0u;
+    const bool full = nib == 0xFu;
+    const int col = 4 + 4 * lane;
+    dev::WarpTracker<4> trk;
+    if constexpr (TRACK) trk.init(nib);
+    for (int m = 0; m < ntiles; ++m) {
+        const int st = m % kStages;
+        dev::mbar_wait(&bar[st], (uint32_t)((m / kStages) & 1));
+        const float* T = tiles + st * kStageFloats;
+        // rows 4*warp .. 4*warp+3 of the tile (tile row index = row + 1)
+        float4 R[6];
+#pragma unroll
+        for (int q = 0; q < 6; ++q) R[q] = *reinterpret_cast<const float4*>(T + (4 * warp + q) * BOXK + col);
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const int64_t row = rs + (int64_t)RB * m + 4 * warp + q;
+            const float4 C = R[q + 1], N = R[q], S = R[q + 2];
+            float w = __shfl_up_sync(dev::kFull, C.w, 1);
+            float e = __shfl_down_sync(dev::kFull, C.x, 1);
+            if (lane == 0) w = T[(4 * warp + q + 1) * BOXK + col - 1];
+            if (lane == 31) e = T[(4 * warp + q + 1) * BOXK + col + 4];
+            if (row < r1) {  // warp-uniform
+                float o[4];
+                o[0] = st5(N.x, S.x, w, C.y);
+                o[1] = st5(N.y, S.y, C.x, C.z);
+                o[2] = st5(N.z, S.z, C.y, C.w);
+                o[3] = st5(N.w, S.w, C.z, e);
+                float* out = dst + row * cols + k;
+                if (full) {
+                    *reinterpret_cast<float4*>(out) = make_float4(o[0], o[1], o[2], o[3]);
+                } else {
+#pragma unroll
+                    for (int c = 0; c < 4; ++c)
+                        if (nib & (1u << c)) out[c] = o[c];
+                }
+                if constexpr (TRACK) trk.mark(t.l1, t.l2, t.l2_shift, row * cols + k0);
+            }
+        }
+        __syncthreads();  // every thread is done with stage st
+        if (tid == 0 && m + kStages < ntiles) {
+            const int mn = m + kStages;
+            asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+            dev::mbar_expect_tx(&bar[st], kTileBytes);
+            dev::tma_load_2d(&map, &bar[st], tiles + st * kStageFloats, (int)(k0 - 4),
+                             (int)(rs + RB * mn - 1 - row_lo));
+        }
+    }
+}
+
+}  // namespace
+
+cudaError_t jacobi2d_tma(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1, int64_t c0,
+                         int64_t c1, int64_t src_lo, int64_t src_hi, Track t, cudaStream_t s, int64_t* launches) {
+    (void)rows;
+    if (r1 <= r0 || c1 <= c0) return cudaSuccess;
+    if (cols % 4 != 0 || (reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) % 16 != 0 ||
+        cols >= (1ll << 31))
+        return cudaErrorNotSupported;
+    auto fn = tma_encode_fn();
+    if (!fn) return cudaErrorNotSupported;
+    // the map covers only the whole rows of src's allocation (row coordinates relative to row_lo)
+    const int64_t row_lo = (src_lo + cols - 1) / cols, row_hi = src_hi / cols;
+    if (r0 - 1 < row_lo || r1 + 1 > row_hi) return cudaErrorInvalidValue;
+    CUtensorMap map;
+    cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)(row_hi - row_lo)};
+    cuuint64_t strides[1] = {(cuuint64_t)cols * 4};
+    cuuint32_t box[2] = {BOXK, BOXR};
+    cuuint32_t es[2] = {1, 1};
+    if (fn(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(src) + row_lo * cols, dims, strides, box, es,
+           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
+           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+        return cudaErrorNotSupported;
+    const int64_t cbase = (c0 / 4) * 4;
+    const size_t smem = (size_t)kStages * kStageFloats * 4;
+    auto kern = t.l1 ? jacobi2d_tma_k<true> : jacobi2d_tma_k<false>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    dim3 grid((unsigned)((c1 - cbase + TK - 1) / TK), (unsigned)((r1 - r0 + RB * kTiles - 1) / (RB * kTiles)));
+    kern<<<grid, 256, smem, s>>>(map, dst, cols, r0, r1, c0, c1, cbase, row_lo, t);
+    if (launches) *launches += 1;
+    return cudaGetLastError();
+}
+
+}  // namespace k
+}  // namespace accmg

@@ -607,8 +607,9 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
     switch (body) {
         case ACCMG_BODY_JACOBI2D_5PT: {
             auto x = static_cast<const accmg_args_jacobi2d*>(args);
-            e = k::jacobi2d((const float*)P(0), (float*)P(1), x->rows, x->cols, a, b, bd->lo[1], bd->hi[1], T(1), 0,
-                            S.stream, L);
+            const Ival al = d[0].region->arange[g];
+            e = k::jacobi2d((const float*)P(0), (float*)P(1), x->rows, x->cols, a, b, bd->lo[1], bd->hi[1], al.lo, al.hi,
+                            T(1), 0, S.stream, L);
             break;
         }
         case ACCMG_BODY_TEST_SPARSE_WRITE: {
