@@ -78,12 +78,15 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t
 constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
                             ((uint32_t)(BM >> 4) << 24);
 
-__device__ __forceinline__ void tile_coords(int64_t t, int num_m, int num_n, int& mb, int& nb) {
-    const int64_t per_group = (int64_t)kGroupM * num_n;
+// Tile raster: groups of `gm_` m-blocks swept across all n-blocks, so the tiles resident at once
+// (one per SM or SM pair) cover a near-square patch of C and share A row-blocks / B column-blocks
+// through L2.
+__device__ __forceinline__ void tile_coords(int64_t t, int num_m, int num_n, int& mb, int& nb, int gm_ = kGroupM) {
+    const int64_t per_group = (int64_t)gm_ * num_n;
     const int64_t g = t / per_group;
     const int64_t r = t % per_group;
-    const int gm = (int)(g * kGroupM);
-    const int rows_in_group = (num_m - gm) < kGroupM ? (num_m - gm) : kGroupM;
+    const int gm = (int)(g * gm_);
+    const int rows_in_group = (num_m - gm) < gm_ ? (num_m - gm) : gm_;
     mb = gm + (int)(r % rows_in_group);
     nb = (int)(r / rows_in_group);
 }
