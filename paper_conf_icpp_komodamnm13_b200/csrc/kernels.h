@@ -99,6 +99,17 @@ cudaError_t scatter_packed(const uint8_t* packed, int64_t n_runs, const PtrList&
 cudaError_t chunk_merge(uint32_t* l1, const uint32_t* l2, int64_t nwords, int chunk_words_log2, const void* values,
                         int esize, const PtrList& dsts, cudaStream_t s, int64_t* launches);
 
+// Batched device copies (data-loader pulls of one phase; src may be a peer's replica mapped
+// through IPC, read over NVLink): up to kMaxCopies ranges in one launch.
+constexpr int kMaxCopies = 32;
+struct CopyList {
+    void* dst[kMaxCopies];
+    const void* src[kMaxCopies];
+    int64_t bytes[kMaxCopies];
+    int n;
+};
+cudaError_t copy_batch(const CopyList& c, cudaStream_t s, int64_t* launches);
+
 // ---- reductions (reductiontoarray merge, L112) -------------------------------------------------
 // acc[i] += srcs.p[j][i] for every j, then dsts.p[j][i] += acc[i] for every j (int64 elements).
 cudaError_t reduce_sum_i64(int64_t* acc, const PtrList& srcs, int64_t n, cudaStream_t s, int64_t* launches);

@@ -392,6 +392,12 @@ int run_xfers(const std::vector<Xfer>& xs) {
     if (S.dry) return 0;
     ProfScope ps(2);
     bool any_nccl = false;
+    // device-to-device pulls of this phase (same-GPU replicas, or peers' replicas mapped through IPC
+    // and read over NVLink): small phases (halos) go as ONE batched copy kernel, large ones through
+    // the copy engines
+    k::CopyList batch{};
+    int64_t batch_bytes = 0;
+    std::vector<std::pair<const Xfer*, const uint8_t*>> d2d;
     for (auto& x : xs) {
         const size_t nb = (size_t)((x.hi - x.lo) * x.r->esize);
         const int64_t off = x.lo * x.r->esize;
@@ -400,17 +406,28 @@ int run_xfers(const std::vector<Xfer>& xs) {
                 CUDA_TRY(cudaMemcpyAsync(x.r->dev[lidx(x.dst)] + off, x.r->host + off, nb, cudaMemcpyHostToDevice,
                                          S.stream));
         } else if (local(x.src) && local(x.dst) && !S.nccl_all) {
-            CUDA_TRY(cudaMemcpyAsync(x.r->dev[lidx(x.dst)] + off, x.r->dev[lidx(x.src)] + off, nb,
-                                     cudaMemcpyDeviceToDevice, S.stream));
+            d2d.push_back({&x, x.r->dev[lidx(x.src)] + off});
         } else if (S.p2p) {
-            // pull from the peer's replica, mapped through IPC: a copy-engine transfer over NVLink
-            if (local(x.dst))
-                CUDA_TRY(cudaMemcpyAsync(x.r->dev[lidx(x.dst)] + off, x.r->gdev[x.src] + off, nb, cudaMemcpyDefault,
-                                         S.stream));
+            if (local(x.dst)) d2d.push_back({&x, x.r->gdev[x.src] + off});
         } else if (local(x.src) || local(x.dst)) {
             any_nccl = true;
         }
     }
+    for (auto& [x, src] : d2d) batch_bytes += (x->hi - x->lo) * x->r->esize;
+    const bool batched = !d2d.empty() && (int)d2d.size() <= k::kMaxCopies && batch_bytes <= (64ll << 20);
+    for (auto& [x, src] : d2d) {
+        const size_t nb = (size_t)((x->hi - x->lo) * x->r->esize);
+        uint8_t* dst = x->r->dev[lidx(x->dst)] + x->lo * x->r->esize;
+        if (batched) {
+            batch.dst[batch.n] = dst;
+            batch.src[batch.n] = src;
+            batch.bytes[batch.n] = (int64_t)nb;
+            ++batch.n;
+        } else {
+            CUDA_TRY(cudaMemcpyAsync(dst, src, nb, cudaMemcpyDefault, S.stream));
+        }
+    }
+    if (batched) CUDA_TRY(k::copy_batch(batch, S.stream, &S.st.kernel_launches));
     if (any_nccl) {
         NCCL_TRY(S.nccl->GroupStart());
         for (auto& x : xs) {
