@@ -180,6 +180,29 @@ def jacobi3d_cfg(n, sweeps, P, declared=True):
     return out
 
 
+def deep_cfg(N, sweeps, P, h):
+    """§8 row f2 (deep halos): `sweeps` Jacobi sweeps as sweeps/h loops of the deep-halo body —
+    one exchange of h halo rows per side per h sweeps, halo rows recomputed redundantly."""
+    Ah = gen.jacobi_field(2, N)
+    Bh = Ah.copy()
+    loops = sweeps // h
+    A.accmg_init(num_partitions=P, device=0, profile=1)
+    try:
+        rA, rB = A.accmg_region_create(Ah), A.accmg_region_create(Bh)
+        for s in range(2):
+            WL.jacobi_deep_loop(rA, rB, s, N, h)
+        A.accmg_barrier()
+        A.accmg_reset_stats()
+        t = wall(lambda: [WL.jacobi_deep_loop(rA, rB, s, N, h) for s in range(2, 2 + loops)])
+        st = A.accmg_get_stats()
+    finally:
+        A.accmg_finalize()
+    out = {"config": "f2_deep_halo", "P": P, "N": N, "h": h, "sweeps": loops * h,
+           "iters_per_s": (N - 2) ** 2 * loops * h / t, "ms_per_sweep": t / (loops * h) * 1e3,
+           "exchanges_per_sweep": 1.0 / h, **{k + "_per_sweep": v / h for k, v in per_loop(st, loops).items()}}
+    return out
+
+
 def footprint_cfg(P):
     """§8 row f4 / Fig. 9 (L249-252): device memory per configuration — User (replicas) and
     System (bitmaps, packed buffers, partials, miss buffers) — normalised to the P=1 User total."""
@@ -288,6 +311,9 @@ def main():
                     emit(gemm_cfg(a.gemm_n, P, a.gemm_reps, a.check))
                 elif cfg == "f2":
                     emit(jacobi3d_cfg(1024, 20, P))
+                elif cfg == "f2deep":
+                    for h in (1, 2, 4, 8):
+                        emit(deep_cfg(32768, 48, P, h))
                 elif cfg == "f3":
                     for row in chunk_sweep_cfg(P):
                         emit(row)

@@ -136,6 +136,11 @@ typedef struct accmg_access {
  *   descs [sums RW (int64 k*d), counts RW (int64 k), centroids W (fp32 k*d)];
  *   if counts[c] > 0: cen[c][j] = (float)(((double)sums[c][j] * 2^-shift) / (double)counts[c]);
  *   then sums[c][*] = 0, counts[c] = 0.
+ * ACCMG_BODY_JACOBI2D_DEEP: as ACCMG_BODY_JACOBI2D_5PT but each loop performs h sweeps (deep halos,
+ *   §8 row f2): dst = J^h(src) on the bounds box, J the 5-point sweep above, rows/columns outside
+ *   the box fixed. Declared form: src stride=C left=right=h*C, dst stride=C — one exchange of h
+ *   halo rows per h sweeps; each partition recomputes the rows of its halo (redundant compute) in
+ *   scratch buffers. args {rows, cols, h}.
  * ACCMG_BODY_JACOBI3D_7PT: bounds ndim=3 [1,n0-1) x [1,n1-1) x [1,n2-1) (or a sub-box); descs
  *   [src R (fp32 n0*n1*n2), dst W (fp32 n0*n1*n2)]; n2 % 4 == 0;
  *   dst[i][j][k] = ((((u+d) + (n+s)) + ((w+e) + (c+c))) * 0.125f with u/d = src[i-1/i+1][j][k],
@@ -157,6 +162,7 @@ typedef struct accmg_access {
 #define ACCMG_BODY_KMEANS_UPDATE     4
 #define ACCMG_BODY_SCATTER           5
 #define ACCMG_BODY_JACOBI3D_7PT      6
+#define ACCMG_BODY_JACOBI2D_DEEP     7
 #define ACCMG_BODY_TEST_SPARSE_WRITE 100
 
 typedef struct { int64_t rows, cols; } accmg_args_jacobi2d;
@@ -165,6 +171,7 @@ typedef struct { int64_t n; int32_t d, k, shift, pad; } accmg_args_kmeans;
 typedef struct { int64_t rows, cols, period; } accmg_args_sparse;
 typedef struct { int64_t n, m; } accmg_args_scatter;
 typedef struct { int64_t n0, n1, n2; } accmg_args_jacobi3d;
+typedef struct { int64_t rows, cols, h; } accmg_args_jacobi2d_deep;
 
 /* ---- statistics (E5-style breakdown, L188; device memory User/System, L249) ------------------
  * Byte counters are this process's: pulls into its partitions (receiver-counted), packets its

@@ -28,6 +28,7 @@ R, W, RW, REDUCE_SUM = 1, 2, 3, 4
 BODY_JACOBI2D_5PT, BODY_GEMM_BF16_F32, BODY_KMEANS_ASSIGN, BODY_KMEANS_UPDATE = 1, 2, 3, 4
 BODY_SCATTER = 5
 BODY_JACOBI3D_7PT = 6
+BODY_JACOBI2D_DEEP = 7
 BODY_TEST_SPARSE_WRITE = 100
 
 
@@ -67,6 +68,10 @@ class accmg_args_sparse(ctypes.Structure):
 
 class accmg_args_jacobi3d(ctypes.Structure):
     _fields_ = [("n0", ctypes.c_int64), ("n1", ctypes.c_int64), ("n2", ctypes.c_int64)]
+
+
+class accmg_args_jacobi2d_deep(ctypes.Structure):
+    _fields_ = [("rows", ctypes.c_int64), ("cols", ctypes.c_int64), ("h", ctypes.c_int64)]
 
 
 class accmg_args_scatter(ctypes.Structure):

@@ -177,6 +177,26 @@ cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, i
     return e;
 }
 
+namespace {
+__global__ void frame_copy_k(const float* __restrict__ src, float* __restrict__ tmp, int64_t cols, int64_t lo,
+                             int64_t hi, int64_t rlo, int64_t rhi, int64_t c0, int64_t c1) {
+    for (int64_t r = lo + blockIdx.x; r < hi; r += gridDim.x) {
+        const bool whole = r < rlo || r >= rhi;
+        for (int64_t c = threadIdx.x; c < cols; c += blockDim.x)
+            if (whole || c < c0 || c >= c1) tmp[r * cols + c] = src[r * cols + c];
+    }
+}
+}  // namespace
+
+cudaError_t frame_copy(const float* src, float* tmp, int64_t cols, int64_t lo, int64_t hi, int64_t rlo, int64_t rhi,
+                       int64_t c0, int64_t c1, cudaStream_t s, int64_t* launches) {
+    if (hi <= lo) return cudaSuccess;
+    const int64_t nb = (hi - lo) < 1184 ? (hi - lo) : 1184;
+    frame_copy_k<<<(unsigned)nb, 256, 0, s>>>(src, tmp, cols, lo, hi, rlo, rhi, c0, c1);
+    if (launches) *launches += 1;
+    return cudaGetLastError();
+}
+
 cudaError_t sparse_rows(const float* in, float* out, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
                         int64_t period, Track t, cudaStream_t s, int64_t* launches) {
     (void)rows;

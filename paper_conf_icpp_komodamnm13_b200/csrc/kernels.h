@@ -42,6 +42,18 @@ cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64
                      int64_t jl, int64_t jh, int64_t kl, int64_t kh, int64_t src_lo, int64_t src_hi, Track t,
                      cudaStream_t s, int64_t* launches);
 
+// Deep-halo body fused: h sweeps per tile in shared memory (TMA-loaded), rows [r0, r1) of dst
+// from src; update box rows [rlo, rhi), columns [c0, c1). cudaErrorNotSupported if the shape does
+// not fit (cols % 4, cols < 128, h > 8): the caller then runs h single sweeps.
+cudaError_t jacobi2d_deep(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
+                          int64_t rlo, int64_t rhi, int64_t c0, int64_t c1, int h, int64_t src_lo, int64_t src_hi,
+                          Track t, cudaStream_t s, int64_t* launches);
+
+// Deep-halo scratch frame: rows [lo, hi) of tmp get src's values outside the update box
+// (rows outside [rlo, rhi) entirely, columns outside [c0, c1) of the others).
+cudaError_t frame_copy(const float* src, float* tmp, int64_t cols, int64_t lo, int64_t hi, int64_t rlo, int64_t rhi,
+                       int64_t c0, int64_t c1, cudaStream_t s, int64_t* launches);
+
 // Test body: rows i in [r0, r1) with i % period == 0: out[i][:] = in[i][:] + 1.0f.
 cudaError_t sparse_rows(const float* in, float* out, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
                         int64_t period, Track t, cudaStream_t s, int64_t* launches);

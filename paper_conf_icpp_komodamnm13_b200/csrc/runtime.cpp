@@ -111,6 +111,13 @@ struct State {
     uint8_t* recv = nullptr;
     int64_t recv_cap = 0;
     // write-miss system buffers (L137): per local partition {index, value} records + counters
+    // deep-halo scratch (two buffers per local partition, global-index bases)
+    struct Deep {
+        float* base[2] = {nullptr, nullptr};
+        uint8_t* alloc[2] = {nullptr, nullptr};
+        int64_t lo = 0, hi = 0;
+    };
+    std::vector<Deep> deep;
     std::vector<uint64_t*> miss_recs;
     int64_t miss_base = 0;
     int64_t miss_cap = 0;
@@ -497,6 +504,36 @@ int ensure_recv(int64_t bytes) {
     return 0;
 }
 
+// ACCMG_DEEP_IMPL: 1 (default) fused shared-memory sweeps where the shape allows, 0 = h
+// single-sweep launches through scratch buffers (kept for comparison and as the general path).
+int deep_impl() {
+    static const int v = [] {
+        const char* e = getenv("ACCMG_DEEP_IMPL");
+        return e ? atoi(e) : 1;
+    }();
+    return v;
+}
+
+// Scratch for the deep-halo body: element range [lo, hi) in two buffers (grow-only, system memory).
+int ensure_deep(int li, int64_t lo, int64_t hi) {
+    if ((int)S.deep.size() < S.V) S.deep.resize(S.V);
+    auto& D = S.deep[li];
+    if (D.alloc[0] && lo >= D.lo && hi <= D.hi) return 0;
+    if (D.alloc[0]) {
+        CUDA_TRY(cudaStreamSynchronize(S.stream));
+        lo = std::min(lo, D.lo);
+        hi = std::max(hi, D.hi);
+        for (int q = 0; q < 2; ++q) dfree(D.alloc[q], (D.hi - D.lo) * 4, true);
+    }
+    for (int q = 0; q < 2; ++q) {
+        TRY(dmalloc((void**)&D.alloc[q], (size_t)(hi - lo) * 4, true));
+        D.base[q] = reinterpret_cast<float*>(D.alloc[q]) - lo;
+    }
+    D.lo = lo;
+    D.hi = hi;
+    return 0;
+}
+
 k::Track track_of(accmg_region_s* r, int li, bool on) {
     static int dbg = -1;
     if (dbg < 0) {
@@ -536,6 +573,7 @@ bool body_spec(int id, BodySpec* b) {
         case ACCMG_BODY_TEST_SPARSE_WRITE: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 1, sizeof(accmg_args_sparse)}; return true;
         case ACCMG_BODY_SCATTER: *b = {3, {ACCMG_R, ACCMG_R, ACCMG_W}, {4, 4, 4}, 1, sizeof(accmg_args_scatter)}; return true;
         case ACCMG_BODY_JACOBI3D_7PT: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 3, sizeof(accmg_args_jacobi3d)}; return true;
+        case ACCMG_BODY_JACOBI2D_DEEP: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 2, sizeof(accmg_args_jacobi2d_deep)}; return true;
         default: return false;
     }
 }
@@ -551,6 +589,15 @@ int validate_body(const accmg_bounds* bd, int body, const accmg_access* d, const
             if (bd->lo[0] < 1 || bd->hi[0] > a->rows - 1 || bd->lo[1] < 1 || bd->hi[1] > a->cols - 1)
                 return bad("jacobi: bounds must lie in [1,rows-1) x [1,cols-1)");
             if (d[0].region == d[1].region) return bad("jacobi: src and dst must differ");
+            return 0;
+        }
+        case ACCMG_BODY_JACOBI2D_DEEP: {
+            auto a = static_cast<const accmg_args_jacobi2d_deep*>(args);
+            if (a->rows < 3 || a->cols < 3 || a->h < 1 || a->h > 64) return bad("jacobi_deep: rows, cols >= 3, 1 <= h <= 64");
+            if (ext(0) != a->rows * a->cols || ext(1) != a->rows * a->cols) return bad("jacobi_deep: region extent != rows*cols");
+            if (bd->lo[0] < 1 || bd->hi[0] > a->rows - 1 || bd->lo[1] < 1 || bd->hi[1] > a->cols - 1)
+                return bad("jacobi_deep: bounds must lie in [1,rows-1) x [1,cols-1)");
+            if (d[0].region == d[1].region) return bad("jacobi_deep: src and dst must differ");
             return 0;
         }
         case ACCMG_BODY_TEST_SPARSE_WRITE: {
@@ -627,6 +674,39 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
             const Ival al = d[0].region->arange[g];
             e = k::jacobi2d((const float*)P(0), (float*)P(1), x->rows, x->cols, a, b, bd->lo[1], bd->hi[1], al.lo, al.hi,
                             T(1), 0, S.stream, L);
+            break;
+        }
+        case ACCMG_BODY_JACOBI2D_DEEP: {
+            // h sweeps: src -> tmp -> tmp' -> ... -> dst over shrinking row ranges; the scratch
+            // buffers hold rows [a-h, b+h) (global-index bases) with src's fixed frame
+            auto x = static_cast<const accmg_args_jacobi2d_deep*>(args);
+            const int64_t C = x->cols, h = x->h, rlo = bd->lo[0], rhi = bd->hi[0];
+            const int64_t lo = std::max<int64_t>(a - h, 0), hi = std::min<int64_t>(b + h, x->rows);
+            const Ival al = d[0].region->arange[g];
+            if (deep_impl() == 1 && h > 1) {  // fused: h sweeps per tile in shared memory
+                e = k::jacobi2d_deep((const float*)P(0), (float*)P(1), x->rows, C, a, b, rlo, rhi, bd->lo[1],
+                                     bd->hi[1], (int)h, al.lo, al.hi, T(1), S.stream, L);
+                if (e != cudaErrorNotSupported) break;
+                e = cudaSuccess;
+            }
+            TRY(ensure_deep(li, lo * C, hi * C));
+            float* tmp[2] = {S.deep[li].base[0], S.deep[li].base[1]};
+            if (h > 1) {
+                for (int q = 0; q < 2; ++q)
+                    CUDA_TRY(k::frame_copy((const float*)P(0), tmp[q], C, lo, hi, rlo, rhi, bd->lo[1], bd->hi[1], S.stream, L));
+            }
+            const float* in = (const float*)P(0);
+            int64_t in_lo = al.lo, in_hi = al.hi;
+            for (int64_t kk = 1; kk <= h && e == cudaSuccess; ++kk) {
+                const bool last = kk == h;
+                float* out = last ? (float*)P(1) : tmp[kk % 2];
+                const int64_t r0 = std::max<int64_t>(a - (h - kk), rlo), r1 = std::min<int64_t>(b + (h - kk), rhi);
+                e = k::jacobi2d(in, out, x->rows, C, r0, r1, bd->lo[1], bd->hi[1], in_lo, in_hi, last ? T(1) : k::Track{},
+                                0, S.stream, L);
+                in = out;
+                in_lo = lo * C;
+                in_hi = hi * C;
+            }
             break;
         }
         case ACCMG_BODY_TEST_SPARSE_WRITE: {
@@ -1037,6 +1117,8 @@ int accmg_finalize(void) {
         dfree(S.d_sizes, 0, true);
         dfree(S.d_flag, 0, true);
         dfree(S.d_miss, 0, true);
+        for (auto& D : S.deep)
+            for (int q = 0; q < 2; ++q) dfree(D.alloc[q], (D.hi - D.lo) * 4, true);
         for (auto p : S.miss_recs) dfree(p, 0, true);
         dfree(S.recv, 0, true);
         if (S.h_pin) cudaFreeHost(S.h_pin);

@@ -46,6 +46,35 @@ def jacobi_run(Ahost: np.ndarray, Bhost: np.ndarray, sweeps: int, declared: bool
     return per
 
 
+def jacobi_deep_descs(src, dst, N: int, h: int, declared: bool = True):
+    """Deep halos (§8 f2): h sweeps per loop need rows i-h..i+h (stride N, left = right = h*N)."""
+    return [A.access(src, A.R, declared, N, h * N, h * N), A.access(dst, A.W, declared, N, 0, 0)]
+
+
+def jacobi_deep_loop(rA, rB, s: int, N: int, h: int, declared: bool = True) -> None:
+    """Loop s of a deep-halo run: dst = J^h(src), alternating A -> B -> A."""
+    src, dst = (rA, rB) if s % 2 == 0 else (rB, rA)
+    A.accmg_loop_launch(A.bounds([1, 1], [N - 1, N - 1]), A.BODY_JACOBI2D_DEEP,
+                        jacobi_deep_descs(src, dst, N, h, declared), A.accmg_args_jacobi2d_deep(N, N, h))
+
+
+def jacobi_deep_run(Ahost: np.ndarray, Bhost: np.ndarray, sweeps: int, h: int, declared: bool = True):
+    """`sweeps` Jacobi sweeps (a multiple of h) as sweeps/h deep-halo loops; the result lands in
+    Ahost when sweeps/h is even, else in Bhost (as jacobi_run with sweeps/h sweeps)."""
+    if sweeps % h:
+        raise ValueError("sweeps must be a multiple of h")
+    N = Ahost.shape[0]
+    rA, rB = A.accmg_region_create(Ahost), A.accmg_region_create(Bhost)
+    try:
+        for s in range(sweeps // h):
+            jacobi_deep_loop(rA, rB, s, N, h, declared)
+        A.accmg_sync_to_host(rA)
+        A.accmg_sync_to_host(rB)
+    finally:
+        A.accmg_region_destroy(rA)
+        A.accmg_region_destroy(rB)
+
+
 def kmeans_loops(rx, rcen, rmem, rsum, rcnt, n: int, d: int, k: int, shift: int = 8) -> None:
     """One k-means iteration = the paper's 2 parallel loops (Table II: KMEANS has 2 loops)."""
     args = A.accmg_args_kmeans(n, d, k, shift, 0)

@@ -185,3 +185,27 @@ def test_scatter_requires_declared_dst(dry):
     assert e.value.code == A.EUNSUPPORTED
     from paper_conf_icpp_komodamnm13_b200 import workloads as WL
     WL.scatter_loop(*regs, n, n)   # declared: accepted (dry run: planning only)
+
+
+@pytest.mark.parametrize("P,h", [(2, 2), (4, 3), (8, 8)])
+def test_deep_halo_plan_vs_model(dry, P, h):
+    """Deep-halo loops (§8 f2): the window of h rows per side, planned as the model plans it."""
+    N = 48
+    dry(P)
+    hA, hB = np.zeros((N, N), np.float32), np.zeros((N, N), np.float32)
+    rA, rB = A.accmg_region_create(hA), A.accmg_region_create(hB)
+    mdl = M.Model(P)
+    mA, mB = mdl.region(N * N, 4), mdl.region(N * N, 4)
+    for s in range(4):
+        before = A.accmg_get_stats()
+        WL.jacobi_deep_loop(rA, rB, s, N, h)
+        after = A.accmg_get_stats()
+        src, dst = (mA, mB) if s % 2 == 0 else (mB, mA)
+        exp = mdl.loop(1, N - 1, [(src, M.R, 1, N, h * N, h * N), (dst, M.W, 1, N, 0, 0)])
+        assert after["bytes_declared"] - before["bytes_declared"] == exp["declared"]
+        assert after["bytes_h2d"] - before["bytes_h2d"] == exp["h2d"]
+        _compare_valid([rA, rB], [mA, mB], P)
+    with pytest.raises(A.AccmgError) as e:
+        A.accmg_loop_launch(A.bounds([1, 1], [N - 1, N - 1]), A.BODY_JACOBI2D_DEEP,
+                            WL.jacobi_deep_descs(rA, rB, N, h), A.accmg_args_jacobi2d_deep(N, N, 0))
+    assert e.value.code == A.EINVAL
