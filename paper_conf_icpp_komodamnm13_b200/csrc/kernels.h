@@ -49,6 +49,12 @@ cudaError_t jacobi2d_deep(const float* src, float* dst, int64_t rows, int64_t co
                           int64_t rlo, int64_t rhi, int64_t c0, int64_t c1, int h, int64_t src_lo, int64_t src_hi,
                           Track t, cudaStream_t s, int64_t* launches);
 
+// Same operation, register-streamed temporal blocking (one warp per 128-column strip marching
+// down the rows, all h levels advanced per input row); 2 <= h <= 8.
+cudaError_t jacobi2d_deep_stream(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
+                                 int64_t rlo, int64_t rhi, int64_t c0, int64_t c1, int h, int64_t src_lo,
+                                 int64_t src_hi, Track t, cudaStream_t s, int64_t* launches);
+
 // Deep-halo scratch frame: rows [lo, hi) of tmp get src's values outside the update box
 // (rows outside [rlo, rhi) entirely, columns outside [c0, c1) of the others).
 cudaError_t frame_copy(const float* src, float* tmp, int64_t cols, int64_t lo, int64_t hi, int64_t rlo, int64_t rhi,

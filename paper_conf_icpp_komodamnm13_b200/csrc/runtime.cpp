@@ -504,12 +504,13 @@ int ensure_recv(int64_t bytes) {
     return 0;
 }
 
-// ACCMG_DEEP_IMPL: 1 (default) fused shared-memory sweeps where the shape allows, 0 = h
-// single-sweep launches through scratch buffers (kept for comparison and as the general path).
+// ACCMG_DEEP_IMPL: 2 (default) register-streamed temporal blocking, 1 = levels through shared
+// memory per tile, 0 = h single-sweep launches through scratch buffers (the general path, also
+// taken by the fused kernels' unsupported shapes).
 int deep_impl() {
     static const int v = [] {
         const char* e = getenv("ACCMG_DEEP_IMPL");
-        return e ? atoi(e) : 1;
+        return e ? atoi(e) : 2;
     }();
     return v;
 }
@@ -683,9 +684,10 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
             const int64_t C = x->cols, h = x->h, rlo = bd->lo[0], rhi = bd->hi[0];
             const int64_t lo = std::max<int64_t>(a - h, 0), hi = std::min<int64_t>(b + h, x->rows);
             const Ival al = d[0].region->arange[g];
-            if (deep_impl() == 1 && h > 1) {  // fused: h sweeps per tile in shared memory
-                e = k::jacobi2d_deep((const float*)P(0), (float*)P(1), x->rows, C, a, b, rlo, rhi, bd->lo[1],
-                                     bd->hi[1], (int)h, al.lo, al.hi, T(1), S.stream, L);
+            if (deep_impl() >= 1 && h > 1) {  // fused: h sweeps per launch without scratch
+                auto fused = deep_impl() == 2 ? k::jacobi2d_deep_stream : k::jacobi2d_deep;
+                e = fused((const float*)P(0), (float*)P(1), x->rows, C, a, b, rlo, rhi, bd->lo[1], bd->hi[1], (int)h,
+                          al.lo, al.hi, T(1), S.stream, L);
                 if (e != cudaErrorNotSupported) break;
                 e = cudaSuccess;
             }
