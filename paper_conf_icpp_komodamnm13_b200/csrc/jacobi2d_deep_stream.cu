@@ -13,7 +13,7 @@
 // slot of row j is j mod 3 at compile time and no register is ever copied. Nothing but the input
 // rows passes through shared memory and only the final level reaches HBM, so h sweeps cost one read
 // and one write of the field; the per-level cost is two shuffles and 16 FP32 operations per 4
-// points. Warps are independent (no CTA barrier): a persistent grid of 16 (h <= 6) or 12 warps per SM
+// points (6 paired FP32 instructions in the interior). Warps are independent (no CTA barrier): a persistent grid of 16 (h <= 6) or 12 warps per SM
 // walks the (strip, segment) items, neighbouring warps on neighbouring strips (shared halo columns
 // hit L2).
 //
@@ -39,13 +39,46 @@ constexpr int kStages = 4;    // per-warp ring
 // registers of level state alone, so they run 1 x 12 warps with up to 168 registers (no spills)
 template <int H> struct Cfg { static constexpr int NW = H >= 7 ? 12 : 8, MINB = H >= 7 ? 1 : 2; };
 constexpr int kMaxWarps = 12;
-constexpr int kSeg = 512;     // output rows per item
+constexpr int kSegMax = 512;  // output rows per item (fewer when a partition is short: balance)
 constexpr int kStageFloats = RS * W;
 constexpr uint32_t kStageBytes = kStageFloats * 4;
 
 __device__ __forceinline__ float st5(float n, float s, float w, float e) {
     return __fmul_rn(__fadd_rn(__fadd_rn(n, s), __fadd_rn(w, e)), 0.25f);
 }
+
+// Level rows live as two packed pairs P = (x, z), Q = (y, w) of a lane's four columns x, y, z, w:
+// the horizontal sums then pair up as (w_in + y, y + w) = (w_in, y) + Q and (x + z, z + e_in) =
+// P + (z, e_in), so a level costs 6 paired FP32 instructions (PTX add/mul.rn.f32x2: per-lane IEEE
+// round-to-nearest, no flush — the bits of the scalar __fadd_rn / __fmul_rn sequence), two
+// shuffles and two register moves per 4 points.
+struct V4 {
+    uint64_t p, q;
+};
+
+__device__ __forceinline__ uint64_t pk(float a, float b) {
+    uint64_t r;
+    asm("mov.b64 %0, {%1, %2};" : "=l"(r) : "f"(a), "f"(b));
+    return r;
+}
+__device__ __forceinline__ void upk(uint64_t v, float& a, float& b) { asm("mov.b64 {%0, %1}, %2;" : "=f"(a), "=f"(b) : "l"(v)); }
+__device__ __forceinline__ uint64_t add2(uint64_t a, uint64_t b) {
+    uint64_t r;
+    asm("add.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ uint64_t mul2(uint64_t a, uint64_t b) {
+    uint64_t r;
+    asm("mul.rn.f32x2 %0, %1, %2;" : "=l"(r) : "l"(a), "l"(b));
+    return r;
+}
+__device__ __forceinline__ float4 to4(const V4& v) {
+    float4 f;
+    upk(v.p, f.x, f.z);
+    upk(v.q, f.y, f.w);
+    return f;
+}
+__device__ __forceinline__ V4 from4(const float4& f) { return V4{pk(f.x, f.z), pk(f.y, f.w)}; }
 
 struct Item {
     unsigned upd, onib;  // lane columns inside the update box / outputs of this strip
@@ -75,9 +108,26 @@ __device__ __forceinline__ float4 jstep(const float4& N, const float4& C, const 
     return o;
 }
 
+template <bool MASK>
+__device__ __forceinline__ V4 jstep2(const V4& N, const V4& C, const V4& S, int j, const Item& it) {
+    if constexpr (MASK) {
+        return from4(jstep<true>(to4(N), to4(C), to4(S), j, it));
+    } else {
+        float x, y, z, w;
+        upk(C.p, x, z);
+        upk(C.q, y, w);
+        const float win = __shfl_up_sync(dev::kFull, w, 1);
+        const float ein = __shfl_down_sync(dev::kFull, x, 1);
+        const uint64_t quarter = 0x3E8000003E800000ull;  // (0.25f, 0.25f)
+        const uint64_t p = add2(add2(N.p, S.p), add2(pk(win, y), C.q));  // x: (n+s)+(w_in+y); z: (n+s)+(y+w)
+        const uint64_t q = add2(add2(N.q, S.q), add2(C.p, pk(z, ein)));  // y: (n+s)+(x+z); w: (n+s)+(z+e_in)
+        return V4{mul2(p, quarter), mul2(q, quarter)};
+    }
+}
+
 // One input row (local index i, i % 3 == PH) through all H levels.
 template <int H, int PH, bool MASK, bool TRACK>
-__device__ __forceinline__ void advance(float4 (&Lv)[H][3], const float4& X, int i, const Item& it,
+__device__ __forceinline__ void advance(V4 (&Lv)[H][3], const V4& X, int i, const Item& it,
                                         dev::WarpTracker<4>& trk, const Track& t) {
     Lv[0][PH] = X;
 #pragma unroll
@@ -85,20 +135,21 @@ __device__ __forceinline__ void advance(float4 (&Lv)[H][3], const float4& X, int
         // level l row j = i - l from level l-1 rows j-1, j, j+1 (slots (PH - l - 1..PH - l + 1) mod 3)
         const int sj = ((PH - l) % 3 + 3) % 3;
         const int sn = (sj + 2) % 3, ss = (sj + 1) % 3;
-        const float4 Y = jstep<MASK>(Lv[l - 1][sn], Lv[l - 1][sj], Lv[l - 1][ss], i - l, it);
+        const V4 Y = jstep2<MASK>(Lv[l - 1][sn], Lv[l - 1][sj], Lv[l - 1][ss], i - l, it);
         if (l < H) {
             Lv[l][sj] = Y;
         } else {
             const int j = i - H;
             if (j >= it.out_lo && j < it.out_hi) {  // warp-uniform
                 float* p = it.gdst + (int64_t)j * it.cols;
+                const float4 f = to4(Y);
                 if (it.onib == 0xFu) {
-                    *reinterpret_cast<float4*>(p) = Y;
+                    *reinterpret_cast<float4*>(p) = f;
                 } else if (it.onib) {
-                    if (it.onib & 1u) p[0] = Y.x;
-                    if (it.onib & 2u) p[1] = Y.y;
-                    if (it.onib & 4u) p[2] = Y.z;
-                    if (it.onib & 8u) p[3] = Y.w;
+                    if (it.onib & 1u) p[0] = f.x;
+                    if (it.onib & 2u) p[1] = f.y;
+                    if (it.onib & 4u) p[2] = f.z;
+                    if (it.onib & 8u) p[3] = f.w;
                 }
                 if constexpr (TRACK) trk.mark(t.l1, t.l2, t.l2_shift, it.e0 + (int64_t)j * it.cols);
             }
@@ -110,11 +161,11 @@ template <int H, bool MASK, bool TRACK>
 __device__ __forceinline__ void run_item(const CUtensorMap* map, uint64_t* bar, float* ring, int nst, uint32_t& g,
                                          int64_t kt, int64_t row0_map, const Item& it, const Track& t) {
     const int lane = threadIdx.x & 31;
-    float4 Lv[H][3];
+    V4 Lv[H][3];
 #pragma unroll
     for (int l = 0; l < H; ++l)
 #pragma unroll
-        for (int q = 0; q < 3; ++q) Lv[l][q] = make_float4(0.f, 0.f, 0.f, 0.f);
+        for (int q = 0; q < 3; ++q) Lv[l][q] = V4{0ull, 0ull};
     dev::WarpTracker<4> trk;
     if constexpr (TRACK) trk.init(it.onib);
     // prologue: the first kStages stages of this item (all slots are free here)
@@ -132,9 +183,9 @@ __device__ __forceinline__ void run_item(const CUtensorMap* map, uint64_t* bar, 
         const int i0 = s * RS;
 #pragma unroll
         for (int rr = 0; rr < RS; rr += 3) {
-            const float4 X0 = *reinterpret_cast<const float4*>(T + (rr + 0) * W);
-            const float4 X1 = *reinterpret_cast<const float4*>(T + (rr + 1) * W);
-            const float4 X2 = *reinterpret_cast<const float4*>(T + (rr + 2) * W);
+            const V4 X0 = from4(*reinterpret_cast<const float4*>(T + (rr + 0) * W));
+            const V4 X1 = from4(*reinterpret_cast<const float4*>(T + (rr + 1) * W));
+            const V4 X2 = from4(*reinterpret_cast<const float4*>(T + (rr + 2) * W));
             advance<H, 0, MASK, TRACK>(Lv, X0, i0 + rr + 0, it, trk, t);
             advance<H, 1, MASK, TRACK>(Lv, X1, i0 + rr + 1, it, trk, t);
             advance<H, 2, MASK, TRACK>(Lv, X2, i0 + rr + 2, it, trk, t);
@@ -154,7 +205,7 @@ template <int H, bool TRACK>
 __global__ void __launch_bounds__(Cfg<H>::NW * 32, Cfg<H>::MINB)
 deep_stream_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, int64_t cols, int64_t r0, int64_t r1,
               int64_t rlo, int64_t rhi, int64_t c0, int64_t c1, int64_t cbase, int64_t row_lo, int hc, int nstrips,
-              int nsegs, Track t) {
+              int nsegs, int kSeg, Track t) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     constexpr int kWarps = Cfg<H>::NW;
     __shared__ __align__(8) uint64_t bars[kMaxWarps][kStages];
@@ -207,7 +258,7 @@ deep_stream_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, 
 
 template <int H>
 cudaError_t launch_h(const CUtensorMap& map, float* dst, int64_t cols, int64_t r0, int64_t r1, int64_t rlo, int64_t rhi,
-                     int64_t c0, int64_t c1, int64_t cbase, int64_t row_lo, int hc, int nstrips, int nsegs, Track t,
+                     int64_t c0, int64_t c1, int64_t cbase, int64_t row_lo, int hc, int nstrips, Track t,
                      cudaStream_t s) {
     auto kern = t.l1 ? deep_stream_k<H, true> : deep_stream_k<H, false>;
     constexpr int kWarps = Cfg<H>::NW;
@@ -217,10 +268,28 @@ cudaError_t launch_h(const CUtensorMap& map, float* dst, int64_t cols, int64_t r
     int dev = 0, nsm = 148;
     cudaGetDevice(&dev);
     cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    // segment length: items are equal, so time ~ waves x rows per item = ceil(items / resident
+    // warps) x (seg + 2h); pick the segment count minimising that (short partitions — 4096 rows of
+    // C2 at P = 8 — would otherwise run 1.3 waves of 512-row items)
+    const int64_t twarps = (int64_t)Cfg<H>::MINB * nsm * kWarps;
+    const int64_t nrows = r1 - r0;
+    int nsegs = 1;
+    double best = 1e300;
+    for (int64_t ns = (nrows + kSegMax - 1) / kSegMax; ns <= std::max<int64_t>(1, nrows / 32); ++ns) {
+        const int64_t sg = (nrows + ns - 1) / ns;
+        const int64_t waves = (ns * nstrips + twarps - 1) / twarps;
+        const double cost = (double)waves * (double)(sg + 2 * H);
+        if (cost < best * 0.999) {
+            best = cost;
+            nsegs = (int)ns;
+        }
+        if (waves > 64) break;
+    }
+    const int seg = (int)((nrows + nsegs - 1) / nsegs);
     const int nitems = nstrips * nsegs;
     const int grid = std::max(1, std::min(Cfg<H>::MINB * nsm, (nitems + kWarps - 1) / kWarps));
     kern<<<grid, kWarps * 32, smem, s>>>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, nsegs,
-                                          t);
+                                          seg, t);
     return cudaGetLastError();
 }
 
@@ -250,16 +319,15 @@ cudaError_t jacobi2d_deep_stream(const float* src, float* dst, int64_t rows, int
     const int64_t cbase = (c0 / 4) * 4;
     const int TK = W - 2 * hc;
     const int nstrips = (int)((c1 - cbase + TK - 1) / TK);
-    const int nsegs = (int)((r1 - r0 + kSeg - 1) / kSeg);
     cudaError_t e;
     switch (h) {
-        case 2: e = launch_h<2>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, nsegs, t, s); break;
-        case 3: e = launch_h<3>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, nsegs, t, s); break;
-        case 4: e = launch_h<4>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, nsegs, t, s); break;
-        case 5: e = launch_h<5>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, nsegs, t, s); break;
-        case 6: e = launch_h<6>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, nsegs, t, s); break;
-        case 7: e = launch_h<7>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, nsegs, t, s); break;
-        default: e = launch_h<8>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, nsegs, t, s); break;
+        case 2: e = launch_h<2>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, t, s); break;
+        case 3: e = launch_h<3>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, t, s); break;
+        case 4: e = launch_h<4>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, t, s); break;
+        case 5: e = launch_h<5>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, t, s); break;
+        case 6: e = launch_h<6>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, t, s); break;
+        case 7: e = launch_h<7>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, t, s); break;
+        default: e = launch_h<8>(map, dst, cols, r0, r1, rlo, rhi, c0, c1, cbase, row_lo, hc, nstrips, t, s); break;
     }
     if (launches) *launches += 1;
     return e;
