@@ -128,6 +128,15 @@ def permutation(seed: int, n: int) -> np.ndarray:
     return out
 
 
+def write_mask(seed: int, n: int, density: float, run: int = 1) -> np.ndarray:
+    """uint8 mask of n elements in segments of `run` elements: segment s is set iff
+    (u(seed, s) >> 40) < density * 2^24 (so density 1 sets everything, 0 nothing)."""
+    nseg = (n + run - 1) // run
+    thr = int(density * (1 << 24))
+    seg = ((u_fill(seed, 0, nseg) >> np.uint64(40)) < np.uint64(thr)).astype(np.uint8)
+    return np.repeat(seg, run)[:n].copy()
+
+
 def bf16_to_f32(a: np.ndarray) -> np.ndarray:
     """Exact widening of bf16 bit patterns to fp32 (a bit shift, no rounding)."""
     return (a.astype(np.uint32) << 16).view(np.float32)

@@ -155,6 +155,9 @@ typedef struct accmg_access {
  *   lie in some partition's window of dst.
  * ACCMG_BODY_TEST_SPARSE_WRITE: bounds ndim=1 rows [0,R); descs [in R (fp32 R*C), out W (fp32 R*C)];
  *   rows i with i % period == 0: out[i][j] = in[i][j] + 1.0f for all j (exercises L2 chunk skipping).
+ * ACCMG_BODY_TEST_MASKED_WRITE: bounds ndim=1 [0,n); descs [in R (fp32 n), mask R (uint8 n),
+ *   out W (fp32 n)]; out[e] = in[e] + 1.0f where mask[e] != 0 (arbitrary dirty-bit patterns for
+ *   the compaction of L133-135: isolated bits, runs across words, tiles and chunks). args {n}.
  */
 #define ACCMG_BODY_JACOBI2D_5PT      1
 #define ACCMG_BODY_GEMM_BF16_F32     2
@@ -164,11 +167,13 @@ typedef struct accmg_access {
 #define ACCMG_BODY_JACOBI3D_7PT      6
 #define ACCMG_BODY_JACOBI2D_DEEP     7
 #define ACCMG_BODY_TEST_SPARSE_WRITE 100
+#define ACCMG_BODY_TEST_MASKED_WRITE 101
 
 typedef struct { int64_t rows, cols; } accmg_args_jacobi2d;
 typedef struct { int64_t M, N, K; } accmg_args_gemm;
 typedef struct { int64_t n; int32_t d, k, shift, pad; } accmg_args_kmeans;
 typedef struct { int64_t rows, cols, period; } accmg_args_sparse;
+typedef struct { int64_t n; } accmg_args_masked;
 typedef struct { int64_t n, m; } accmg_args_scatter;
 typedef struct { int64_t n0, n1, n2; } accmg_args_jacobi3d;
 typedef struct { int64_t rows, cols, h; } accmg_args_jacobi2d_deep;

@@ -39,6 +39,7 @@ def lib() -> ctypes.CDLL:
         L.orc_jacobi_run.argtypes = [vp, vp, i64, i32, i32]
         L.orc_jacobi_sweep_rect.argtypes = [vp, vp, i64, i64, i32]
         L.orc_sparse_rows.argtypes = [vp, vp, i64, i64, i32, vp]
+        L.orc_masked_write.argtypes = [vp, vp, vp, i64, i32, vp]
         L.orc_gemm_rows_f64.argtypes = [vp, vp, i64, i64, i64, vp, i64, vp, i32]
         L.orc_kmeans_assign.argtypes = [vp, i64, i32, i32, vp, vp, i32]
         L.orc_kmeans_update.argtypes = [vp, i64, i32, i32, vp, vp, vp, vp]
@@ -129,6 +130,15 @@ def sparse_rows(inp: np.ndarray, out: np.ndarray, period: int, P: int = 1, track
     N = inp.shape[0]
     bms = np.zeros((P, nwords(N * N)), dtype=np.uint32) if track else None
     lib().orc_sparse_rows(inp.ctypes.data, out.ctypes.data, N, period, P, _p(bms))
+    return bms
+
+
+def masked_write(inp: np.ndarray, mask: np.ndarray, out: np.ndarray, P: int = 1, track: bool = False):
+    """out[e] = inp[e] + 1 where mask[e] (flat arrays, in place on out); P bitmaps if track."""
+    n = inp.size
+    assert inp.dtype == np.float32 and out.dtype == np.float32 and mask.dtype == np.uint8
+    bms = np.zeros((P, nwords(n)), dtype=np.uint32) if track else None
+    lib().orc_masked_write(inp.ctypes.data, mask.ctypes.data, out.ctypes.data, n, P, _p(bms))
     return bms
 
 

@@ -176,6 +176,19 @@ void orc_sparse_rows(const float* in, float* out, int64_t N, int64_t period, int
     }
 }
 
+/* Masked-write test loop (exercises the dirty-bit compaction of L133-135 with arbitrary bit
+ * patterns): iterations e in [0, n); iteration e writes only if mask[e] != 0:
+ *   out[e] = in[e] + 1.0f.   Bit e of partition orc_owner(0, n, P, e)'s bitmap is set per write.
+ * pin: tests — brute-force Python loop on small n, bitmaps = mask bits split by partition. */
+void orc_masked_write(const float* in, const uint8_t* mask, float* out, int64_t n, int P, uint32_t* bitmaps) {
+    int64_t nwords = (n + 31) / 32;
+    for (int64_t e = 0; e < n; ++e) {
+        if (!mask[e]) continue;
+        out[e] = in[e] + 1.0f;
+        if (bitmaps) set_bit(bitmaps + (int64_t)orc_owner(0, n, P, e) * nwords, e);
+    }
+}
+
 /* ------------------------------------------------------------------------------------ */
 /* Dense matmul (config C3): R[i][j] = sum_{k=0}^{K-1} (double)A[i][k] * (double)B[k][j],
  * k ascending, fp64. A, B are bf16 bit patterns (row-major [M][K], [K][N]); bf16 -> fp64 is

@@ -30,6 +30,7 @@ BODY_SCATTER = 5
 BODY_JACOBI3D_7PT = 6
 BODY_JACOBI2D_DEEP = 7
 BODY_TEST_SPARSE_WRITE = 100
+BODY_TEST_MASKED_WRITE = 101
 
 
 class accmg_config(ctypes.Structure):
@@ -64,6 +65,10 @@ class accmg_args_kmeans(ctypes.Structure):
 
 class accmg_args_sparse(ctypes.Structure):
     _fields_ = [("rows", ctypes.c_int64), ("cols", ctypes.c_int64), ("period", ctypes.c_int64)]
+
+
+class accmg_args_masked(ctypes.Structure):
+    _fields_ = [("n", ctypes.c_int64)]
 
 
 class accmg_args_jacobi3d(ctypes.Structure):

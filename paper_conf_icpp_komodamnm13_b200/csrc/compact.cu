@@ -11,10 +11,12 @@
 //
 // Passes: count (per 2048-word tile: run starts / run ends / elements, via the word masks
 //   start = w & ~((w << 1) | msb(prev)),  end = w & ~((w >> 1) | (lsb(next) << 31))),
-// scan (one block: tile offsets + header; clears L2), write (warp ballots + popc prefix sums;
-// coalesced gathers of the payload; clears L1 as it goes). HBM-bound: per dirty element
-// 1/8 B bitmap + esize read + esize written, + 16 B per run.
+// scan (one block: tile offsets + header; clears L2), write (persistent producer/consumer kernel:
+// bulk-copied bitmap words and values, block scans of word popcounts, coalesced payload stores;
+// clears L1 as it goes). HBM-bound: per dirty element 1/8 B bitmap + esize read + esize written,
+// + 16 B per run.
 #include "kernels.h"
+#include "tma_dev.cuh"
 #include "track.cuh"
 
 namespace accmg {
@@ -227,6 +229,250 @@ write_k(uint32_t* __restrict__ l1, int64_t nwords, const int64_t* __restrict__ t
     }
 }
 
+// Pass 3, default (impl 0): persistent, warp-specialised. Same output as write_k.
+// Measured: a one-tile-per-block kernel spends most of a tile's life in dependent global loads
+// (tile counts -> bitmap words -> offsets, ~5 us each under full HBM load) before any payload
+// moves, so it capped at ~4 TB/s whatever the ring depth. Here each block walks its tiles
+// t = blockIdx.x + k * gridDim.x with one producer warp running ahead of eight consumer warps:
+//  * producer (warp 8, one lane): reads the tile's counts / offsets / edge words into a
+//    double-buffered tile record, bulk-copies (cp.async.bulk) the tile's 8 KiB of bitmap words
+//    into that record and, for dense tiles, the values through an NST-stage ring of 8 KiB stages
+//    (mbarrier full/empty pairs), skipping clean tiles; it is up to two tiles ahead;
+//  * consumers (warps 0-7): per tile, clear the L1 words, scan the word popcounts (payload offset
+//    of each word inside the tile), write the run starts / ends, then store the dirty elements of
+//    each ring stage with coalesced stores (dense tiles) or gather them with kU predicated
+//    coalesced loads in flight per warp (sparse / ragged / unaligned tiles).
+constexpr int kU = 16;
+constexpr int kPad = 4;  // sw[kPad - 1] = previous tile's last word; sw[kPad + nw] = next tile's first
+constexpr uint32_t kStageBytes = 8192;
+constexpr int64_t kDenseElems = (int64_t)kTileWords * 32 / 2;
+constexpr int kConsumers = 256;  // warps 0-7; warp 8 is the producer
+
+__device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+                     dev::smem_u32(dst)),
+                 "l"(reinterpret_cast<uint64_t>(src)), "r"(bytes), "r"(dev::smem_u32(bar))
+                 : "memory");
+}
+__device__ __forceinline__ void consumers_sync() { asm volatile("bar.sync 1, %0;" ::"n"(kConsumers) : "memory"); }
+
+struct TileRec {  // one dirty tile, written by the producer before it arrives on the record's full barrier
+    int64_t t, off_s, off_e, off_el;
+    uint32_t edge_prev, edge_next;
+    int nw, dense;  // t < 0: end of this block's tiles
+};
+
+template <typename T, int NST>
+__global__ void __launch_bounds__(kConsumers + 32)
+write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const int64_t* __restrict__ tile_counts,
+             const int64_t* __restrict__ tile_offs, const uint32_t* __restrict__ tile_edges, int64_t ntiles,
+             const T* __restrict__ values, uint8_t* __restrict__ packed, int64_t n_runs, int aligned) {
+    constexpr int SCW = kStageBytes / (32 * sizeof(T));  // words per stage
+    constexpr int NSC = kTileWords / SCW;                 // stages per tile
+    extern __shared__ __align__(128) unsigned char ring[];  // NST x kStageBytes
+    __shared__ __align__(16) uint32_t sw[2][kTileWords + 2 * kPad];
+    __shared__ int32_t spre[kTileWords];
+    __shared__ int32_t wred[3][kConsumers / 32];
+    __shared__ TileRec rec[2];
+    __shared__ __align__(8) uint64_t full[NST], empty[NST], rfull[2], rempty[2];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    if (tid == 0) {
+        for (int q = 0; q < NST; ++q) { dev::mbar_init(&full[q], 1); dev::mbar_init(&empty[q], kConsumers / 32); }
+        for (int q = 0; q < 2; ++q) { dev::mbar_init(&rfull[q], 1); dev::mbar_init(&rempty[q], kConsumers / 32); }
+        dev::mbar_fence_init();
+    }
+    __syncthreads();
+
+    if (warp == kConsumers / 32) {  // ---------------- producer ----------------
+        if (lane != 0) return;
+        uint32_t seq = 0, kk = 0;
+        for (int64_t t = blockIdx.x;; t += gridDim.x) {
+            const bool end = t >= ntiles;
+            const int64_t el = end ? 0 : tile_counts[3 * t + 2];
+            if (!end && el == 0) continue;  // clean tile: nothing to pack
+            const int b = kk & 1;
+            dev::mbar_wait(&rempty[b], ((kk >> 1) & 1) ^ 1);  // consumers released this record
+            TileRec& r = rec[b];
+            if (end) {
+                r.t = -1;
+                dev::mbar_arrive(&rfull[b]);
+                return;
+            }
+            const int64_t w0 = t * kTileWords;
+            const int nw = (int)((w0 + kTileWords < nwords ? w0 + kTileWords : nwords) - w0);
+            const bool dense = aligned && el >= kDenseElems && nw == kTileWords && (w0 + kTileWords) * 32 <= extent;
+            r.t = t;
+            r.off_s = tile_offs[3 * t];
+            r.off_e = tile_offs[3 * t + 1];
+            r.off_el = tile_offs[3 * t + 2];
+            r.edge_prev = t > 0 ? tile_edges[2 * (t - 1) + 1] : 0u;
+            r.edge_next = t + 1 < ntiles ? tile_edges[2 * (t + 1)] : 0u;
+            r.nw = nw;
+            r.dense = dense;
+            if (nw == kTileWords) {  // the words are 16-byte aligned (w0 * 4 is a multiple of 8 KiB)
+                dev::mbar_expect_tx(&rfull[b], kTileWords * 4);
+                bulk_load(&sw[b][kPad], l1 + w0, kTileWords * 4, &rfull[b]);
+            } else {
+                dev::mbar_arrive(&rfull[b]);  // ragged last tile: the consumers load its words
+            }
+            ++kk;
+            if (!dense) continue;
+            for (int q = 0; q < NSC; ++q, ++seq) {
+                const int st = seq % NST;
+                dev::mbar_wait(&empty[st], ((seq / NST) & 1) ^ 1);
+                dev::mbar_expect_tx(&full[st], kStageBytes);
+                bulk_load(ring + st * kStageBytes, values + (w0 + (int64_t)q * SCW) * 32, kStageBytes, &full[st]);
+            }
+        }
+    }
+
+    // ---------------- consumers ----------------
+    int64_t* run_start = reinterpret_cast<int64_t*>(packed + 16);
+    int64_t* run_end = run_start + n_runs;
+    T* payload = reinterpret_cast<T*>(packed + 16 + 16 * n_runs);
+    const uint32_t lt = (1u << lane) - 1u;
+    uint32_t seq = 0;
+    for (uint32_t kk = 0;; ++kk) {
+        const int b = kk & 1;
+        dev::mbar_wait(&rfull[b], (kk >> 1) & 1);
+        const TileRec r = rec[b];
+        if (r.t < 0) break;
+        uint32_t* W = sw[b];
+        const int64_t w0 = r.t * kTileWords;
+        const int nw = r.nw;
+        if (nw == kTileWords) {
+            uint4* g = reinterpret_cast<uint4*>(l1 + w0);
+            for (int i = tid; i < kTileWords / 4; i += kConsumers) g[i] = make_uint4(0u, 0u, 0u, 0u);
+        } else {
+            for (int i = tid; i < nw; i += kConsumers) {
+                W[kPad + i] = l1[w0 + i];
+                l1[w0 + i] = 0u;
+            }
+        }
+        if (tid == 0) {
+            W[kPad - 1] = r.edge_prev;
+            W[kPad + nw] = r.edge_next;
+        }
+        consumers_sync();
+        // thread tid owns words [8 tid, 8 tid + 8): counts, then a block exclusive scan
+        const int i0 = tid * kWordsPerThread;
+        int cel = 0, cs = 0, ce = 0;
+#pragma unroll
+        for (int j = 0; j < kWordsPerThread; ++j) {
+            const int i = i0 + j;
+            if (i < nw) {
+                const uint32_t w = W[kPad + i];
+                cel += __popc(w);
+                cs += __popc(start_mask(w, W[kPad + i - 1]));
+                ce += __popc(end_mask(w, W[kPad + i + 1]));
+            }
+        }
+        const int iel = warp_incl_scan(cel), is = warp_incl_scan(cs), ie = warp_incl_scan(ce);
+        if (lane == 31) { wred[0][warp] = iel; wred[1][warp] = is; wred[2][warp] = ie; }
+        consumers_sync();
+        int oel = iel - cel, os = is - cs, oe = ie - ce;
+        for (int i = 0; i < warp; ++i) { oel += wred[0][i]; os += wred[1][i]; oe += wred[2][i]; }
+        {
+            int64_t ks = r.off_s + os, ke = r.off_e + oe;
+            int run = oel;
+#pragma unroll
+            for (int j = 0; j < kWordsPerThread; ++j) {
+                const int i = i0 + j;
+                if (i < nw) {
+                    const uint32_t w = W[kPad + i];
+                    spre[i] = run;
+                    run += __popc(w);
+                    const int64_t gw = w0 + i;
+                    for (uint32_t m = start_mask(w, W[kPad + i - 1]); m; m &= m - 1) run_start[ks++] = gw * 32 + (__ffs(m) - 1);
+                    for (uint32_t m = end_mask(w, W[kPad + i + 1]); m; m &= m - 1) run_end[ke++] = gw * 32 + __ffs(m);
+                }
+            }
+        }
+        consumers_sync();
+        T* tile_payload = payload + r.off_el;
+        if (r.dense) {
+            for (int q = 0; q < NSC; ++q, ++seq) {
+                const int st = seq % NST;
+                dev::mbar_wait(&full[st], (seq / NST) & 1);
+                const T* V = reinterpret_cast<const T*>(ring + st * kStageBytes);
+#pragma unroll
+                for (int j = warp; j < SCW; j += kConsumers / 32) {
+                    const int i = q * SCW + j;
+                    const uint32_t m = W[kPad + i];
+                    if ((m >> lane) & 1u) tile_payload[spre[i] + __popc(m & lt)] = V[j * 32 + lane];
+                }
+                __syncwarp();
+                if (lane == 0) dev::mbar_arrive(&empty[st]);
+            }
+        } else {
+            const T* vt = values + w0 * 32 + lane;
+            for (int base = warp * kU; base < nw; base += (kConsumers / 32) * kU) {
+                uint32_t m[kU];
+                T v[kU];
+#pragma unroll
+                for (int u = 0; u < kU; ++u) {
+                    m[u] = base + u < nw ? W[kPad + base + u] : 0u;
+                    v[u] = ((m[u] >> lane) & 1u) ? vt[(int64_t)(base + u) * 32] : T(0);
+                }
+#pragma unroll
+                for (int u = 0; u < kU; ++u)
+                    if ((m[u] >> lane) & 1u) tile_payload[spre[base + u] + __popc(m[u] & lt)] = v[u];
+            }
+        }
+        consumers_sync();  // spre / wred / this record are free again
+        if (lane == 0) dev::mbar_arrive(&rempty[b]);
+    }
+}
+
+template <typename T, int NST>
+cudaError_t launch_write_pipe_st(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
+                                 const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
+                                 uint8_t* packed, int64_t n_runs, cudaStream_t s) {
+    auto kern = write_pipe_k<T, NST>;
+    const size_t smem = (size_t)NST * kStageBytes;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    static int flat = -1;  // ACCMG_COMPACT_IMPL=2: gather path only (measurement)
+    if (flat < 0) {
+        const char* v = getenv("ACCMG_COMPACT_IMPL");
+        flat = (v && atoi(v) == 2) ? 1 : 0;
+    }
+    const int aligned = !flat && (reinterpret_cast<uintptr_t>(values) % 16) == 0;
+    int dev = 0, sms = 148, per_sm = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kConsumers + 32, smem);
+    int64_t grid = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
+    if (grid > ntiles) grid = ntiles;
+    kern<<<(unsigned)grid, kConsumers + 32, smem, s>>>(l1, nwords, extent, tile_counts, tile_offs, tile_edges, ntiles,
+                                                        static_cast<const T*>(values), packed, n_runs, aligned);
+    return cudaGetLastError();
+}
+
+// Ring depth: ACCMG_COMPACT_STAGES. Measured (C5, P = 2 and 8, profiles/r01/compact_pipe.log):
+// more blocks per SM beat deeper rings -- 3 stages (4 blocks/SM) 1.59 ms per loop, 6: 1.71,
+// 10: 1.71, 24 (1 block/SM): 2.09; the one-tile-per-block kernel was 2.37 and write_k 2.21.
+template <typename T>
+cudaError_t launch_write_stream(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
+                                const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
+                                uint8_t* packed, int64_t n_runs, cudaStream_t s) {
+    static int st = -1;
+    if (st < 0) {
+        const char* v = getenv("ACCMG_COMPACT_STAGES");
+        st = v ? atoi(v) : 3;
+    }
+    switch (st) {
+        case 2: return launch_write_pipe_st<T, 2>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s);
+        case 6: return launch_write_pipe_st<T, 6>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s);
+        case 8: return launch_write_pipe_st<T, 8>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s);
+        case 4: return launch_write_pipe_st<T, 4>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s);
+        case 10: return launch_write_pipe_st<T, 10>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s);
+        case 16: return launch_write_pipe_st<T, 16>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s);
+        case 24: return launch_write_pipe_st<T, 24>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s);
+        default: return launch_write_pipe_st<T, 3>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s);
+    }
+}
+
 // ---- scatter of packed runs ----------------------------------------------------------------------
 __device__ __forceinline__ void seg(int64_t n, int b, int64_t& lo, int64_t& hi) {
     lo = n * b / kScatterBlocks;
@@ -383,10 +629,27 @@ cudaError_t compact_scan(const int64_t* tile_counts, int64_t ntiles, int64_t* ti
     return cudaGetLastError();
 }
 
-cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t ntiles, const int64_t* tile_counts,
+cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
                           const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
                           int esize, uint8_t* packed, int64_t n_runs, cudaStream_t s, int64_t* launches) {
     dim3 g((unsigned)ntiles);
+    static int impl = -1;  // ACCMG_COMPACT_IMPL: 0 = write_stream_k (default), 1 = write_k (ballot groups)
+    if (impl < 0) {
+        const char* v = getenv("ACCMG_COMPACT_IMPL");
+        impl = v ? atoi(v) : 0;
+    }
+    if (impl != 1) {
+        cudaError_t e;
+        switch (esize) {
+            case 1: e = launch_write_stream<uint8_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s); break;
+            case 2: e = launch_write_stream<uint16_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s); break;
+            case 4: e = launch_write_stream<uint32_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s); break;
+            case 8: e = launch_write_stream<uint64_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, s); break;
+            default: return cudaErrorInvalidValue;
+        }
+        if (launches) *launches += 1;
+        return e;
+    }
     switch (esize) {
         case 1: write_k<uint8_t><<<g, kThreads, 0, s>>>(l1, nwords, tile_counts, tile_offs, tile_edges, ntiles, (const uint8_t*)values, packed, n_runs); break;
         case 2: write_k<uint16_t><<<g, kThreads, 0, s>>>(l1, nwords, tile_counts, tile_offs, tile_edges, ntiles, (const uint16_t*)values, packed, n_runs); break;

@@ -152,6 +152,21 @@ sparse_rows_kernel(const float* __restrict__ in, float* __restrict__ out, int64_
     }
 }
 
+template <bool TRACK>
+__global__ void __launch_bounds__(256)
+masked_write_kernel(const float* __restrict__ in, const uint8_t* __restrict__ mask, float* __restrict__ out, int64_t e0,
+                    int64_t e1, Track t) {
+    const int lane = threadIdx.x & 31;
+    int64_t l2c = -1;
+    for (int64_t base = e0 + ((int64_t)blockIdx.x * 256 + threadIdx.x - lane); base < e1;
+         base += (int64_t)gridDim.x * 256) {
+        const int64_t e = base + lane;
+        const bool w = e < e1 && mask[e] != 0;
+        if (w) out[e] = __fadd_rn(in[e], 1.0f);
+        if constexpr (TRACK) dev::track_warp<1>(t.l1, t.l2, t.l2_shift, base, w ? 1u : 0u, l2c);
+    }
+}
+
 }  // namespace
 
 cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
@@ -206,6 +221,17 @@ cudaError_t sparse_rows(const float* in, float* out, int64_t rows, int64_t cols,
     dim3 grid((unsigned)((cols + 255) / 256), (unsigned)(nsel < 65535 ? nsel : 65535));
     if (t.l1) sparse_rows_kernel<true><<<grid, 256, 0, s>>>(in, out, cols, first, r1, period, t);
     else sparse_rows_kernel<false><<<grid, 256, 0, s>>>(in, out, cols, first, r1, period, t);
+    if (launches) *launches += 1;
+    return cudaGetLastError();
+}
+
+cudaError_t masked_write(const float* in, const uint8_t* mask, float* out, int64_t e0, int64_t e1, Track t,
+                         cudaStream_t s, int64_t* launches) {
+    if (e1 <= e0) return cudaSuccess;
+    int64_t nb = (e1 - e0 + 255) / 256;
+    if (nb > 148 * 8) nb = 148 * 8;
+    if (t.l1) masked_write_kernel<true><<<(unsigned)nb, 256, 0, s>>>(in, mask, out, e0, e1, t);
+    else masked_write_kernel<false><<<(unsigned)nb, 256, 0, s>>>(in, mask, out, e0, e1, t);
     if (launches) *launches += 1;
     return cudaGetLastError();
 }

@@ -63,6 +63,9 @@ cudaError_t frame_copy(const float* src, float* tmp, int64_t cols, int64_t lo, i
 // Test body: rows i in [r0, r1) with i % period == 0: out[i][:] = in[i][:] + 1.0f.
 cudaError_t sparse_rows(const float* in, float* out, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
                         int64_t period, Track t, cudaStream_t s, int64_t* launches);
+// Test body: e in [e0, e1) with mask[e] != 0: out[e] = in[e] + 1.0f (warp-aggregated tracking).
+cudaError_t masked_write(const float* in, const uint8_t* mask, float* out, int64_t e0, int64_t e1, Track t,
+                         cudaStream_t s, int64_t* launches);
 
 // k-means assignment + reductiontoarray over points [p0, p1): member[p] = argmin_c (fmaf chain),
 // sums[member][j] += x*2^shift (int64), counts[member] += 1 into the partition's partials.
@@ -103,7 +106,8 @@ cudaError_t compact_count(const uint32_t* l1, const uint32_t* l2, int64_t nwords
 cudaError_t compact_scan(const int64_t* tile_counts, int64_t ntiles, int64_t* tile_offs, int64_t* totals,
                          uint32_t* l2, int64_t nl2words, cudaStream_t s, int64_t* launches);
 // Pass 3: run starts/ends and payload into the canonical packed buffer; clears L1 words.
-cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t ntiles, const int64_t* tile_counts,
+// values holds elements [0, extent) (global indices).
+cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
                           const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
                           int esize, uint8_t* packed, int64_t n_runs, cudaStream_t s, int64_t* launches);
 // Scatter the runs of a canonical packed buffer into ndst replicas at the same global indices.

@@ -572,6 +572,9 @@ bool body_spec(int id, BodySpec* b) {
             *b = {3, {ACCMG_RW, ACCMG_RW, ACCMG_W}, {8, 8, 4}, 1, sizeof(accmg_args_kmeans)};
             return true;
         case ACCMG_BODY_TEST_SPARSE_WRITE: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 1, sizeof(accmg_args_sparse)}; return true;
+        case ACCMG_BODY_TEST_MASKED_WRITE:
+            *b = {3, {ACCMG_R, ACCMG_R, ACCMG_W}, {4, 1, 4}, 1, sizeof(accmg_args_masked)};
+            return true;
         case ACCMG_BODY_SCATTER: *b = {3, {ACCMG_R, ACCMG_R, ACCMG_W}, {4, 4, 4}, 1, sizeof(accmg_args_scatter)}; return true;
         case ACCMG_BODY_JACOBI3D_7PT: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 3, sizeof(accmg_args_jacobi3d)}; return true;
         case ACCMG_BODY_JACOBI2D_DEEP: *b = {2, {ACCMG_R, ACCMG_W}, {4, 4}, 2, sizeof(accmg_args_jacobi2d_deep)}; return true;
@@ -607,6 +610,14 @@ int validate_body(const accmg_bounds* bd, int body, const accmg_access* d, const
             if (ext(0) != a->rows * a->cols || ext(1) != a->rows * a->cols) return bad("sparse: extent != rows*cols");
             if (bd->lo[0] < 0 || bd->hi[0] > a->rows) return bad("sparse: bounds outside [0,rows)");
             if (d[0].region == d[1].region) return bad("sparse: in and out must differ");
+            return 0;
+        }
+        case ACCMG_BODY_TEST_MASKED_WRITE: {
+            auto a = static_cast<const accmg_args_masked*>(args);
+            if (a->n < 1) return bad("masked: n >= 1");
+            if (ext(0) != a->n || ext(1) != a->n || ext(2) != a->n) return bad("masked: extents != n");
+            if (bd->lo[0] < 0 || bd->hi[0] > a->n) return bad("masked: bounds outside [0,n)");
+            if (d[0].region == d[2].region) return bad("masked: in and out must differ");
             return 0;
         }
         case ACCMG_BODY_JACOBI3D_7PT: {
@@ -716,6 +727,9 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
             e = k::sparse_rows((const float*)P(0), (float*)P(1), x->rows, x->cols, a, b, x->period, T(1), S.stream, L);
             break;
         }
+        case ACCMG_BODY_TEST_MASKED_WRITE:
+            e = k::masked_write((const float*)P(0), (const uint8_t*)P(1), (float*)P(2), a, b, T(2), S.stream, L);
+            break;
         case ACCMG_BODY_JACOBI3D_7PT: {
             auto x = static_cast<const accmg_args_jacobi3d*>(args);
             const Ival al = d[0].region->arange[g];
@@ -817,7 +831,7 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
             TRY(ensure_packed(t, t.packed_bytes));
             CUDA_TRY(cudaMemcpyAsync(t.packed, t.totals, 16, cudaMemcpyDeviceToDevice, S.stream));
             ProfScope ps(1);
-            CUDA_TRY(k::compact_write(t.l1, t.nwords, t.ntiles, t.tile_counts, t.tile_offs, t.tile_edges, r->dev[li],
+            CUDA_TRY(k::compact_write(t.l1, t.nwords, r->extent, t.ntiles, t.tile_counts, t.tile_offs, t.tile_edges, r->dev[li],
                                       (int)r->esize, t.packed, t.n_runs, S.stream, &S.st.kernel_launches));
             t.has_packed = true;
         }

@@ -109,6 +109,30 @@ def test_sparse_rows_body():
     assert np.array_equal(bits.any(axis=1), np.arange(N) % 7 == 0)
 
 
+@pytest.mark.parametrize("P", [1, 3])
+def test_masked_write_body_brute_force(P):
+    n = 1000
+    src = gen.u_fill(9, 0, n).astype(np.float32)
+    mask = gen.write_mask(10, n, 0.4, 3)
+    dst = np.full(n, -5.0, dtype=np.float32)
+    bms = oracle.masked_write(src, mask, dst, P=P, track=True)
+    bounds = [((g * n) // P, ((g + 1) * n) // P) for g in range(P)]   # L108 chunks, by hand
+    for e in range(n):
+        exp = float(np.float32(src[e]) + np.float32(1.0)) if mask[e] else -5.0
+        assert float(dst[e]) == exp
+        for g, (a, b) in enumerate(bounds):
+            bit = (int(bms[g][e // 32]) >> (e % 32)) & 1
+            assert bit == (1 if (mask[e] and a <= e < b) else 0)
+
+
+def test_write_mask_recipe():
+    m = gen.write_mask(3, 1000, 0.5, 7)
+    assert m.size == 1000 and set(np.unique(m)) <= {0, 1}
+    assert all(len(set(m[s:s + 7])) == 1 for s in range(0, 1000, 7))   # constant on segments
+    assert 0.3 < m.mean() < 0.7
+    assert gen.write_mask(3, 100, 1.0).all() and not gen.write_mask(3, 100, 0.0).any()
+
+
 # ---- GEMM -------------------------------------------------------------------------------------
 def _bf16(x):
     return (np.asarray(x, dtype=np.float32).view(np.uint32) >> 16).astype(np.uint16)
