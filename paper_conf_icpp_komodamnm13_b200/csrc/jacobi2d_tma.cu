@@ -6,8 +6,10 @@
 // completing on mbarriers; 8 warps compute 4 rows x 4 columns per lane from shared memory
 // (horizontal neighbours by shuffle) and store 128-bit vectors of interior points. The halo rows
 // of a tile are the previous / next tile's edge rows, so their second read hits L2.
-// Kept beside the register-marching kernel (impl = 1, the default) to compare the two designs on
-// the same shapes: see profiles/ and DESIGN.md.
+// The default body (measured faster than the register-marching kernel, impl = 1: profiles/ and
+// DESIGN.md). Write tracking (undeclared dst) runs once per CTA after its stores: mark_rect sets
+// the words of its 256-row x 128-column rectangle (plain stores for owned words, atomicOr on words
+// shared with the neighbouring strips) and the rows' chunk bits.
 #include "kernels.h"
 #include "tma_dev.cuh"
 #include "tma_host.h"
@@ -58,8 +60,6 @@ jacobi2d_tma_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst,
     for (int c = 0; c < 4; ++c) nib |= (k + c >= c0 && k + c < c1) ? (1u << c) : 0u;
     const bool full = nib == 0xFu;
     const int col = 4 + 4 * lane;
-    dev::WarpTracker<4> trk;
-    if constexpr (TRACK) trk.init(nib);
     for (int m = 0; m < ntiles; ++m) {
         const int st = m % kStages;
         dev::mbar_wait(&bar[st], (uint32_t)((m / kStages) & 1));
@@ -90,7 +90,6 @@ jacobi2d_tma_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst,
                     for (int c = 0; c < 4; ++c)
                         if (nib & (1u << c)) out[c] = o[c];
                 }
-                if constexpr (TRACK) trk.mark(t.l1, t.l2, t.l2_shift, row * cols + k0);
             }
         }
         __syncthreads();  // every thread is done with stage st
@@ -101,6 +100,10 @@ jacobi2d_tma_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst,
             dev::tma_load_2d(&map, &bar[st], tiles + st * kStageFloats, (int)(k0 - 4),
                              (int)(rs + RB * mn - 1 - row_lo));
         }
+    }
+    if constexpr (TRACK) {  // dirty bits of the CTA's rectangle, once, after its stores
+        const int64_t re = rs + (int64_t)RB * kTiles < r1 ? rs + (int64_t)RB * kTiles : r1;
+        dev::mark_rect(t.l1, t.l2, t.l2_shift, rs, re, cols, k0 > c0 ? k0 : c0, k0 + TK < c1 ? k0 + TK : c1, tid, 256);
     }
 }
 
