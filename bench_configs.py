@@ -311,6 +311,8 @@ def main():
                     emit(gemm_cfg(a.gemm_n, P, a.gemm_reps, a.check))
                 elif cfg == "f2":
                     emit(jacobi3d_cfg(1024, 20, P))
+                elif cfg == "f2u":  # 3-D stencil without declarations: tracked body + compaction + propagation
+                    emit(jacobi3d_cfg(1024, 6, P, declared=False))
                 elif cfg == "f2deep":
                     for h in (1, 2, 4, 8):
                         emit(deep_cfg(32768, 48, P, h))

@@ -126,9 +126,8 @@ __device__ __forceinline__ V4 jstep2(const V4& N, const V4& C, const V4& S, int 
 }
 
 // One input row (local index i, i % 3 == PH) through all H levels.
-template <int H, int PH, bool MASK, bool TRACK>
-__device__ __forceinline__ void advance(V4 (&Lv)[H][3], const V4& X, int i, const Item& it,
-                                        dev::WarpTracker<4>& trk, const Track& t) {
+template <int H, int PH, bool MASK>
+__device__ __forceinline__ void advance(V4 (&Lv)[H][3], const V4& X, int i, const Item& it) {
     Lv[0][PH] = X;
 #pragma unroll
     for (int l = 1; l <= H; ++l) {
@@ -151,7 +150,6 @@ __device__ __forceinline__ void advance(V4 (&Lv)[H][3], const V4& X, int i, cons
                     if (it.onib & 4u) p[2] = f.z;
                     if (it.onib & 8u) p[3] = f.w;
                 }
-                if constexpr (TRACK) trk.mark(t.l1, t.l2, t.l2_shift, it.e0 + (int64_t)j * it.cols);
             }
         }
     }
@@ -166,8 +164,6 @@ __device__ __forceinline__ void run_item(const CUtensorMap* map, uint64_t* bar, 
     for (int l = 0; l < H; ++l)
 #pragma unroll
         for (int q = 0; q < 3; ++q) Lv[l][q] = V4{0ull, 0ull};
-    dev::WarpTracker<4> trk;
-    if constexpr (TRACK) trk.init(it.onib);
     // prologue: the first kStages stages of this item (all slots are free here)
     if (lane == 0) {
         for (int s = 0; s < kStages && s < nst; ++s) {
@@ -186,9 +182,9 @@ __device__ __forceinline__ void run_item(const CUtensorMap* map, uint64_t* bar, 
             const V4 X0 = from4(*reinterpret_cast<const float4*>(T + (rr + 0) * W));
             const V4 X1 = from4(*reinterpret_cast<const float4*>(T + (rr + 1) * W));
             const V4 X2 = from4(*reinterpret_cast<const float4*>(T + (rr + 2) * W));
-            advance<H, 0, MASK, TRACK>(Lv, X0, i0 + rr + 0, it, trk, t);
-            advance<H, 1, MASK, TRACK>(Lv, X1, i0 + rr + 1, it, trk, t);
-            advance<H, 2, MASK, TRACK>(Lv, X2, i0 + rr + 2, it, trk, t);
+            advance<H, 0, MASK>(Lv, X0, i0 + rr + 0, it);
+            advance<H, 1, MASK>(Lv, X1, i0 + rr + 1, it);
+            advance<H, 2, MASK>(Lv, X2, i0 + rr + 2, it);
         }
         __syncwarp();  // every lane has consumed the slot
         if (lane == 0 && s + kStages < nst) {
@@ -253,6 +249,9 @@ deep_stream_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, 
             run_item<H, false, TRACK>(&map, bar, ring, nst, g, kt, ybeg - row_lo, it, t);
         else
             run_item<H, true, TRACK>(&map, bar, ring, nst, g, kt, ybeg - row_lo, it, t);
+        if constexpr (TRACK)  // dirty bits of the item's output rectangle, after its stores
+            dev::mark_rect(t.l1, t.l2, t.l2_shift, y0, y0 + lc, cols, std::max<int64_t>(k0, c0),
+                           std::min<int64_t>(k0 + TK, c1), lane, 32);
     }
 }
 

@@ -12,7 +12,8 @@
 // element crosses HBM once (+ the 2 halo rows / 2 halo planes per segment, L2-resident). Threads
 // read the 7 operands from shared memory (horizontal neighbours by warp shuffle), use explicit
 // round-to-nearest adds in the stated order, and store 128-bit vectors of interior points. The
-// optional fused epilogue sets the two-level dirty bits (L133-135).
+// optional fused epilogue sets the two-level dirty bits (L133-135) once per CTA after its stores
+// (mark_rect over its planes: owned words by plain stores, words shared with neighbours by atomicOr).
 #include "kernels.h"
 #include "tma_dev.cuh"
 #include "tma_host.h"
@@ -66,8 +67,6 @@ jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, i
     for (int c = 0; c < 4; ++c) nib |= (k + c >= kl && k + c < kh) ? (1u << c) : 0u;
     const bool full = nib == 0xFu;
     const int col = 4 + 4 * lane;  // tile column of k
-    dev::WarpTracker<4> trk;
-    if constexpr (TRACK) trk.init(nib);
     dev::mbar_wait(&bar[0], 0);
     dev::mbar_wait(&bar[1], 0);
     for (int64_t i = ps; i < pe; ++i) {
@@ -104,7 +103,6 @@ jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, i
                     for (int c = 0; c < 4; ++c)
                         if (nib & (1u << c)) out[c] = o[c];
                 }
-                if constexpr (TRACK) trk.mark(t.l1, t.l2, t.l2_shift, (i * n1 + j) * n2 + k0);
             }
         }
         __syncthreads();  // every thread is done with plane i-1 (stage (q-2) % kStages)
@@ -115,6 +113,10 @@ jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, i
             dev::tma_load_3d(&map, &bar[qn % kStages], tile[qn % kStages], (int)(k0 - 4), (int)(j0 - 1),
                              (int)(ps - 1 + qn - plane_lo));
         }
+    }
+    if constexpr (TRACK) {  // dirty bits of the CTA's 16 x 128 column in each of its planes, after its stores
+        const int64_t je = j0 + TJ < jh ? j0 + TJ : jh, ka = k0 > kl ? k0 : kl, kb = k0 + TK < kh ? k0 + TK : kh;
+        dev::mark_rect(t.l1, t.l2, t.l2_shift, ps * n1 + j0, ps * n1 + je, n2, ka, kb, tid, 256, (int)(pe - ps), n1);
     }
 }
 

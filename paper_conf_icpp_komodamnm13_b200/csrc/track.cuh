@@ -188,20 +188,25 @@ struct WarpTracker {
 };
 
 // Block-level epilogue for a CTA that wrote every element of the rectangle rows [rs, re) x
-// columns [ca, cb) of a row-major array with `cols` columns (and nothing else in this loop): all
-// threads of the block (tid < nthr) call it once after their stores. Thread i handles (row, word)
-// pair i, so one warp-wide store covers 32 words of several rows instead of one mark per row and
-// warp. A word lying entirely inside one row's written range holds only this CTA's elements and was
-// cleared by the last compaction: plain store. Words shared with a neighbouring CTA: atomicOr. Each
-// row's chunk bits are set unless the previous row already set them (check-first atomics).
+// columns [ca, cb) of a row-major array with `cols` columns (and nothing else in this loop); with
+// nplanes > 1 the same rectangle repeated every `pstride` rows (a 3-D block: planes of a
+// [n0*n1][n2] view). All threads of the block (tid < nthr) call it once after their stores.
+// Thread i handles (row, word) pair i, so one warp-wide store covers 32 words of several rows
+// instead of one mark per row and warp. A word lying entirely inside one row's written range holds
+// only this CTA's elements and was cleared by the last compaction: plain store. Words shared with a
+// neighbouring CTA: atomicOr. Each row's chunk bits are set unless the previous row of the same
+// plane already set them (check-first atomics).
 __device__ __forceinline__ void mark_rect(uint32_t* __restrict__ l1, uint32_t* __restrict__ l2, int l2_shift, int64_t rs,
-                                          int64_t re, int64_t cols, int64_t ca, int64_t cb, int tid, int nthr) {
-    if (rs >= re || ca >= cb) return;
+                                          int64_t re, int64_t cols, int64_t ca, int64_t cb, int tid, int nthr,
+                                          int nplanes = 1, int64_t pstride = 0) {
+    if (rs >= re || ca >= cb || nplanes < 1) return;
+    const int nr = (int)(re - rs);
     const int nwr = (int)((cb - ca + 31) >> 5) + 1;  // words one row can touch
-    const int npairs = (int)(re - rs) * nwr;
+    const int npairs = nplanes * nr * nwr;
     for (int i = tid; i < npairs; i += nthr) {
-        const int dr = i / nwr, q = i - dr * nwr;
-        const int64_t e0 = (rs + dr) * cols + ca, e1 = e0 + (cb - ca);
+        const int row = i / nwr, q = i - row * nwr;
+        const int pl = row / nr, dr = row - pl * nr;
+        const int64_t e0 = (rs + pl * pstride + dr) * cols + ca, e1 = e0 + (cb - ca);
         const int64_t w = (e0 >> 5) + q;
         if (w * 32 >= e1) continue;
         const int64_t lo = e0 > w * 32 ? e0 : w * 32, hi = e1 < w * 32 + 32 ? e1 : w * 32 + 32;
@@ -210,11 +215,12 @@ __device__ __forceinline__ void mark_rect(uint32_t* __restrict__ l1, uint32_t* _
         if (n == 32) l1[w] = v;
         else atomicOr(l1 + w, v);
     }
-    for (int64_t r = rs + tid; r < re; r += nthr) {
-        const int64_t e0 = r * cols + ca;
+    for (int row = tid; row < nplanes * nr; row += nthr) {
+        const int pl = row / nr, dr = row - pl * nr;
+        const int64_t e0 = (rs + pl * pstride + dr) * cols + ca;
         int64_t c0 = e0 >> l2_shift;
         const int64_t c1 = (e0 + (cb - ca) - 1) >> l2_shift;
-        if (r > rs && c0 == ((e0 - cols + (cb - ca) - 1) >> l2_shift)) ++c0;  // previous row set it
+        if (dr > 0 && c0 == ((e0 - cols + (cb - ca) - 1) >> l2_shift)) ++c0;  // previous row set it
         for (int64_t c = c0; c <= c1; ++c) set_chunk_bit(l2, c);
     }
 }

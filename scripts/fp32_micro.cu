@@ -42,15 +42,17 @@ __global__ void k_fadd2(float* out, float a, float b) {
     out[blockIdx.x * blockDim.x + threadIdx.x] = s;
 }
 
-// the k-means inner step: d = x + (-c); acc = fma(d, d, acc), packed
+// the k-means inner step: d = x + (-c); acc = fma(d, d, acc), packed. The add's operand is the
+// running accumulator so the compiler cannot hoist it out of the loop (an earlier version added
+// two loop invariants, the FADD2 was hoisted and the pair was counted at twice its real rate).
 __global__ void k_pair(float* out, float a, float b) {
-    float2 acc[8], xv[8];
-    for (int i = 0; i < 8; ++i) { acc[i] = make_float2(0, 0); xv[i] = make_float2(threadIdx.x * 0.001f + i, i); }
-    const float2 nc = make_float2(-a, -b);
+    float2 acc[8];
+    for (int i = 0; i < 8; ++i) acc[i] = make_float2(threadIdx.x * 1e-9f, i * 1e-9f);
+    const float2 nc = make_float2(-a * 1e-6f, -b * 1e-6f);
     for (int it = 0; it < kIters; ++it)
 #pragma unroll
         for (int i = 0; i < 8; ++i) {
-            const float2 d = __fadd2_rn(xv[i], nc);
+            const float2 d = __fadd2_rn(acc[i], nc);
             acc[i] = __ffma2_rn(d, d, acc[i]);
         }
     float s = 0;
