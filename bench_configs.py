@@ -140,8 +140,10 @@ def kmeans_cfg(n, iters, P, check):
     out = {"config": "c4", "P": P, "n": n, "iters_timed": its, "iters_per_s": n * its / t,
            "ms_per_iteration": t / its * 1e3, **per_loop(st, 2 * its), "gen_s": tgen,
            "fp32_lane_ops_per_s": lane_ops / (ms_assign / 1e3)}
-    # FP32 peak at the clock: 148 SMs x 128 lanes x 2 ops (FFMA2 packs 2) per cycle
-    out["frac_of_fp32_fma_peak_1965MHz"] = out["fp32_lane_ops_per_s"] / (148 * 128 * 2 * 1.965e9)
+    # FP32 lane peak at the clock: 148 SMs x 128 lanes x 1.965 GHz = 3.72e13 lane-ops/s (FFMA2 packs
+    # two lanes into one instruction, not two ops into one lane; scripts/fp32_micro.cu measures
+    # 3.69e13 for the FADD2+FFMA2 pair the distance uses)
+    out["frac_of_fp32_lane_peak_1965MHz"] = out["fp32_lane_ops_per_s"] / (148 * 128 * 1.965e9)
     if check:
         ok = np.array_equal(member, lab)
         # closed form: centroids are the exact means of the generated clusters

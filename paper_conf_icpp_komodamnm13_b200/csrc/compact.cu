@@ -98,45 +98,47 @@ count_k(const uint32_t* __restrict__ l1, const uint32_t* __restrict__ l2, int64_
 }
 
 // One block: exclusive scan of the per-tile triples {starts, ends, elems}, 1024 tiles per step
-// (coalesced loads, warp-shuffle scans, one carry per step), then the L2 popcount + clear.
+// (coalesced loads of the next step issued before the current one is scanned; warp-shuffle scans;
+// double-buffered warp totals, so two barriers per step and every thread carries the running
+// totals in registers), then the L2 popcount + clear.
 __global__ void __launch_bounds__(1024)
 scan_k(const int64_t* __restrict__ tile_counts, int64_t ntiles, int64_t* __restrict__ tile_offs,
        int64_t* __restrict__ totals, uint32_t* __restrict__ l2, int64_t nl2words) {
-    __shared__ int64_t wsum[3][32];
-    __shared__ int64_t carry[3];
+    __shared__ int64_t wsum[2][3][32];
+    __shared__ int64_t wtot[2][3];
     __shared__ unsigned long long nchunks;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    if (tid < 3) carry[tid] = 0;
     if (tid == 0) nchunks = 0ull;
-    __syncthreads();
-    for (int64_t base = 0; base < ntiles; base += 1024) {
-        const int64_t t = base + tid;
+    int64_t carry[3] = {0, 0, 0}, vn[3];
+#pragma unroll
+    for (int q = 0; q < 3; ++q) vn[q] = tid < ntiles ? tile_counts[3 * tid + q] : 0;
+    int buf = 0;
+    for (int64_t base = 0; base < ntiles; base += 1024, buf ^= 1) {
+        const int64_t t = base + tid, tn = t + 1024;
         int64_t v[3], inc[3];
 #pragma unroll
         for (int q = 0; q < 3; ++q) {
-            v[q] = t < ntiles ? tile_counts[3 * t + q] : 0;
+            v[q] = vn[q];
+            vn[q] = tn < ntiles ? tile_counts[3 * tn + q] : 0;  // next step's loads in flight
             inc[q] = warp_incl_scan(v[q]);
-            if (lane == 31) wsum[q][warp] = inc[q];
+            if (lane == 31) wsum[buf][q][warp] = inc[q];
         }
         __syncthreads();
         if (warp == 0) {
 #pragma unroll
             for (int q = 0; q < 3; ++q) {
-                const int64_t x = wsum[q][lane];
+                const int64_t x = wsum[buf][q][lane];
                 const int64_t xi = warp_incl_scan(x);
-                wsum[q][lane] = xi - x;  // exclusive warp offsets
+                wsum[buf][q][lane] = xi - x;  // exclusive warp offsets
+                if (lane == 31) wtot[buf][q] = xi;
             }
         }
         __syncthreads();
 #pragma unroll
-        for (int q = 0; q < 3; ++q)
-            if (t < ntiles) tile_offs[3 * t + q] = carry[q] + wsum[q][warp] + inc[q] - v[q];
-        __syncthreads();
-        if (tid == 1023) {
-#pragma unroll
-            for (int q = 0; q < 3; ++q) carry[q] += wsum[q][31] + inc[q];
+        for (int q = 0; q < 3; ++q) {
+            if (t < ntiles) tile_offs[3 * t + q] = carry[q] + wsum[buf][q][warp] + inc[q] - v[q];
+            carry[q] += wtot[buf][q];
         }
-        __syncthreads();
     }
     unsigned long long pc = 0;
     for (int64_t w = tid; w < nl2words; w += 1024) { pc += __popc(l2[w]); l2[w] = 0u; }

@@ -316,9 +316,19 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
             case 6: e = cu2 ? launch_assign16<2, 2, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
                             : launch_assign16<2, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
             case 7: e = launch_assign16<1, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            // default: measured fastest on B200 (profiles/r01/kmeans_variants.txt)
-            default: e = cu2 ? launch_assign16<2, 2, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                             : launch_assign16<2, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 8: e = launch_assign16<2, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 9: e = cu2 ? launch_assign16<2, 2, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                            : launch_assign16<2, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 10: e = cu2 ? launch_assign16<1, 2, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                             : launch_assign16<1, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 11: e = (kc % 4 == 0) ? launch_assign16<1, 4, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                                       : launch_assign16<1, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 12: e = cu2 ? launch_assign16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                             : launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            // default: measured fastest on B200 (profiles/r01/kmeans_variants.txt): 2 point pairs and
+            // 2 centroids per thread, 256 threads, 2 blocks/SM (16 warps/SM, 125 registers)
+            default: e = cu2 ? launch_assign16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                             : launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
         }
         if (e != cudaSuccess) return e;
     } else {
