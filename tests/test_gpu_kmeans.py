@@ -73,3 +73,17 @@ def test_off_grid_input_is_reported():
         with pytest.raises(A.AccmgError) as e:
             WL.kmeans_run(x, 8, 1)
         assert e.value.code == A.EDATA
+
+
+@pytest.mark.parametrize("k", [37, 600])
+def test_d16_odd_k_and_k_beyond_constant_memory(k):
+    """d = 16 fast paths: odd k (one centroid per step) and k > 512 (centroids no longer fit the
+    constant-memory kernel: the shared-memory kernel runs), with duplicated points (ties)."""
+    from paper_conf_icpp_komodamnm13_b200 import workloads as WL
+    n = 40000
+    x = gen.kmeans_points(6, n, 16, k, gen.KM_OVERLAP)
+    x[1] = x[0]                                   # duplicate initial centroid -> ties, an empty cluster
+    ocen, omem = oracle.kmeans_run(x, k, 3)
+    with runtime(num_partitions=2):
+        cen, mem = WL.kmeans_run(x, k, 3)
+    assert np.array_equal(mem, omem) and np.array_equal(cen, ocen)
