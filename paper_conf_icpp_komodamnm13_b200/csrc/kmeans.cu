@@ -182,6 +182,124 @@ assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __
     flush_block(s_sum, s_cnt, sums, counts, kc, D);
 }
 
+// Centroids in constant memory (default for d = 16, k <= kConstCen): the loop over c is
+// warp-uniform, so the compiler reads each centroid value with a uniform-datapath LDCU into a
+// uniform register and FADD2 takes it as a broadcast scalar operand with a free negation
+// (`FADD2 R, R.F32x2, -UR.F32`: x + (-c) == x - c exactly). No shared-memory loads on the vector
+// pipes and no centroid copies in vector registers (108 instead of 125 registers at 2 blocks/SM).
+// The loop over this thread's point groups takes its trip count from block-uniform values only:
+// with a per-thread grid-stride condition the compiler cannot prove the centroid loop convergent
+// and falls back to vector LDC loads (measured: 8 % slower).
+constexpr int kConstCen = 512;
+__constant__ float c_cen[kConstCen * 16];
+
+template <int NP, int CU, int NT, int MINB>
+__global__ void __launch_bounds__(NT, MINB)
+assign_c16(const float* __restrict__ x, int32_t* __restrict__ member, int64_t* __restrict__ sums,
+           int64_t* __restrict__ counts, int64_t p0, int64_t p1, int kc, int shift, int* err) {
+    constexpr int D = 16;
+    extern __shared__ __align__(16) unsigned char smem[];
+    unsigned long long* s_sum = reinterpret_cast<unsigned long long*>(smem);  // kc*D
+    unsigned long long* s_cnt = s_sum + kc * D;                             // kc
+    for (int i = threadIdx.x; i < kc * D; i += NT) s_sum[i] = 0ull;
+    for (int i = threadIdx.x; i < kc; i += NT) s_cnt[i] = 0ull;
+    __syncthreads();
+    constexpr int PPT = 2 * NP;
+    const float scale = (float)(1 << shift);
+    const int64_t n = p1 - p0;
+    const int64_t ngroups = (n + PPT - 1) / PPT;
+    // trip count from block-uniform values only, so the centroid loop below runs under uniform
+    // control flow (the condition for the uniform-datapath LDCU of c_cen); lanes past the end
+    // compute on zeros and store nothing
+    const int64_t first = (int64_t)blockIdx.x * NT, stride = (int64_t)gridDim.x * NT;
+    const int64_t trips = first < ngroups ? (ngroups - first + stride - 1) / stride : 0;
+    for (int64_t it = 0; it < trips; ++it) {
+        const int64_t grp = first + it * stride + threadIdx.x;
+        const int64_t pb = p0 + grp * PPT;
+        uint64_t xp[NP][D];  // pair h = (x[pb+2h][j], x[pb+2h+1][j])
+#pragma unroll
+        for (int h = 0; h < NP; ++h) {
+            const bool ok0 = pb + 2 * h < p1, ok1 = pb + 2 * h + 1 < p1;
+#pragma unroll
+            for (int j = 0; j < D; j += 4) {
+                const float4 a = ok0 ? __ldg(reinterpret_cast<const float4*>(x + (pb + 2 * h) * D + j))
+                                     : make_float4(0.f, 0.f, 0.f, 0.f);
+                const float4 b = ok1 ? __ldg(reinterpret_cast<const float4*>(x + (pb + 2 * h + 1) * D + j))
+                                     : make_float4(0.f, 0.f, 0.f, 0.f);
+                xp[h][j] = pk2m(a.x, b.x);
+                xp[h][j + 1] = pk2m(a.y, b.y);
+                xp[h][j + 2] = pk2m(a.z, b.z);
+                xp[h][j + 3] = pk2m(a.w, b.w);
+            }
+        }
+        float bd[PPT];
+        int bi[PPT];
+#pragma unroll
+        for (int q = 0; q < PPT; ++q) { bd[q] = __int_as_float(0x7f800000); bi[q] = 0; }
+#pragma unroll 1
+        for (int c = 0; c < kc; c += CU) {
+            uint64_t acc[CU][NP];
+#pragma unroll
+            for (int u = 0; u < CU; ++u)
+#pragma unroll
+                for (int h = 0; h < NP; ++h) acc[u][h] = 0ull;
+#pragma unroll
+            for (int j = 0; j < D; ++j) {
+#pragma unroll
+                for (int u = 0; u < CU; ++u) {
+                    const float nj = -c_cen[(c + u) * D + j];
+                    const uint64_t n2 = pk2(nj, nj);
+#pragma unroll
+                    for (int h = 0; h < NP; ++h) acc[u][h] = fma2sq(add2(xp[h][j], n2), acc[u][h]);
+                }
+            }
+            // centroids in ascending order: strict < keeps the lowest index on ties
+#pragma unroll
+            for (int u = 0; u < CU; ++u)
+#pragma unroll
+                for (int h = 0; h < NP; ++h) {
+                    float d0, d1;
+                    upk2(acc[u][h], d0, d1);
+                    if (d0 < bd[2 * h]) { bd[2 * h] = d0; bi[2 * h] = c + u; }
+                    if (d1 < bd[2 * h + 1]) { bd[2 * h + 1] = d1; bi[2 * h + 1] = c + u; }
+                }
+        }
+#pragma unroll
+        for (int q = 0; q < PPT; ++q) {
+            if (pb + q >= p1) continue;
+            member[pb + q] = bi[q];
+            atomicAdd(s_cnt + bi[q], 1ull);
+#pragma unroll
+            for (int j = 0; j < D; ++j) {
+                float xa, xb;
+                upk2(xp[q / 2][j], xa, xb);
+                const float xv = (q & 1) ? xb : xa;
+                atomicAdd(s_sum + bi[q] * D + j, (unsigned long long)fixed_of(xv, scale, err));
+            }
+        }
+    }
+    flush_block(s_sum, s_cnt, sums, counts, kc, D);
+}
+
+template <int NP, int CU, int NT, int MINB>
+cudaError_t launch_assign_c16(const float* x, const float* cen, int32_t* member, int64_t* sums, int64_t* counts,
+                              int64_t p0, int64_t p1, int kc, int shift, int* err, cudaStream_t s, int sms) {
+    auto kern = assign_c16<NP, CU, NT, MINB>;
+    cudaError_t e = cudaMemcpyToSymbolAsync(c_cen, cen, (size_t)kc * 16 * sizeof(float), 0, cudaMemcpyDeviceToDevice, s);
+    if (e != cudaSuccess) return e;
+    const size_t smem = (size_t)kc * 16 * 8 + (size_t)kc * 8;
+    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    int per_sm = 0;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem);
+    const int64_t groups = (p1 - p0 + 2 * NP - 1) / (2 * NP);
+    int64_t blocks = (groups + NT - 1) / NT;
+    const int64_t cap = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
+    if (blocks > cap) blocks = cap;
+    kern<<<(unsigned)blocks, NT, smem, s>>>(x, member, sums, counts, p0, p1, kc, shift, err);
+    return cudaGetLastError();
+}
+
 template <int NP, int CU, int NT, int MINB = 1>
 cudaError_t launch_assign16(const float* x, const float* cen, int32_t* member, int64_t* sums, int64_t* counts,
                             int64_t p0, int64_t p1, int kc, int shift, int* err, cudaStream_t s, int sms) {
@@ -325,10 +443,27 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
                                        : launch_assign16<1, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
             case 12: e = cu2 ? launch_assign16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
                              : launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            // default: measured fastest on B200 (profiles/r01/kmeans_variants.txt): 2 point pairs and
-            // 2 centroids per thread, 256 threads, 2 blocks/SM (16 warps/SM, 125 registers)
-            default: e = cu2 ? launch_assign16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                             : launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 17: e = cu2 ? launch_assign_c16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                             : launch_assign_c16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 13: e = cu2 ? launch_assign_c16<2, 2, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                             : launch_assign_c16<2, 1, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 14: e = cu2 ? launch_assign_c16<2, 2, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                             : launch_assign_c16<2, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 15: e = (kc % 4 == 0) ? launch_assign_c16<2, 4, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                                       : launch_assign_c16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 16: e = (kc % 4 == 0) ? launch_assign_c16<1, 4, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                                       : launch_assign_c16<1, 1, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            // default: centroids in constant memory when they fit (kc <= kConstCen), else the
+            // shared-memory kernel; measured on B200 (profiles/r01/kmeans_variants.txt)
+            default:
+                if (kc <= kConstCen)  // 3 blocks/SM (24 warps; ptxas keeps 80 registers + 24 B of spills
+                                      // outside the centroid loop): 21.05 ms vs 21.43 for 2 blocks/SM
+                    e = cu2 ? launch_assign_c16<2, 2, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                            : launch_assign_c16<2, 1, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms);
+                else
+                    e = cu2 ? launch_assign16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                            : launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms);
+                break;
         }
         if (e != cudaSuccess) return e;
     } else {
