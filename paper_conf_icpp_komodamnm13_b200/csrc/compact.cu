@@ -563,7 +563,10 @@ scatter_k(const uint8_t* __restrict__ packed, int64_t n_runs, const PtrList dsts
 
 // The paper's protocol (L133-135): for every chunk whose second-level bit is set, the whole chunk's
 // first-level bits decide which elements overwrite the peers' copies ("merged by the dirty bits").
-// One block per dirty chunk; lanes = bits of one word; clears the chunk's L1 words afterwards.
+// One block per dirty chunk (grid-stride); each warp takes kMU consecutive words at a time: all
+// their bitmap words, then all their dirty values are loaded (kMU x 128 B in flight per warp)
+// before the stores to every destination; clears the chunk's L1 words afterwards.
+constexpr int kMU = 8;
 template <typename T>
 __global__ void __launch_bounds__(kThreads)
 chunk_merge_k(uint32_t* __restrict__ l1, const uint32_t* __restrict__ l2, int64_t nwords, int cw_log2,
@@ -574,11 +577,18 @@ chunk_merge_k(uint32_t* __restrict__ l1, const uint32_t* __restrict__ l2, int64_
     for (int64_t c = blockIdx.x; c < nchunks; c += gridDim.x) {
         if (!((l2[c >> 5] >> (c & 31)) & 1u)) continue;  // clean chunk: skipped (block-uniform)
         const int64_t w0 = c * cwords, w1 = w0 + cwords < nwords ? w0 + cwords : nwords;
-        for (int64_t w = w0 + warp; w < w1; w += kThreads / 32) {
-            const uint32_t m = l1[w];
-            if ((m >> lane) & 1u) {
-                const T v = src[w * 32 + lane];
-                for (int d = 0; d < dsts.n; ++d) static_cast<T*>(dsts.p[d])[w * 32 + lane] = v;
+        for (int64_t wb = w0 + (int64_t)warp * kMU; wb < w1; wb += (int64_t)(kThreads / 32) * kMU) {
+            uint32_t m[kMU];
+            T v[kMU];
+#pragma unroll
+            for (int u = 0; u < kMU; ++u) m[u] = wb + u < w1 ? l1[wb + u] : 0u;
+#pragma unroll
+            for (int u = 0; u < kMU; ++u) v[u] = ((m[u] >> lane) & 1u) ? src[(wb + u) * 32 + lane] : T(0);
+            for (int d = 0; d < dsts.n; ++d) {
+                T* dp = static_cast<T*>(dsts.p[d]);
+#pragma unroll
+                for (int u = 0; u < kMU; ++u)
+                    if ((m[u] >> lane) & 1u) dp[(wb + u) * 32 + lane] = v[u];
             }
         }
         __syncthreads();
@@ -681,7 +691,7 @@ cudaError_t scatter_packed(const uint8_t* packed, int64_t n_runs, const PtrList&
 
 cudaError_t chunk_merge(uint32_t* l1, const uint32_t* l2, int64_t nwords, int chunk_words_log2, const void* values,
                         int esize, const PtrList& dsts, cudaStream_t s, int64_t* launches) {
-    const unsigned g = 148 * 4;
+    const unsigned g = 148 * 8;
     switch (esize) {
         case 1: chunk_merge_k<uint8_t><<<g, kThreads, 0, s>>>(l1, l2, nwords, chunk_words_log2, (const uint8_t*)values, dsts); break;
         case 2: chunk_merge_k<uint16_t><<<g, kThreads, 0, s>>>(l1, l2, nwords, chunk_words_log2, (const uint16_t*)values, dsts); break;
