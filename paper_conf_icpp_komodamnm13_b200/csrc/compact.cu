@@ -500,12 +500,24 @@ runlen_sum_k(const uint8_t* __restrict__ packed, int64_t n_runs, int64_t* __rest
     }
 }
 
-__global__ void __launch_bounds__(32) runlen_scan_k(int64_t* __restrict__ scratch) {
-    if (threadIdx.x == 0) {
-        int64_t run = 0;
-        for (int b = 0; b < kScatterBlocks; ++b) { scratch[kScatterBlocks + b] = run; run += scratch[b]; }
+// Exclusive scan of the kScatterBlocks segment sums (one block; was a single-thread loop: 20 us).
+__global__ void __launch_bounds__(1024) runlen_scan_k(int64_t* __restrict__ scratch) {
+    static_assert(kScatterBlocks <= 1024, "one element per thread");
+    __shared__ int64_t wsum[32];
+    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+    const int64_t v = tid < kScatterBlocks ? scratch[tid] : 0;
+    const int64_t inc = warp_incl_scan(v);
+    if (lane == 31) wsum[warp] = inc;
+    __syncthreads();
+    if (warp == 0) {
+        const int64_t x = wsum[lane];
+        wsum[lane] = warp_incl_scan(x) - x;
     }
+    __syncthreads();
+    if (tid < kScatterBlocks) scratch[kScatterBlocks + tid] = wsum[warp] + inc - v;
 }
+
+constexpr int kSU = 16;  // loads in flight per lane (scatter)
 
 template <typename T>
 __global__ void __launch_bounds__(kThreads)
@@ -517,7 +529,7 @@ scatter_k(const uint8_t* __restrict__ packed, int64_t n_runs, const PtrList dsts
     int64_t lo, hi;
     seg(n_runs, blockIdx.x, lo, hi);
     __shared__ int64_t s_start[kThreads], s_len[kThreads], s_off[kThreads];
-    __shared__ int64_t carry;
+    __shared__ int64_t carry, s_tot;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     if (tid == 0) carry = scratch[kScatterBlocks + blockIdx.x];
     __syncthreads();
@@ -534,25 +546,41 @@ scatter_k(const uint8_t* __restrict__ packed, int64_t n_runs, const PtrList dsts
         s_start[tid] = r < hi ? rs[r] : 0;
         s_len[tid] = len;
         s_off[tid] = carry + wo + inc - len;
+        if (tid == kThreads - 1) s_tot = wo + inc;
         __syncthreads();
         if (tid == kThreads - 1) carry += wo + inc;
         const int nr = (int)((hi - base) < kThreads ? (hi - base) : kThreads);
-        for (int q = warp; q < nr; q += kThreads / 32) {
-            const int64_t st = s_start[q], ln = s_len[q], of = s_off[q];
-            // 8 independent loads per lane in flight, then the stores to every destination
-            for (int64_t x0 = 0; x0 < ln; x0 += 32 * 8) {
-                T v[8];
+        // the chunk's payload [p0, p0 + tot) split evenly over the warps (runs differ in length:
+        // one run per warp left warps idle), each warp walking the runs that overlap its range
+        const int64_t p0 = s_off[0], tot = s_tot;
+        const int64_t plo = p0 + tot * warp / (kThreads / 32), phi = p0 + tot * (warp + 1) / (kThreads / 32);
+        int q = 0;
+        {
+            int a = 0, b = nr - 1;  // first run q with s_off[q] + s_len[q] > plo
+            while (a < b) {
+                const int m = (a + b) >> 1;
+                if (s_off[m] + s_len[m] > plo) b = m;
+                else a = m + 1;
+            }
+            q = a;
+        }
+        for (; q < nr && s_off[q] < phi; ++q) {
+            const int64_t st = s_start[q], of = s_off[q];
+            const int64_t xa = (plo > of ? plo : of) - of, xb = (phi < of + s_len[q] ? phi : of + s_len[q]) - of;
+            // kSU independent loads per lane in flight, then the stores to every destination
+            for (int64_t x0 = xa; x0 < xb; x0 += 32 * kSU) {
+                T v[kSU];
 #pragma unroll
-                for (int u = 0; u < 8; ++u) {
+                for (int u = 0; u < kSU; ++u) {
                     const int64_t x = x0 + 32 * u + lane;
-                    v[u] = x < ln ? payload[of + x] : T(0);
+                    v[u] = x < xb ? payload[of + x] : T(0);
                 }
                 for (int d = 0; d < dsts.n; ++d) {
                     T* dp = static_cast<T*>(dsts.p[d]) + st;
 #pragma unroll
-                    for (int u = 0; u < 8; ++u) {
+                    for (int u = 0; u < kSU; ++u) {
                         const int64_t x = x0 + 32 * u + lane;
-                        if (x < ln) dp[x] = v[u];
+                        if (x < xb) dp[x] = v[u];
                     }
                 }
             }
@@ -677,7 +705,7 @@ cudaError_t scatter_packed(const uint8_t* packed, int64_t n_runs, const PtrList&
                            int64_t* scratch, cudaStream_t s, int64_t* launches) {
     if (n_runs == 0 || dsts.n == 0) return cudaSuccess;
     runlen_sum_k<<<kScatterBlocks, kThreads, 0, s>>>(packed, n_runs, scratch);
-    runlen_scan_k<<<1, 32, 0, s>>>(scratch);
+    runlen_scan_k<<<1, 1024, 0, s>>>(scratch);
     switch (esize) {
         case 1: scatter_k<uint8_t><<<kScatterBlocks, kThreads, 0, s>>>(packed, n_runs, dsts, scratch); break;
         case 2: scatter_k<uint16_t><<<kScatterBlocks, kThreads, 0, s>>>(packed, n_runs, dsts, scratch); break;

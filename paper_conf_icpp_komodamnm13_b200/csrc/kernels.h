@@ -112,7 +112,7 @@ cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t extent, int64_t 
                           int esize, uint8_t* packed, int64_t n_runs, cudaStream_t s, int64_t* launches);
 // Scatter the runs of a canonical packed buffer into ndst replicas at the same global indices.
 // scratch: >= 2 * kScatterBlocks int64.
-constexpr int kScatterBlocks = 592;  // 4 x 148 SMs
+constexpr int kScatterBlocks = 592;  // 4 x 148 SMs (64 registers x 256 threads: 4 resident per SM)
 cudaError_t scatter_packed(const uint8_t* packed, int64_t n_runs, const PtrList& dsts, int esize,
                            int64_t* scratch, cudaStream_t s, int64_t* launches);
 
