@@ -106,10 +106,14 @@ cudaError_t compact_count(const uint32_t* l1, const uint32_t* l2, int64_t nwords
 cudaError_t compact_scan(const int64_t* tile_counts, int64_t ntiles, int64_t* tile_offs, int64_t* totals,
                          uint32_t* l2, int64_t nl2words, cudaStream_t s, int64_t* launches);
 // Pass 3: run starts/ends and payload into the canonical packed buffer; clears L1 words.
-// values holds elements [0, extent) (global indices).
+// values holds elements [0, extent) (global indices). push.n > 0 (only when compact_can_push()):
+// every dirty element is also stored at its global index into each replica of push (the other
+// partitions' replicas, local or IPC-mapped peers): compaction and propagation in one pass.
+bool compact_can_push();
 cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
                           const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
-                          int esize, uint8_t* packed, int64_t n_runs, cudaStream_t s, int64_t* launches);
+                          int esize, uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s,
+                          int64_t* launches);
 // Scatter the runs of a canonical packed buffer into ndst replicas at the same global indices.
 // scratch: >= 2 * kScatterBlocks int64.
 constexpr int kScatterBlocks = 592;  // 4 x 148 SMs (64 registers x 256 threads: 4 resident per SM)

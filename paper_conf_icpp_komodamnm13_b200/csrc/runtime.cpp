@@ -770,6 +770,21 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
 }
 
 // ---- coherence of undeclared writes (L129-135) -----------------------------------------------------
+// Every replica of r other than local partition li's: the local ones and (P2P mode) the peers'
+// replicas through their IPC mappings over NVLink.
+k::PtrList push_list(accmg_region_s* r, int li) {
+    const int g = first_local() + li;
+    k::PtrList dl{};
+    if (S.p2p) {
+        for (int h = 0; h < S.P; ++h)
+            if (h != g) dl.p[dl.n++] = r->gdev[h];
+    } else {
+        for (int h = 0; h < S.V; ++h)
+            if (h != li) dl.p[dl.n++] = r->dev[h];
+    }
+    return dl;
+}
+
 int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
     // 1. per local replica: (debug snapshot), count, scan
     {
@@ -808,7 +823,10 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
                                                    S.stream, &S.st.kernel_launches));
         }
     }
-    // 2. sizes to the host (one synchronisation for all regions)
+    // 2. sizes to the host (one synchronisation for all regions); with the P2P transport (or one
+    // process) the write pass also pushes every dirty element into the other replicas, so the
+    // packed buffer is not re-read by a separate scatter pass
+    const bool fused = !S.use_nccl && k::compact_can_push();
     int slot = 0;
     for (auto* r : regs)
         for (int li = 0; li < S.V; ++li, ++slot)
@@ -831,8 +849,10 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
             TRY(ensure_packed(t, t.packed_bytes));
             CUDA_TRY(cudaMemcpyAsync(t.packed, t.totals, 16, cudaMemcpyDeviceToDevice, S.stream));
             ProfScope ps(1);
+            k::PtrList push{};
+            if (fused) push = push_list(r, li);
             CUDA_TRY(k::compact_write(t.l1, t.nwords, r->extent, t.ntiles, t.tile_counts, t.tile_offs, t.tile_edges, r->dev[li],
-                                      (int)r->esize, t.packed, t.n_runs, S.stream, &S.st.kernel_launches));
+                                      (int)r->esize, t.packed, t.n_runs, push, S.stream, &S.st.kernel_launches));
             t.has_packed = true;
         }
     // 3. sizes of every partition's packet (all-gather across processes when needed)
@@ -904,22 +924,13 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
     // 4. exchange + scatter
     ProfScope ps(2);
     if (!multi) {
+        if (fused) return 0;  // pushed by the write pass
         // sender-side push: one scatter kernel writes the runs into every other replica — the
         // local ones and (P2P mode) the peers' replicas through their IPC mappings over NVLink
         for (auto* r : regs)
-            for (int li = 0; li < S.V; ++li) {
-                const int g = first_local() + li;
-                k::PtrList dl{};
-                if (S.p2p) {
-                    for (int h = 0; h < S.P; ++h)
-                        if (h != g) dl.p[dl.n++] = r->gdev[h];
-                } else {
-                    for (int h = 0; h < S.V; ++h)
-                        if (h != li) dl.p[dl.n++] = r->dev[h];
-                }
-                CUDA_TRY(k::scatter_packed(r->trk[li].packed, r->trk[li].n_runs, dl, (int)r->esize, S.scratch, S.stream,
-                                           &S.st.kernel_launches));
-            }
+            for (int li = 0; li < S.V; ++li)
+                CUDA_TRY(k::scatter_packed(r->trk[li].packed, r->trk[li].n_runs, push_list(r, li), (int)r->esize,
+                                           S.scratch, S.stream, &S.st.kernel_launches));
         return 0;
     }
     // receive every packet that comes from another process (or, in NCCL_ALL mode, from anyone) once

@@ -37,6 +37,19 @@ def main():
         x = gen.kmeans_points(5, 20000, 16, 32, gen.KM_OVERLAP)
         cen, mem = WL.kmeans_run(x, 32, 5)
         res = {"cen": cen, "mem": mem}
+    if work == "masked":
+        n = (1 << 20) + 4321
+        src = (gen.u_fill(21, 0, n) >> np.uint64(40)).astype(np.float32) * np.float32(2.0 ** -24)
+        dst = np.full(n, -1.0, dtype=np.float32)
+        ri, ro = A.accmg_region_create(src), A.accmg_region_create(dst)
+        for seed, dens, run in ((22, 0.5, 1), (23, 0.3, 70001), (24, 0.9, 40)):
+            m = gen.write_mask(seed, n, dens, run)
+            rm = A.accmg_region_create(m)
+            A.accmg_loop_launch(A.bounds([0], [n]), A.BODY_TEST_MASKED_WRITE,
+                                [A.access(ri, A.R), A.access(rm, A.R), A.access(ro, A.W)], A.accmg_args_masked(n))
+            A.accmg_region_destroy(rm)
+        A.accmg_sync_to_host(ro)
+        res = {"out": dst}
     if work == "scatter":
         n = 50000
         src = gen.jacobi_field(3, 317, 0, 317).reshape(-1)[:n].copy()
