@@ -1,14 +1,15 @@
 // Loop body variant: 2-D 5-point Jacobi with TMA-staged shared-memory tiles (impl = 2).
 //
 // Same operation and rounding as jacobi.cu. Each CTA owns a 128-column strip and a segment of
-// kTiles x 32 rows; one thread streams (32 + 2) x 136-float tiles (rows with their halo rows,
-// columns with 4 halo columns each side) through a 4-stage ring with cp.async.bulk.tensor.2d
+// tpc x 32 rows (tpc <= 8, chosen per launch to balance the waves); one thread streams
+// (32 + 2) x 136-float tiles (rows with their halo rows, columns with 4 halo columns each side)
+// through a 4-stage ring with cp.async.bulk.tensor.2d
 // completing on mbarriers; 8 warps compute 4 rows x 4 columns per lane from shared memory
 // (horizontal neighbours by shuffle) and store 128-bit vectors of interior points. The halo rows
 // of a tile are the previous / next tile's edge rows, so their second read hits L2.
 // The default body (measured faster than the register-marching kernel, impl = 1: profiles/ and
 // DESIGN.md). Write tracking (undeclared dst) runs once per CTA after its stores: mark_rect sets
-// the words of its 256-row x 128-column rectangle (plain stores for owned words, atomicOr on words
+// the words of its (32 tpc)-row x 128-column rectangle (plain stores for owned words, atomicOr on words
 // shared with the neighbouring strips) and the rows' chunk bits.
 #include "kernels.h"
 #include "tma_dev.cuh"
@@ -24,7 +25,7 @@ constexpr int RB = 32;             // rows computed per tile
 constexpr int BOXK = TK + 8;
 constexpr int BOXR = RB + 2;
 constexpr int kStages = 4;
-constexpr int kTiles = 8;          // tiles per CTA (256 rows)
+constexpr int kMaxTiles = 8;       // tiles per CTA (up to 256 rows; chosen per launch)
 constexpr uint32_t kTileBytes = BOXK * BOXR * 4;
 constexpr int kStageFloats = ((kTileBytes + 127) / 128) * 32;  // 128-byte aligned stages
 
@@ -35,15 +36,15 @@ __device__ __forceinline__ float st5(float n, float s, float w, float e) {
 template <bool TRACK>
 __global__ void __launch_bounds__(256)
 jacobi2d_tma_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, int64_t cols, int64_t r0, int64_t r1,
-               int64_t c0, int64_t c1, int64_t cbase, int64_t row_lo, Track t) {
+               int64_t c0, int64_t c1, int64_t cbase, int64_t row_lo, int tpc, Track t) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     float* tiles = reinterpret_cast<float*>(smem_raw);
     __shared__ __align__(8) uint64_t bar[kStages];
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int64_t k0 = cbase + (int64_t)blockIdx.x * TK;
-    const int64_t rs = r0 + (int64_t)blockIdx.y * (RB * kTiles);
+    const int64_t rs = r0 + (int64_t)blockIdx.y * (RB * tpc);
     if (rs >= r1) return;
-    const int ntiles = (int)((((r1 - rs) < RB * kTiles ? (r1 - rs) : RB * kTiles) + RB - 1) / RB);
+    const int ntiles = (int)((((r1 - rs) < RB * tpc ? (r1 - rs) : RB * tpc) + RB - 1) / RB);
     if (tid == 0) {
         for (int s = 0; s < kStages; ++s) dev::mbar_init(&bar[s], 1);
         dev::mbar_fence_init();
@@ -102,7 +103,7 @@ jacobi2d_tma_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst,
         }
     }
     if constexpr (TRACK) {  // dirty bits of the CTA's rectangle, once, after its stores
-        const int64_t re = rs + (int64_t)RB * kTiles < r1 ? rs + (int64_t)RB * kTiles : r1;
+        const int64_t re = rs + (int64_t)RB * tpc < r1 ? rs + (int64_t)RB * tpc : r1;
         dev::mark_rect(t.l1, t.l2, t.l2_shift, rs, re, cols, k0 > c0 ? k0 : c0, k0 + TK < c1 ? k0 + TK : c1, tid, 256);
     }
 }
@@ -135,8 +136,26 @@ cudaError_t jacobi2d_tma(const float* src, float* dst, int64_t rows, int64_t col
     auto kern = t.l1 ? jacobi2d_tma_k<true> : jacobi2d_tma_k<false>;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
     if (e != cudaSuccess) return e;
-    dim3 grid((unsigned)((c1 - cbase + TK - 1) / TK), (unsigned)((r1 - r0 + RB * kTiles - 1) / (RB * kTiles)));
-    kern<<<grid, 256, smem, s>>>(map, dst, cols, r0, r1, c0, c1, cbase, row_lo, t);
+    // rows per CTA (32 x tpc): the grid runs in waves of (resident CTAs per SM x SMs); pick tpc so
+    // that waves x (rows + 2 halo rows) per CTA is smallest -- a 4095-row partition (C2 at P = 8)
+    // runs 10 waves of 256-row CTAs with the last one 23 % full, but 15 full waves of 160 rows
+    int dev = 0, nsm = 148, per_sm = 1;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 256, smem);
+    const int64_t strips = (c1 - cbase + TK - 1) / TK, slots = (int64_t)nsm * (per_sm > 0 ? per_sm : 1);
+    int tpc = kMaxTiles;
+    int64_t best = -1;
+    for (int q = kMaxTiles; q >= 2; --q) {
+        const int64_t segs = (r1 - r0 + RB * q - 1) / (RB * q);
+        const int64_t cost = (strips * segs + slots - 1) / slots * (RB * q + 2);
+        if (best < 0 || cost * 100 < best * 98) {  // smaller tiles only for a >= 2 % gain
+            best = cost;
+            tpc = q;
+        }
+    }
+    dim3 grid((unsigned)strips, (unsigned)((r1 - r0 + RB * tpc - 1) / (RB * tpc)));
+    kern<<<grid, 256, smem, s>>>(map, dst, cols, r0, r1, c0, c1, cbase, row_lo, tpc, t);
     if (launches) *launches += 1;
     return cudaGetLastError();
 }
