@@ -193,7 +193,7 @@ assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __
 constexpr int kConstCen = 512;
 __constant__ float c_cen[kConstCen * 16];
 
-template <int NP, int CU, int NT, int MINB>
+template <int NP, int CU, int NT, int MINB, int UNR = 1>
 __global__ void __launch_bounds__(NT, MINB)
 assign_c16(const float* __restrict__ x, int32_t* __restrict__ member, int64_t* __restrict__ sums,
            int64_t* __restrict__ counts, int64_t p0, int64_t p1, int kc, int shift, int* err) {
@@ -236,7 +236,7 @@ assign_c16(const float* __restrict__ x, int32_t* __restrict__ member, int64_t* _
         int bi[PPT];
 #pragma unroll
         for (int q = 0; q < PPT; ++q) { bd[q] = __int_as_float(0x7f800000); bi[q] = 0; }
-#pragma unroll 1
+#pragma unroll UNR
         for (int c = 0; c < kc; c += CU) {
             uint64_t acc[CU][NP];
 #pragma unroll
@@ -281,10 +281,10 @@ assign_c16(const float* __restrict__ x, int32_t* __restrict__ member, int64_t* _
     flush_block(s_sum, s_cnt, sums, counts, kc, D);
 }
 
-template <int NP, int CU, int NT, int MINB>
+template <int NP, int CU, int NT, int MINB, int UNR = 1>
 cudaError_t launch_assign_c16(const float* x, const float* cen, int32_t* member, int64_t* sums, int64_t* counts,
                               int64_t p0, int64_t p1, int kc, int shift, int* err, cudaStream_t s, int sms) {
-    auto kern = assign_c16<NP, CU, NT, MINB>;
+    auto kern = assign_c16<NP, CU, NT, MINB, UNR>;
     cudaError_t e = cudaMemcpyToSymbolAsync(c_cen, cen, (size_t)kc * 16 * sizeof(float), 0, cudaMemcpyDeviceToDevice, s);
     if (e != cudaSuccess) return e;
     const size_t smem = (size_t)kc * 16 * 8 + (size_t)kc * 8;
@@ -443,6 +443,11 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
                                        : launch_assign16<1, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
             case 12: e = cu2 ? launch_assign16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
                              : launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 18: e = cu2 ? launch_assign_c16<2, 2, 256, 3, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                             : launch_assign_c16<2, 1, 256, 3, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 19: e = cu2 ? launch_assign_c16<2, 2, 256, 2, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                             : launch_assign_c16<2, 1, 256, 2, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
+            case 20: e = launch_assign_c16<2, 1, 256, 2, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
             case 17: e = cu2 ? launch_assign_c16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
                              : launch_assign_c16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
             case 13: e = cu2 ? launch_assign_c16<2, 2, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
