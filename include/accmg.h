@@ -56,6 +56,9 @@ extern "C" {
 /* dirty_protocol */
 #define ACCMG_DIRTY_RUNS   0
 #define ACCMG_DIRTY_CHUNKS 1
+/* halo_mode (declared windows) */
+#define ACCMG_HALO_AUTO 0      /* push predicted halos from the writing kernel when the body can */
+#define ACCMG_HALO_PULL 1      /* the paper's data loader only: pull before read (L119, L125) */
 
 typedef struct accmg_config {
     int32_t num_partitions;    /* P, the number of tasks groups every loop is divided into (L108);
@@ -78,6 +81,15 @@ typedef struct accmg_config {
                                   ACCMG_DIRTY_CHUNKS (the paper's protocol, L133-135: every dirty
                                   chunk with its first-level bits, merged by the bits; same-node
                                   transports only) */
+    int32_t halo_mode;         /* ACCMG_HALO_AUTO (default): when a loop writes a declared window and
+                                  another partition's last declared read window of that array
+                                  overlaps it (iterative codes reuse their patterns, L125), a body
+                                  that supports it (2-D Jacobi) stores those rows into that
+                                  partition's replica too (P2P mapping over NVLink, or a local
+                                  replica) and the rows count as valid there, so the next reader
+                                  pulls nothing; the bytes are accounted as declared transfers.
+                                  ACCMG_HALO_PULL: pull-before-read only. */
+    int32_t pad_;
     uint8_t nccl_unique_id[128]; /* world_size > 1: the job's id, made on rank 0 by
                                     accmg_nccl_unique_id() (NCCL modes) or accmg_unique_id() (P2P),
                                     broadcast by the caller (e.g. torch.distributed); P2P mode names

@@ -24,6 +24,7 @@ _lib = ctypes.CDLL(LIB_PATH)
 OK, EINVAL, ECUDA, ENCCL, ENOMEM, ESTATE, EUNSUPPORTED, ECONFLICT, EDATA = 0, -1, -2, -3, -4, -5, -6, -7, -8
 XCHG_AUTO, XCHG_NCCL_ALL, XCHG_NCCL = 0, 1, 2
 DIRTY_RUNS, DIRTY_CHUNKS = 0, 1
+HALO_AUTO, HALO_PULL = 0, 1
 R, W, RW, REDUCE_SUM = 1, 2, 3, 4
 BODY_JACOBI2D_5PT, BODY_GEMM_BF16_F32, BODY_KMEANS_ASSIGN, BODY_KMEANS_UPDATE = 1, 2, 3, 4
 BODY_SCATTER = 5
@@ -37,7 +38,8 @@ class accmg_config(ctypes.Structure):
     _fields_ = [("num_partitions", ctypes.c_int32), ("world_size", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("device", ctypes.c_int32), ("dirty_chunk_bytes", ctypes.c_int64),
                 ("exchange_mode", ctypes.c_int32), ("debug_checks", ctypes.c_int32), ("profile", ctypes.c_int32),
-                ("dirty_protocol", ctypes.c_int32), ("nccl_unique_id", ctypes.c_uint8 * 128)]
+                ("dirty_protocol", ctypes.c_int32), ("halo_mode", ctypes.c_int32), ("pad_", ctypes.c_int32),
+                ("nccl_unique_id", ctypes.c_uint8 * 128)]
 
 
 class accmg_bounds(ctypes.Structure):
@@ -177,9 +179,10 @@ def accmg_unique_id() -> bytes:
 
 def accmg_init(num_partitions: int = 1, world_size: int = 1, rank: int = 0, device: int = 0,
                dirty_chunk_bytes: int = 0, exchange_mode: int = XCHG_AUTO, debug_checks: int = 0,
-               profile: int = 0, nccl_unique_id: bytes | None = None, dirty_protocol: int = DIRTY_RUNS) -> None:
+               profile: int = 0, nccl_unique_id: bytes | None = None, dirty_protocol: int = DIRTY_RUNS,
+               halo_mode: int = HALO_AUTO) -> None:
     c = accmg_config(num_partitions, world_size, rank, device, dirty_chunk_bytes, exchange_mode, debug_checks,
-                     profile, dirty_protocol)
+                     profile, dirty_protocol, halo_mode)
     if nccl_unique_id is not None:
         ctypes.memmove(c.nccl_unique_id, nccl_unique_id, 128)
     _check(_lib.accmg_init(ctypes.byref(c)), "accmg_init")

@@ -51,9 +51,9 @@ __device__ __forceinline__ float st5(float n, float s, float w, float e) {
 }
 
 template <int VEC, bool TRACK, int kUnroll = TRACK ? kUnrollTrack : kUnrollPlain>
-__global__ void __launch_bounds__(kWarps * 32)
+__global__ void __launch_bounds__(kWarps * 32, 4)
 jacobi_rows(const float* __restrict__ src, float* __restrict__ dst, int64_t cols, int64_t r0, int64_t r1,
-            int64_t c0, int64_t c1, int64_t cbase, Track t) {
+            int64_t c0, int64_t c1, int64_t cbase, Track t, const HaloPush push) {
     const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
     const int64_t cw = cbase + ((int64_t)blockIdx.x * kWarps + warp) * (32 * VEC);  // warp's first column
     if (cw >= c1) return;                                                           // warp-uniform
@@ -113,6 +113,16 @@ jacobi_rows(const float* __restrict__ src, float* __restrict__ dst, int64_t cols
             } else {
                 if (nib) q[0] = o[0];
             }
+            if (push.n) {  // predicted readers' copies (rare rows; static indices)
+#pragma unroll
+                for (int pi = 0; pi < kMaxPush; ++pi) {
+                    if (pi >= push.n || r < push.lo[pi] || r >= push.hi[pi]) continue;  // warp-uniform
+                    float* pq = push.dst[pi] + r * cols + c;
+#pragma unroll
+                    for (int k = 0; k < VEC; ++k)
+                        if (nib & (1u << k)) pq[k] = o[k];
+                }
+            }
         }
         rb[0] = rb[kUnroll];
         rb[1] = rb[kUnroll + 1];
@@ -123,15 +133,15 @@ jacobi_rows(const float* __restrict__ src, float* __restrict__ dst, int64_t cols
 
 template <int VEC>
 cudaError_t launch_rows(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
-                        int64_t c0, int64_t c1, Track t, cudaStream_t s) {
+                        int64_t c0, int64_t c1, Track t, const HaloPush& push, cudaStream_t s) {
     (void)rows;
     const int64_t span = 32 * VEC * kWarps;
     const int64_t cbase = (c0 / (32 * VEC)) * (32 * VEC);
     dim3 grid((unsigned)((c1 - cbase + span - 1) / span), (unsigned)((r1 - r0 + kRowsPerSeg - 1) / kRowsPerSeg));
     if (t.l1)
-        jacobi_rows<VEC, true><<<grid, kWarps * 32, 0, s>>>(src, dst, cols, r0, r1, c0, c1, cbase, t);
+        jacobi_rows<VEC, true><<<grid, kWarps * 32, 0, s>>>(src, dst, cols, r0, r1, c0, c1, cbase, t, push);
     else
-        jacobi_rows<VEC, false><<<grid, kWarps * 32, 0, s>>>(src, dst, cols, r0, r1, c0, c1, cbase, t);
+        jacobi_rows<VEC, false><<<grid, kWarps * 32, 0, s>>>(src, dst, cols, r0, r1, c0, c1, cbase, t, push);
     return cudaGetLastError();
 }
 
@@ -171,7 +181,7 @@ masked_write_kernel(const float* __restrict__ in, const uint8_t* __restrict__ ma
 
 cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
                      int64_t c0, int64_t c1, int64_t src_lo, int64_t src_hi, Track t, int impl, cudaStream_t s,
-                     int64_t* launches) {
+                     int64_t* launches, const HaloPush& push) {
     if (r1 <= r0 || c1 <= c0) return cudaSuccess;
     if (impl == 0) {
         static int env = -1;
@@ -182,12 +192,12 @@ cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, i
         impl = env;
     }
     if (impl == 2) {
-        cudaError_t e = jacobi2d_tma(src, dst, rows, cols, r0, r1, c0, c1, src_lo, src_hi, t, s, launches);
+        cudaError_t e = jacobi2d_tma(src, dst, rows, cols, r0, r1, c0, c1, src_lo, src_hi, t, s, launches, push);
         if (e != cudaErrorNotSupported) return e;  // shapes the TMA variant does not take fall through
     }
     const bool vec4 = (cols % 4 == 0) && ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) % 16 == 0);
-    cudaError_t e = vec4 ? launch_rows<4>(src, dst, rows, cols, r0, r1, c0, c1, t, s)
-                         : launch_rows<1>(src, dst, rows, cols, r0, r1, c0, c1, t, s);
+    cudaError_t e = vec4 ? launch_rows<4>(src, dst, rows, cols, r0, r1, c0, c1, t, push, s)
+                         : launch_rows<1>(src, dst, rows, cols, r0, r1, c0, c1, t, push, s);
     if (launches) *launches += 1;
     return e;
 }

@@ -36,7 +36,7 @@ __device__ __forceinline__ float st5(float n, float s, float w, float e) {
 template <bool TRACK>
 __global__ void __launch_bounds__(256)
 jacobi2d_tma_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, int64_t cols, int64_t r0, int64_t r1,
-               int64_t c0, int64_t c1, int64_t cbase, int64_t row_lo, int tpc, Track t) {
+               int64_t c0, int64_t c1, int64_t cbase, int64_t row_lo, int tpc, Track t, const HaloPush push) {
     extern __shared__ __align__(128) unsigned char smem_raw[];
     float* tiles = reinterpret_cast<float*>(smem_raw);
     __shared__ __align__(8) uint64_t bar[kStages];
@@ -91,6 +91,19 @@ jacobi2d_tma_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst,
                     for (int c = 0; c < 4; ++c)
                         if (nib & (1u << c)) out[c] = o[c];
                 }
+#pragma unroll
+                for (int pi = 0; pi < kMaxPush; ++pi) {  // predicted readers' copies (static indices:
+                    // the parameter block stays in constant space)
+                    if (pi >= push.n || row < push.lo[pi] || row >= push.hi[pi]) continue;  // warp-uniform
+                    float* pout = push.dst[pi] + row * cols + k;
+                    if (full) {
+                        *reinterpret_cast<float4*>(pout) = make_float4(o[0], o[1], o[2], o[3]);
+                    } else {
+#pragma unroll
+                        for (int c = 0; c < 4; ++c)
+                            if (nib & (1u << c)) pout[c] = o[c];
+                    }
+                }
             }
         }
         __syncthreads();  // every thread is done with stage st
@@ -111,7 +124,8 @@ jacobi2d_tma_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst,
 }  // namespace
 
 cudaError_t jacobi2d_tma(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1, int64_t c0,
-                         int64_t c1, int64_t src_lo, int64_t src_hi, Track t, cudaStream_t s, int64_t* launches) {
+                         int64_t c1, int64_t src_lo, int64_t src_hi, Track t, cudaStream_t s, int64_t* launches,
+                         const HaloPush& push) {
     (void)rows;
     if (r1 <= r0 || c1 <= c0) return cudaSuccess;
     if (cols % 4 != 0 || (reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) % 16 != 0 ||
@@ -155,7 +169,7 @@ cudaError_t jacobi2d_tma(const float* src, float* dst, int64_t rows, int64_t col
         }
     }
     dim3 grid((unsigned)strips, (unsigned)((r1 - r0 + RB * tpc - 1) / (RB * tpc)));
-    kern<<<grid, 256, smem, s>>>(map, dst, cols, r0, r1, c0, c1, cbase, row_lo, tpc, t);
+    kern<<<grid, 256, smem, s>>>(map, dst, cols, r0, r1, c0, c1, cbase, row_lo, tpc, t, push);
     if (launches) *launches += 1;
     return cudaGetLastError();
 }

@@ -24,6 +24,16 @@ struct PtrList {
     int n;
 };
 
+// Predicted-halo push of a row-block body: rows [lo[k], hi[k]) of its output are stored also into
+// dst[k] (another partition's replica of the output array, global-index base; a local replica or
+// a peer's mapped over NVLink), from the same registers as the local store.
+constexpr int kMaxPush = 4;
+struct HaloPush {
+    float* dst[kMaxPush];
+    int64_t lo[kMaxPush], hi[kMaxPush];
+    int n;
+};
+
 // ---- loop bodies -----------------------------------------------------------------------------
 // 5-point Jacobi on rows [r0, r1) x cols [c0, c1) of a rows x cols fp32 array (global indices);
 // [src_lo, src_hi) = elements allocated behind src.
@@ -31,9 +41,10 @@ struct PtrList {
 // 2 = TMA-staged shared-memory tiles (jacobi2d_tma.cu).
 cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
                      int64_t c0, int64_t c1, int64_t src_lo, int64_t src_hi, Track t, int impl, cudaStream_t s,
-                     int64_t* launches);
+                     int64_t* launches, const HaloPush& push = HaloPush{});
 cudaError_t jacobi2d_tma(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1, int64_t c0,
-                         int64_t c1, int64_t src_lo, int64_t src_hi, Track t, cudaStream_t s, int64_t* launches);
+                         int64_t c1, int64_t src_lo, int64_t src_hi, Track t, cudaStream_t s, int64_t* launches,
+                         const HaloPush& push);
 
 // 3-D 7-point Jacobi (TMA-staged tiles) on planes [i0, i1) x rows [jl, jh) x cols [kl, kh) of an
 // n0 x n1 x n2 fp32 array; needs n2 % 4 == 0 (else cudaErrorNotSupported).

@@ -67,6 +67,8 @@ struct accmg_region_s {
     std::vector<uint8_t*> abase;     // V cudaMalloc'd pointers
     std::vector<Ival> arange;        // P allocated element range of every partition (global table)
     std::vector<IntervalSet> valid;  // P partitions
+    std::vector<IntervalSet> last_read;  // P: declared read windows of the last loop that read this
+                                         // region (halo-push prediction, L125); empty = no prediction
     IntervalSet host_valid;          // this process's host copy
     std::vector<Trk> trk;            // V
     std::vector<int64_t*> partial;   // V reduction partials (REDUCE_SUM)
@@ -89,7 +91,8 @@ struct State {
     bool init = false;
     accmg_config cfg{};
     int P = 1, W = 1, rank = 0, V = 1;
-    bool dry = false, nccl_all = false, p2p = false, use_nccl = false, chunks = false;
+    bool dry = false, nccl_all = false, p2p = false, use_nccl = false, chunks = false, halo_pull = false;
+    std::vector<k::HaloPush> cur_push;  // per local partition: this loop's predicted-halo pushes
     accmg::Bootstrap boot;
     uint64_t* sig = nullptr;         // P2P barrier flags (W entries), mapped by every peer
     std::vector<void*> peer_sig;     // W
@@ -685,7 +688,7 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
             auto x = static_cast<const accmg_args_jacobi2d*>(args);
             const Ival al = d[0].region->arange[g];
             e = k::jacobi2d((const float*)P(0), (float*)P(1), x->rows, x->cols, a, b, bd->lo[1], bd->hi[1], al.lo, al.hi,
-                            T(1), 0, S.stream, L);
+                            T(1), 0, S.stream, L, S.cur_push[li]);
             break;
         }
         case ACCMG_BODY_JACOBI2D_DEEP: {
@@ -1087,6 +1090,9 @@ int accmg_init(const accmg_config* cfg) {
     if (c.dirty_protocol != ACCMG_DIRTY_RUNS && c.dirty_protocol != ACCMG_DIRTY_CHUNKS)
         return fail(ACCMG_EINVAL, "init: bad dirty_protocol", false);
     S.chunks = c.dirty_protocol == ACCMG_DIRTY_CHUNKS;
+    if (c.halo_mode != ACCMG_HALO_AUTO && c.halo_mode != ACCMG_HALO_PULL)
+        return fail(ACCMG_EINVAL, "init: bad halo_mode", false);
+    S.halo_pull = c.halo_mode == ACCMG_HALO_PULL;
     if (S.chunks && S.use_nccl) return fail(ACCMG_EUNSUPPORTED, "init: the chunk protocol needs a same-node transport", false);
     if (S.dry) {
         S.init = true;
@@ -1169,6 +1175,7 @@ int accmg_region_create(void* host_array, size_t elem_size, int64_t extent, accm
     r->esize = (int64_t)elem_size;
     r->extent = extent;
     r->valid.assign(S.P, IntervalSet());
+    r->last_read.assign(S.P, IntervalSet());
     r->host_valid = IntervalSet(0, extent);
     r->trk.assign(S.V, Trk());
     r->dev.assign(S.V, nullptr);
@@ -1190,6 +1197,69 @@ int accmg_region_destroy(accmg_region r) {
     free_region(r);
     return 0;
 }
+
+namespace {
+// One predicted-halo push: partition g's body also stores elements [lo, hi) of descriptor desc's
+// array (rows of g's write window) into partition h's replica.
+struct PushPiece {
+    int desc, g, h;
+    int64_t lo, hi;
+};
+
+// Plans the pushes of one loop and sets S.cur_push for the local partitions. Only bodies that can
+// store their output rows twice take part (2-D Jacobi, output = descriptor 1). A piece is
+// W_g ∩ last_read[h] ∩ valid[h]: rows g writes that h read in the last loop reading this array (so
+// h is predicted to read them next, L125) and whose other elements h already holds (the body
+// stores only the interior columns; the rest of the row is unchanged and must be valid there).
+// Pieces must be whole rows, at most kMaxPush per writer, and the target replica must be
+// addressable (same process, or P2P mappings). The plan is a pure function of the global state, so
+// every process computes the same validity and byte counts.
+int plan_pushes(int body_id, const accmg_access* descs, const void* args,
+                const std::vector<std::vector<IntervalSet>>& need, std::vector<PushPiece>& out) {
+    S.cur_push.assign(S.V, k::HaloPush{});
+    if (S.halo_pull || S.P < 2 || body_id != ACCMG_BODY_JACOBI2D_5PT) return 0;
+    const int di = 1;
+    const accmg_access& d = descs[di];
+    if (!d.declared) return 0;
+    accmg_region_s* r = d.region;
+    const int64_t cols = static_cast<const accmg_args_jacobi2d*>(args)->cols;
+    for (int g = 0; g < S.P; ++g) {
+        std::vector<PushPiece> mine;
+        bool ok = true;
+        for (int h = 0; h < S.P && ok; ++h) {
+            if (h == g || r->last_read[h].empty()) continue;
+            if (!(rank_of(h) == rank_of(g) || S.p2p)) continue;  // unreachable without a mapping
+            IntervalSet piece = need[di][g].intersect(r->last_read[h]).intersect(r->valid[h]);
+            for (auto& iv : piece.items()) {
+                if (iv.lo % cols || iv.hi % cols || (int)mine.size() == k::kMaxPush) {
+                    ok = false;
+                    break;
+                }
+                mine.push_back({di, g, h, iv.lo, iv.hi});
+            }
+        }
+        if (!ok || mine.empty()) continue;
+        for (auto& pc : mine) {
+            out.push_back(pc);
+            const int64_t nb = (pc.hi - pc.lo) * r->esize;
+            if (local(pc.h)) {  // bytes are counted by the receiving process (as for pulls)
+                S.st.bytes_interpartition += nb;
+                S.st.bytes_declared += nb;
+                if (rank_of(pc.g) != rank_of(pc.h)) S.st.bytes_remote += nb;
+            }
+            if (local(g) && !S.dry) {
+                k::HaloPush& hp = S.cur_push[lidx(g)];
+                uint8_t* base = S.p2p ? r->gdev[pc.h] : r->dev[lidx(pc.h)];
+                hp.dst[hp.n] = reinterpret_cast<float*>(base);
+                hp.lo[hp.n] = pc.lo / cols;
+                hp.hi[hp.n] = pc.hi / cols;
+                ++hp.n;
+            }
+        }
+    }
+    return 0;
+}
+}  // namespace
 
 int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_access* descs, int n_descs,
                       const void* args, size_t args_bytes) {
@@ -1243,6 +1313,9 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
     TRY(run_xfers(xs));
     for (int i = 0; i < n_descs; ++i)
         for (int g = 0; g < S.P; ++g) descs[i].region->valid[g].add(need[i][g]);
+    // predicted-halo push (halo_mode AUTO, L125: iterative codes reuse their access patterns)
+    std::vector<PushPiece> pushes;
+    TRY(plan_pushes(body_id, descs, args, need, pushes));
 
     std::vector<bool> tracked(n_descs, false);
     std::vector<accmg_region_s*> tracked_regs;
@@ -1331,16 +1404,25 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
             r->host_valid.clear();
         } else if (descs[i].mode & ACCMG_W) {
             if (descs[i].declared) {
-                // the writer becomes the only holder of its write window
+                // the writer becomes the only holder of its write window, except for the rows it
+                // pushed into its predicted readers' replicas
                 for (int g = 0; g < S.P; ++g)
                     for (int h = 0; h < S.P; ++h)
                         if (h != g) r->valid[h].subtract(need[i][g]);
+                for (auto& pc : pushes)
+                    if (pc.desc == i) r->valid[pc.h].add(IntervalSet(pc.lo, pc.hi));
                 for (int g = 0; g < S.P; ++g) r->host_valid.subtract(need[i][g]);
             } else {
                 r->host_valid.clear();  // any element may have changed; every replica is coherent again
             }
         }
     }
+    // remember this loop's declared read windows (the prediction of the next loop's reads)
+    for (int i = 0; i < n_descs; ++i)
+        if (descs[i].mode & ACCMG_R) {
+            accmg_region_s* r = descs[i].region;
+            for (int g = 0; g < S.P; ++g) r->last_read[g] = descs[i].declared ? need[i][g] : IntervalSet();
+        }
     S.st.loops += 1;
     return 0;
 }

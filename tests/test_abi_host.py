@@ -52,7 +52,7 @@ def _compare_valid(regs_c, regs_m, P):
 @pytest.mark.parametrize("P", [1, 2, 3, 5, 8])
 def test_declared_jacobi_plan_vs_model(dry, P):
     N, S = 40, 5
-    dry(P)
+    dry(P, halo_mode=A.HALO_PULL)   # the paper's data loader: pull before read (the model's semantics)
     hA = np.zeros((N, N), np.float32)
     hB = np.zeros((N, N), np.float32)
     rA, rB = A.accmg_region_create(hA), A.accmg_region_create(hB)
@@ -115,6 +115,44 @@ def test_c1_worked_example_dry(dry):
     assert per[0] == 0 and all(p == 2048 for p in per[2:])
     # W_0 = [256, 32768) is owned by partition 0 after a write of the B array
     assert A.accmg_debug_valid(rB, 0)[0][1] >= 32768
+
+
+@pytest.mark.parametrize("P", [2, 3, 8])
+def test_halo_push_dry(P):
+    """halo_mode AUTO: from the second write of an array on, each writer's boundary rows are pushed
+    into the neighbours that read them in the previous loop (predicted from L125), so the steady
+    state pulls nothing and moves the same bytes per loop; validity is a superset of the pull-only
+    loader's (the pushed rows are valid one loop earlier) and the copy-out is identical."""
+    N, S = 40, 7
+    X = 2 * (P - 1) * 4 * N
+    res = {}
+    for mode in (A.HALO_PULL, A.HALO_AUTO):
+        A.accmg_init(num_partitions=P, device=-1, halo_mode=mode)
+        try:
+            h = [np.zeros((N, N), np.float32) for _ in range(2)]
+            rA, rB = A.accmg_region_create(h[0]), A.accmg_region_create(h[1])
+            per, prev = [], A.accmg_get_stats()
+            for s in range(S):
+                WL.jacobi_sweep(rA, rB, s, N, True)
+                cur = A.accmg_get_stats()
+                per.append((cur["bytes_declared"] - prev["bytes_declared"], cur["bytes_h2d"] - prev["bytes_h2d"]))
+                prev = cur
+            valid = [[A.accmg_debug_valid(r, g) for g in range(P)] for r in (rA, rB)]
+            A.accmg_sync_to_host(rA)
+            res[mode] = (per, valid, A.accmg_get_stats()["bytes_d2h"])
+        finally:
+            A.accmg_finalize()
+    pull, auto = res[A.HALO_PULL], res[A.HALO_AUTO]
+    assert [b for b, _ in pull[0]] == [0] + [X] * (S - 1)
+    assert [b for b, _ in auto[0]] == [0, 2 * X] + [X] * (S - 2)       # loop 1 pulls B and pushes A
+    assert [h for _, h in auto[0]] == [h for _, h in pull[0]]
+    assert auto[2] == pull[2]
+    for va, vp in zip(auto[1], pull[1]):
+        for ga, gp in zip(va, vp):
+            cover = np.zeros(N * N, bool)
+            for lo, hi in ga:
+                cover[lo:hi] = True
+            assert all(cover[lo:hi].all() for lo, hi in gp)
 
 
 def test_reduce_and_replica_bytes_dry(dry):

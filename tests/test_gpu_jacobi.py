@@ -43,14 +43,21 @@ def test_c1_declared_p2_bitexact_and_2048_bytes():
 
 
 @pytest.mark.parametrize("P", [1, 2, 3, 4, 5, 7, 8])
-def test_partition_invariance_bitexact(P):
+@pytest.mark.parametrize("halo", ["auto", "pull"])
+def test_partition_invariance_bitexact(P, halo):
+    """Any partition count gives the 1-partition result bit for bit, with the body pushing its
+    boundary rows into the neighbours' replicas (auto: S loops' worth of halo bytes, the last one
+    unused) or with pull-before-read only (S - 1 loops' worth)."""
+    from paper_conf_icpp_komodamnm13_b200 import accmg as Acc
     N, S = 1024, 6
     A0 = gen.jacobi_field(2, N)
     oA, oB = _oracle_run(A0, S)
-    A, B, _, st = _gpu_run(A0, S, P)
+    mode = Acc.HALO_AUTO if halo == "auto" else Acc.HALO_PULL
+    A, B, _, st = _gpu_run(A0, S, P, halo_mode=mode)
     assert np.array_equal(A, oA) and np.array_equal(B, oB)
     if P > 1:
-        assert st["bytes_declared"] == (S - 1) * 2 * (P - 1) * 4 * N
+        loops = S if halo == "auto" else S - 1
+        assert st["bytes_declared"] == loops * 2 * (P - 1) * 4 * N
 
 
 @pytest.mark.parametrize("N", [3, 5, 7, 65, 130, 257])

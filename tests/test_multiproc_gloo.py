@@ -29,7 +29,7 @@ def _worker(rank, world, port, V, q):
     from paper_conf_icpp_komodamnm13_b200 import workloads as WL
     os.environ.update(MASTER_ADDR="127.0.0.1", MASTER_PORT=str(port))
     dist.init_process_group("gloo", rank=rank, world_size=world)
-    A.accmg_init(num_partitions=world * V, world_size=world, rank=rank, device=-1)
+    A.accmg_init(num_partitions=world * V, world_size=world, rank=rank, device=-1, halo_mode=A.HALO_PULL)
     N, S = 64, 5
     hA = np.zeros((N, N), np.float32)
     hB = np.zeros((N, N), np.float32)
