@@ -115,6 +115,7 @@ def gemm_cfg(N, P, reps, check):
 
 def kmeans_cfg(n, iters, P, check):
     d, k = 16, 256
+    pk = peaks()
     t0 = time.perf_counter()
     x, lab, _ = gen.kmeans_points(4, n, d, k, gen.KM_LATTICE, labels=True)
     tgen = time.perf_counter() - t0
@@ -144,6 +145,11 @@ def kmeans_cfg(n, iters, P, check):
     # two lanes into one instruction, not two ops into one lane; scripts/fp32_micro.cu measures
     # 3.69e13 for the FADD2+FFMA2 pair the distance uses)
     out["frac_of_fp32_lane_peak_1965MHz"] = out["fp32_lane_ops_per_s"] / (148 * 128 * 1.965e9)
+    # tensor-core assign (default, kmeans_tc.cu): HBM-bound streaming of the points (64 B read +
+    # 4 B member written per point); the FP32 figures above are then "equivalent" lane-ops
+    out["assign_hbm_gbs"] = n * (d * 4 + 4) / (ms_assign / 1e3) / 1e9
+    out["assign_frac_of_measured_hbm"] = out["assign_hbm_gbs"] / pk["hbm_gbs"]
+    out["kmeans_impl"] = os.environ.get("ACCMG_KMEANS_IMPL", "0")
     if check:
         ok = np.array_equal(member, lab)
         # closed form: centroids are the exact means of the generated clusters

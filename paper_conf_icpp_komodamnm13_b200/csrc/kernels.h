@@ -84,6 +84,11 @@ cudaError_t masked_write(const float* in, const uint8_t* mask, float* out, int64
 cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int64_t* sums, int64_t* counts,
                           int64_t p0, int64_t p1, int d, int kc, int shift, int* err_flag, cudaStream_t s,
                           int64_t* launches);
+// Same loop with the distance cross term on the tcgen05 tensor cores and an exact fmaf re-check of
+// the candidates (kmeans_tc.cu): d == 16, 1 <= kc <= 256, x 16-byte aligned.
+int kmeans_tc_supported(const float* x, int d, int kc);
+cudaError_t kmeans_assign_tc(const float* x, const float* cen, int32_t* member, int64_t* sums, int64_t* counts,
+                             int64_t p0, int64_t p1, int kc, int shift, int* err_flag, cudaStream_t s, int sms);
 // k-means update over clusters [c0, c1); tracked writes of centroids, sums, counts.
 cudaError_t kmeans_update(int64_t* sums, int64_t* counts, float* cen, int64_t c0, int64_t c1, int d, int shift,
                           Track t_sums, Track t_counts, Track t_cen, cudaStream_t s, int64_t* launches);

@@ -416,6 +416,19 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
                           int64_t* launches) {
     if (p1 <= p0) return cudaSuccess;
     const int sms = sm_count();
+    // implementation (ACCMG_KMEANS_IMPL): 0 = tensor-core filter + exact re-check where supported
+    // (default), 1 = FP32-pipe kernels only
+    static int impl = -1;
+    if (impl < 0) {
+        const char* v = getenv("ACCMG_KMEANS_IMPL");
+        impl = v ? atoi(v) : 0;
+    }
+    if (impl == 0 && kmeans_tc_supported(x, d, kc)) {
+        cudaError_t e = kmeans_assign_tc(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms);
+        if (e != cudaSuccess) return e;
+        if (launches) *launches += 1;
+        return cudaSuccess;
+    }
     if (d == 16 && (reinterpret_cast<uintptr_t>(x) % 16) == 0) {
         // variant (tuning knob, default chosen from measurements in profiles/)
         static int variant = -1;
