@@ -120,6 +120,17 @@ __device__ __forceinline__ uint64_t sdesc_sw128(uint32_t saddr) {
 __device__ __forceinline__ uint32_t sw_off(uint32_t m, uint32_t kbyte) {
     return m * 128u + ((((kbyte >> 4) ^ (m & 7u)) << 4) | (kbyte & 15u));
 }
+// wait with a suspend-time hint: a warp that waits for a free stage sleeps instead of spinning on
+// issue slots the converter / epilogue warps of its SM sub-partition need
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n"
+        "WAITS_%=:\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%0], %1, %2;\n\t"
+        "@!p bra WAITS_%=;\n}" ::"r"(smem_u32(bar)),
+        "r"(parity), "r"(20000u)
+        : "memory");
+}
 __device__ __forceinline__ void sts_u8(uint32_t addr, uint32_t v) {
     asm volatile("st.shared.u8 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
 }
@@ -324,7 +335,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             for (int64_t i = 0; i < nt; ++i) {
                 const int64_t t = blockIdx.x + i * gridDim.x;
                 const int s = (int)(i % XS);
-                mbar_wait(&xempty[s], (uint32_t)((i / XS) & 1) ^ 1u);
+                mbar_wait_sleep(&xempty[s], (uint32_t)((i / XS) & 1) ^ 1u);
                 mbar_expect_tx(&xfull[s], kXBytes);  // rows past the end are zero-filled
                 dev::tma_load_2d(&xmap, &xfull[s], smem + OFF_X + s * kXBytes, 0, (int)(t * TM));
             }
@@ -385,9 +396,9 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
                 xv[4 * j] = v.x; xv[4 * j + 1] = v.y; xv[4 * j + 2] = v.z; xv[4 * j + 3] = v.w;
             }
             mbar_arrive(&xempty[s]);
-            mbar_wait(&aempty[a], (uint32_t)((i / AS) & 1) ^ 1u);
+            mbar_wait_sleep(&aempty[a], (uint32_t)((i / AS) & 1) ^ 1u);
             const int bs = (int)(i % BS);
-            mbar_wait(&bempty[bs], (uint32_t)((i / BS) & 1) ^ 1u);
+            mbar_wait_sleep(&bempty[bs], (uint32_t)((i / BS) & 1) ^ 1u);
             uint4 h0, l0, h1, l1;
             split8(xv, h0, l0);
             split8(xv + 8, h1, l1);
