@@ -333,9 +333,6 @@ def main():
                 elif cfg == "f1":
                     emit(scatter_cfg(1 << 26, P, 5))
                 elif cfg == "c4":
-                    if a.kmeans_n * 16 * 4 * P > (100 << 30):
-                        emit({"config": cfg, "P": P, "skipped": "full-extent virtual replicas would exceed 100 GiB"})
-                        continue
                     emit(kmeans_cfg(a.kmeans_n, a.kmeans_iters, P, a.check))
             except Exception as e:  # report and continue with the next config
                 emit({"config": cfg, "P": P, "error": repr(e)})
