@@ -14,6 +14,8 @@
 // round-to-nearest adds in the stated order, and store 128-bit vectors of interior points. The
 // optional fused epilogue sets the two-level dirty bits (L133-135) once per CTA after its stores
 // (mark_rect over its planes: owned words by plain stores, words shared with neighbours by atomicOr).
+#include <cstdlib>
+
 #include "kernels.h"
 #include "tma_dev.cuh"
 #include "tma_host.h"
@@ -24,26 +26,33 @@ namespace k {
 namespace {
 
 constexpr int TK = 128;          // k columns per CTA (32 lanes x float4)
-constexpr int TJ = 16;           // j rows per CTA (8 warps x 2 rows)
 constexpr int BOXK = TK + 8;     // k halo: 4 on each side (keeps 16-byte alignment)
-constexpr int BOXJ = TJ + 2;     // j halo: 1 on each side
-constexpr int kStages = 4;
-constexpr int kPlaneSeg = 32;    // planes per CTA
-constexpr int kTileFloats = BOXK * BOXJ;
-constexpr uint32_t kTileBytes = kTileFloats * 4;
-constexpr int kStageFloats = ((kTileBytes + 127) / 128) * 32;  // TMA destinations are 128-byte aligned
+// TJ: j rows per CTA (8 warps x TJ/8 rows); SEG: planes per CTA. Tile = (TJ + 2) x BOXK floats.
+template <int TJ, int kStages>
+struct Geo {
+    static constexpr int BOXJ = TJ + 2;  // j halo: 1 on each side
+    static constexpr uint32_t kTileBytes = BOXK * BOXJ * 4;
+    static constexpr int kStageFloats = ((kTileBytes + 127) / 128) * 32;  // TMA destinations 128-B aligned
+    static constexpr size_t kSmem = (size_t)kStages * kStageFloats * 4 + kStages * 8 + 128;
+};
 
 __device__ __forceinline__ float s7(float u, float d, float n, float s, float w, float e, float c) {
     const float ud = __fadd_rn(u, d), ns = __fadd_rn(n, s), we = __fadd_rn(w, e), cc = __fadd_rn(c, c);
     return __fmul_rn(__fadd_rn(__fadd_rn(ud, ns), __fadd_rn(we, cc)), 0.125f);
 }
 
-template <bool TRACK>
+template <bool TRACK, int TJ, int kPlaneSeg, int kStages>
 __global__ void __launch_bounds__(256)
 jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, int64_t n1, int64_t n2, int64_t i0,
              int64_t i1, int64_t jl, int64_t jh, int64_t kl, int64_t kh, int64_t kbase, int64_t plane_lo, Track t) {
-    __shared__ __align__(128) float tile[kStages][kStageFloats];
-    __shared__ __align__(8) uint64_t bar[kStages];
+    using G = Geo<TJ, kStages>;
+    constexpr int BOXJ = G::BOXJ;
+    constexpr uint32_t kTileBytes = G::kTileBytes;
+    extern __shared__ __align__(128) unsigned char smem3[];
+    float(*tile)[G::kStageFloats] = reinterpret_cast<float(*)[G::kStageFloats]>(
+        smem3 + ((128 - (dev::smem_u32(smem3) & 127)) & 127));
+    uint64_t* bar = reinterpret_cast<uint64_t*>(&tile[kStages][0]);
+    (void)BOXJ;
     const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
     const int64_t k0 = kbase + (int64_t)blockIdx.x * TK;
     const int64_t j0 = jl + (int64_t)blockIdx.y * TJ;
@@ -76,8 +85,8 @@ jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, i
         const float* P1 = tile[(q - 1) % kStages];
         const float* P2 = tile[q % kStages];
 #pragma unroll
-        for (int r = 0; r < 2; ++r) {
-            const int tr = 2 * warp + r + 1;  // tile row of j
+        for (int r = 0; r < TJ / 8; ++r) {
+            const int tr = (TJ / 8) * warp + r + 1;  // tile row of j
             const int64_t j = j0 + tr - 1;
             const float4 C = *reinterpret_cast<const float4*>(P1 + tr * BOXK + col);
             const float4 N = *reinterpret_cast<const float4*>(P1 + (tr - 1) * BOXK + col);
@@ -106,8 +115,8 @@ jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, i
             }
         }
         __syncthreads();  // every thread is done with plane i-1 (stage (q-2) % kStages)
-        if (tid == 0 && q + 2 < count) {
-            const int qn = q + 2;
+        if (tid == 0 && q + kStages - 2 < count) {  // the stage of plane i-1 takes plane i-1+kStages
+            const int qn = q + kStages - 2;
             asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
             dev::mbar_expect_tx(&bar[qn % kStages], kTileBytes);
             dev::tma_load_3d(&map, &bar[qn % kStages], tile[qn % kStages], (int)(k0 - 4), (int)(j0 - 1),
@@ -118,6 +127,21 @@ jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, i
         const int64_t je = j0 + TJ < jh ? j0 + TJ : jh, ka = k0 > kl ? k0 : kl, kb = k0 + TK < kh ? k0 + TK : kh;
         dev::mark_rect(t.l1, t.l2, t.l2_shift, ps * n1 + j0, ps * n1 + je, n2, ka, kb, tid, 256, (int)(pe - ps), n1);
     }
+}
+
+template <int TJ, int SEG, int NS = 4>
+cudaError_t launch3d(const CUtensorMap& map, float* dst, int64_t n1, int64_t n2, int64_t i0, int64_t i1, int64_t jl,
+                     int64_t jh, int64_t kl, int64_t kh, int64_t plane_lo, Track t, cudaStream_t s, int64_t* launches) {
+    const int64_t kbase = (kl / 4) * 4;
+    dim3 grid((unsigned)((kh - kbase + TK - 1) / TK), (unsigned)((jh - jl + TJ - 1) / TJ),
+              (unsigned)((i1 - i0 + SEG - 1) / SEG));
+    const size_t smem = Geo<TJ, NS>::kSmem;
+    auto kern = t.l1 ? jacobi3d_tma<true, TJ, SEG, NS> : jacobi3d_tma<false, TJ, SEG, NS>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;
+    kern<<<grid, 256, smem, s>>>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, kbase, plane_lo, t);
+    if (launches) *launches += 1;
+    return cudaGetLastError();
 }
 
 }  // namespace
@@ -139,21 +163,41 @@ cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64
     CUtensorMap map;
     cuuint64_t dims[3] = {(cuuint64_t)n2, (cuuint64_t)n1, (cuuint64_t)(plane_hi - plane_lo)};
     cuuint64_t strides[2] = {(cuuint64_t)n2 * 4, (cuuint64_t)n1 * n2 * 4};
-    cuuint32_t box[3] = {BOXK, BOXJ, 1};
+    static int vbox = -1;
+    if (vbox < 0) {
+        const char* v = getenv("ACCMG_J3D_VARIANT");
+        vbox = v ? atoi(v) : 0;
+    }
+    cuuint32_t box[3] = {BOXK, (cuuint32_t)((vbox == 1 || vbox == 3 || vbox == 6) ? 34 : 18), 1};
     cuuint32_t es[3] = {1, 1, 1};
     if (fn(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(src) + plane_lo * pl, dims, strides, box, es,
            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
         return cudaErrorNotSupported;
-    const int64_t kbase = (kl / 4) * 4;
-    dim3 grid((unsigned)((kh - kbase + TK - 1) / TK), (unsigned)((jh - jl + TJ - 1) / TJ),
-              (unsigned)((i1 - i0 + kPlaneSeg - 1) / kPlaneSeg));
-    if (t.l1)
-        jacobi3d_tma<true><<<grid, 256, 0, s>>>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, kbase, plane_lo, t);
-    else
-        jacobi3d_tma<false><<<grid, 256, 0, s>>>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, kbase, plane_lo, t);
-    if (launches) *launches += 1;
-    return cudaGetLastError();
+    // tile variant (ACCMG_J3D_VARIANT): 0 = 16 rows x 32 planes, 4 stages; 1 = 32 x 32; 2 = 16 x 64;
+    // 3 = 32 x 64; 4 / 5 = 16 x 32 with 6 / 8 stages; 6 = 32 x 32, 6 stages; 7 = 16 x 64, 6 stages.
+    // Default (-1): 8 stages (more bytes in flight per SM, 2 CTAs/SM) when the grid is at least 16
+    // waves of them, else 4 stages (5 CTAs/SM, shorter tail) — profiles/r01/f2_variants.jsonl
+    static int variant = -2;
+    if (variant == -2) {
+        const char* v = getenv("ACCMG_J3D_VARIANT");
+        variant = v ? atoi(v) : -1;
+    }
+    int var = variant;
+    if (var < 0) {
+        const int64_t ctas = ((kh - (kl / 4) * 4 + TK - 1) / TK) * ((jh - jl + 15) / 16) * ((i1 - i0 + 31) / 32);
+        var = ctas >= 16 * 2 * 148 ? 5 : 0;
+    }
+    switch (var) {
+        case 1: return launch3d<32, 32>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
+        case 2: return launch3d<16, 64>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
+        case 3: return launch3d<32, 64>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
+        case 4: return launch3d<16, 32, 6>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
+        case 5: return launch3d<16, 32, 8>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
+        case 6: return launch3d<32, 32, 6>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
+        case 7: return launch3d<16, 64, 6>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
+        default: return launch3d<16, 32>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
+    }
 }
 
 }  // namespace k

@@ -385,9 +385,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
         const float scale = (float)(1 << shift);
         int bad = 0;
         for (int64_t i = 0; i < nt; ++i) {
-            const int64_t t = blockIdx.x + i * gridDim.x;
             const int s = (int)(i % XS), a = (int)(i % AS);
-            const bool valid = p0 + t * TM + r < p1;
             mbar_wait(&xfull[s], (uint32_t)((i / XS) & 1));
             float xv[16];
 #pragma unroll
@@ -410,7 +408,12 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             sts_v4(ad + sw_off(r, 64), l0);
             sts_v4(ad + sw_off(r, 80), l1);
             // fixed point x * 2^shift, biased to unsigned: u = v + 2^31; byte b of dim j -> row 4j + b
+            // row m = 4j + b has swizzle phase m & 7 = 4 (j & 1) + b: eight per-thread base addresses,
+            // the row offset m * 128 is the store's immediate (st.shared.u8 keeps the low byte)
             const uint32_t ab = sAB + bs * kABBytes;
+            uint32_t base[8];
+#pragma unroll
+            for (int k = 0; k < 8; ++k) base[k] = ab + ((((uint32_t)r >> 4) ^ (uint32_t)k) << 4) + ((uint32_t)r & 15u);
 #pragma unroll
             for (int j = 0; j < 16; ++j) {
                 const float v = xv[j] * scale;  // exact: power-of-two scaling
@@ -420,7 +423,8 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
                 bad |= !ok;
                 const uint32_t u = (uint32_t)__float2int_rn(v) ^ 0x80000000u;
 #pragma unroll
-                for (int b = 0; b < 4; ++b) sts_u8(ab + sw_off(4 * j + b, r), (u >> (8 * b)) & 0xFFu);
+                for (int b = 0; b < 4; ++b)
+                    sts_u8(base[4 * (j & 1) + b] + (uint32_t)((4 * j + b) * 128), u >> (8 * b));
             }
             fence_async_smem();
             mbar_arrive(&afull[a]);
