@@ -269,7 +269,7 @@ __global__ void __launch_bounds__(kConsumers + 32)
 write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const int64_t* __restrict__ tile_counts,
              const int64_t* __restrict__ tile_offs, const uint32_t* __restrict__ tile_edges, int64_t ntiles,
              const T* __restrict__ values, uint8_t* __restrict__ packed, int64_t n_runs, int aligned,
-             const PtrList push) {
+             const PtrList push, int keep) {
     constexpr int SCW = kStageBytes / (32 * sizeof(T));  // words per stage
     constexpr int NSC = kTileWords / SCW;                 // stages per tile
     extern __shared__ __align__(128) unsigned char ring[];  // NST x kStageBytes
@@ -386,8 +386,10 @@ write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const in
                     spre[i] = run;
                     run += __popc(w);
                     const int64_t gw = w0 + i;
-                    for (uint32_t m = start_mask(w, W[kPad + i - 1]); m; m &= m - 1) run_start[ks++] = gw * 32 + (__ffs(m) - 1);
-                    for (uint32_t m = end_mask(w, W[kPad + i + 1]); m; m &= m - 1) run_end[ke++] = gw * 32 + __ffs(m);
+                    if (keep) {
+                        for (uint32_t m = start_mask(w, W[kPad + i - 1]); m; m &= m - 1) run_start[ks++] = gw * 32 + (__ffs(m) - 1);
+                        for (uint32_t m = end_mask(w, W[kPad + i + 1]); m; m &= m - 1) run_end[ke++] = gw * 32 + __ffs(m);
+                    }
                 }
             }
         }
@@ -404,7 +406,7 @@ write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const in
                     const uint32_t m = W[kPad + i];
                     if ((m >> lane) & 1u) {
                         const T v = V[j * 32 + lane];
-                        tile_payload[spre[i] + __popc(m & lt)] = v;
+                        if (keep) tile_payload[spre[i] + __popc(m & lt)] = v;
                         const int64_t e = (w0 + i) * 32 + lane;
                         for (int d = 0; d < push.n; ++d) static_cast<T*>(push.p[d])[e] = v;
                     }
@@ -425,7 +427,7 @@ write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const in
 #pragma unroll
                 for (int u = 0; u < kU; ++u)
                     if ((m[u] >> lane) & 1u) {
-                        tile_payload[spre[base + u] + __popc(m[u] & lt)] = v[u];
+                        if (keep) tile_payload[spre[base + u] + __popc(m[u] & lt)] = v[u];
                         const int64_t e = (w0 + base + u) * 32 + lane;
                         for (int d = 0; d < push.n; ++d) static_cast<T*>(push.p[d])[e] = v[u];
                     }
@@ -439,7 +441,7 @@ write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const in
 template <typename T, int NST>
 cudaError_t launch_write_pipe_st(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
                                  const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
-                                 uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s) {
+                                 uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s, int keep) {
     auto kern = write_pipe_k<T, NST>;
     const size_t smem = (size_t)NST * kStageBytes;
     cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
@@ -457,7 +459,7 @@ cudaError_t launch_write_pipe_st(uint32_t* l1, int64_t nwords, int64_t extent, i
     int64_t grid = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
     if (grid > ntiles) grid = ntiles;
     kern<<<(unsigned)grid, kConsumers + 32, smem, s>>>(l1, nwords, extent, tile_counts, tile_offs, tile_edges, ntiles,
-                                                        static_cast<const T*>(values), packed, n_runs, aligned, push);
+                                                        static_cast<const T*>(values), packed, n_runs, aligned, push, keep);
     return cudaGetLastError();
 }
 
@@ -467,21 +469,21 @@ cudaError_t launch_write_pipe_st(uint32_t* l1, int64_t nwords, int64_t extent, i
 template <typename T>
 cudaError_t launch_write_stream(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
                                 const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
-                                uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s) {
+                                uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s, int keep) {
     static int st = -1;
     if (st < 0) {
         const char* v = getenv("ACCMG_COMPACT_STAGES");
         st = v ? atoi(v) : 3;
     }
     switch (st) {
-        case 2: return launch_write_pipe_st<T, 2>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s);
-        case 6: return launch_write_pipe_st<T, 6>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s);
-        case 8: return launch_write_pipe_st<T, 8>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s);
-        case 4: return launch_write_pipe_st<T, 4>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s);
-        case 10: return launch_write_pipe_st<T, 10>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s);
-        case 16: return launch_write_pipe_st<T, 16>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s);
-        case 24: return launch_write_pipe_st<T, 24>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s);
-        default: return launch_write_pipe_st<T, 3>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s);
+        case 2: return launch_write_pipe_st<T, 2>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
+        case 6: return launch_write_pipe_st<T, 6>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
+        case 8: return launch_write_pipe_st<T, 8>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
+        case 4: return launch_write_pipe_st<T, 4>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
+        case 10: return launch_write_pipe_st<T, 10>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
+        case 16: return launch_write_pipe_st<T, 16>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
+        case 24: return launch_write_pipe_st<T, 24>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
+        default: return launch_write_pipe_st<T, 3>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
     }
 }
 
@@ -700,17 +702,17 @@ bool compact_can_push() {
 cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
                           const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
                           int esize, uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s,
-                          int64_t* launches) {
+                          int64_t* launches, int keep) {
     dim3 g((unsigned)ntiles);
     const int impl = compact_impl();
     if (push.n > 0 && impl == 1) return cudaErrorNotSupported;
     if (impl != 1) {
         cudaError_t e;
         switch (esize) {
-            case 1: e = launch_write_stream<uint8_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s); break;
-            case 2: e = launch_write_stream<uint16_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s); break;
-            case 4: e = launch_write_stream<uint32_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s); break;
-            case 8: e = launch_write_stream<uint64_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s); break;
+            case 1: e = launch_write_stream<uint8_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
+            case 2: e = launch_write_stream<uint16_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
+            case 4: e = launch_write_stream<uint32_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
+            case 8: e = launch_write_stream<uint64_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
             default: return cudaErrorInvalidValue;
         }
         if (launches) *launches += 1;

@@ -129,7 +129,7 @@ bool compact_can_push();
 cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
                           const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
                           int esize, uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s,
-                          int64_t* launches);
+                          int64_t* launches, int keep_packed = 1);
 // Scatter the runs of a canonical packed buffer into ndst replicas at the same global indices.
 // scratch: >= 2 * kScatterBlocks int64.
 constexpr int kScatterBlocks = 592;  // 4 x 148 SMs (64 registers x 256 threads: 4 resident per SM)

@@ -849,14 +849,21 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
             if (S.h_pin[4 * slot + 3] != t.n_runs) return fail(ACCMG_ECUDA, "compaction: run starts != run ends", true);
             t.packed_bytes = 16 + 16 * t.n_runs + r->esize * t.n_elems;
             if (S.chunks) continue;  // merged already; nothing to pack
-            TRY(ensure_packed(t, t.packed_bytes));
-            CUDA_TRY(cudaMemcpyAsync(t.packed, t.totals, 16, cudaMemcpyDeviceToDevice, S.stream));
+            // the canonical packed buffer is materialised only when something reads it: the
+            // message-passing transport, the separate scatter pass, or debug inspection; with the
+            // fused push the write pass stores each dirty element into the other replicas only
+            const bool keep = !fused || S.cfg.debug_checks;
+            if (keep) {
+                TRY(ensure_packed(t, t.packed_bytes));
+                CUDA_TRY(cudaMemcpyAsync(t.packed, t.totals, 16, cudaMemcpyDeviceToDevice, S.stream));
+            }
             ProfScope ps(1);
             k::PtrList push{};
             if (fused) push = push_list(r, li);
             CUDA_TRY(k::compact_write(t.l1, t.nwords, r->extent, t.ntiles, t.tile_counts, t.tile_offs, t.tile_edges, r->dev[li],
-                                      (int)r->esize, t.packed, t.n_runs, push, S.stream, &S.st.kernel_launches));
-            t.has_packed = true;
+                                      (int)r->esize, keep ? t.packed : nullptr, t.n_runs, push, S.stream,
+                                      &S.st.kernel_launches, keep ? 1 : 0));
+            t.has_packed = keep;
         }
     // 3. sizes of every partition's packet (all-gather across processes when needed)
     std::vector<int64_t> runs(S.P * regs.size()), elems(S.P * regs.size()), chunks(S.P * regs.size());
