@@ -1,3 +1,6 @@
+"""Phase timing of the tensor-core k-means kernel: needs a build of kmeans_tc.cu with the clock64
+instrumentation (km_prof[] counters + accmg_km_prof_read, see profiles/r01/kmeans_tc.log); the
+default build does not export accmg_km_prof_read."""
 import ctypes, os, sys
 sys.path.insert(0, '/root/repo')
 import numpy as np
