@@ -425,9 +425,12 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
     }
     if (impl == 0 && kmeans_tc_supported(x, d, kc)) {
         cudaError_t e = kmeans_assign_tc(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms);
-        if (e != cudaSuccess) return e;
-        if (launches) *launches += 1;
-        return cudaSuccess;
+        if (e == cudaSuccess) {
+            if (launches) *launches += 1;
+            return cudaSuccess;
+        }
+        if (e != cudaErrorNotSupported) return e;
+        (void)cudaGetLastError();  // unsupported shape for the tensor-core kernel: FP32-pipe kernels below
     }
     if (d == 16 && (reinterpret_cast<uintptr_t>(x) % 16) == 0) {
         // variant (tuning knob, default chosen from measurements in profiles/)

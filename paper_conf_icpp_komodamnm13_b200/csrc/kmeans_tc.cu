@@ -594,6 +594,7 @@ int kmeans_tc_supported(const float* x, int d, int kc) {
 cudaError_t kmeans_assign_tc(const float* x, const float* cen, int32_t* member, int64_t* sums, int64_t* counts,
                              int64_t p0, int64_t p1, int kc, int shift, int* err_flag, cudaStream_t s, int sms) {
     if (p1 <= p0) return cudaSuccess;
+    if (p1 - p0 > (int64_t)INT32_MAX - TM) return cudaErrorNotSupported;  // TMA row coordinates are int32
     const int npad = ((kc + 31) / 32) * 32;
     cudaError_t e = cudaFuncSetAttribute(assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemTC);
     if (e != cudaSuccess) return e;
