@@ -479,11 +479,11 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
                         for (int g = 0; g < 8; ++g) gm[h * 32 + ch * 8 + g] = -0x1p120f;
                     }
                 }
+                if (h < nh) {  // this half's accumulator is consumed: the next tile's MMAs may start
+                    tc_fence_before();
+                    mbar_arrive(&dempty[h]);
+                }
             }
-            tc_fence_before();
-#pragma unroll
-            for (int h = 0; h < 2; ++h)
-                if (h < nh) mbar_arrive(&dempty[h]);
             float vm[8];
 #pragma unroll
             for (int u = 0; u < 8; ++u)
