@@ -60,7 +60,7 @@ def test_wide_dynamic_range():
     _run(x, 100, 3, P=2, shift=0)
 
 
-@pytest.mark.parametrize("k", [1, 31, 32, 33, 255, 256])
+@pytest.mark.parametrize("k", [1, 31, 32, 33, 128, 129, 160, 200, 255, 256])
 def test_k_edges_ragged_n(k):
     n = 7 * 128 + 77
     x = gen.kmeans_points(7, n, 16, max(k, 2), gen.KM_OVERLAP)
