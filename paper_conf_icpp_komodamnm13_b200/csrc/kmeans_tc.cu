@@ -78,7 +78,8 @@ constexpr int OFF_X = OFF_OH + OS * kOHBytes;
 constexpr int kGrpBytes = 272;
 constexpr int OFF_PC = OFF_X + XS * kXBytes;
 constexpr int OFF_BAR = OFF_PC + (KMAX / 4) * kGrpBytes;
-constexpr int kNumBars = 2 * XS + 2 * AS + BS + 4 + 2 * OS + 1;
+constexpr int kMaxQ = 8;                // distance accumulator column groups (>= KMAX / QW)
+constexpr int kNumBars = 2 * XS + 2 * AS + BS + 2 * kMaxQ + 2 * OS + 1;
 constexpr int OFF_MISC = OFF_BAR + kNumBars * 8;    // tmem slot, Cinf bits, C2 bits
 constexpr int kSmemTC = OFF_MISC + 16 + 1024;       // + alignment slack
 static_assert(OFF_AB % 1024 == 0 && OFF_BD % 1024 == 0 && OFF_OH % 1024 == 0 && OFF_X % 1024 == 0, "align");
@@ -216,6 +217,9 @@ __device__ __forceinline__ float next_below(float a) {
     return __int_as_float(a > 0.f ? b - 1 : b + 1);
 }
 
+// QW: width (centroid columns) of each distance accumulator; each has its own full / empty
+// barriers, so the MMAs of the next tile refill a group as soon as the epilogue has read it
+template <int QW>
 __global__ void __launch_bounds__(kThreadsTC, 1)
 assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ cen, int32_t* __restrict__ member,
           int64_t* __restrict__ sums, int64_t* __restrict__ counts, int64_t p0, int64_t p1, int kc, int npad,
@@ -234,8 +238,8 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
     uint64_t* aempty = afull + AS;
     uint64_t* bempty = aempty + AS;
     uint64_t* dfull = bempty + BS;
-    uint64_t* dempty = dfull + 2;
-    uint64_t* ofull = dempty + 2;
+    uint64_t* dempty = dfull + kMaxQ;
+    uint64_t* ofull = dempty + kMaxQ;
     uint64_t* oempty = ofull + OS;
     uint64_t* sdone = oempty + OS;
     uint32_t* misc = reinterpret_cast<uint32_t*>(smem + OFF_MISC);  // [0] tmem, [1] Cinf bits, [2] C2 bits
@@ -243,7 +247,9 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t ntiles = (p1 - p0 + TM - 1) / TM;
     const int64_t nt = blockIdx.x < ntiles ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
-    const int nh = (npad + 127) / 128;  // 128-centroid halves
+    const int nh = (npad + 127) / 128;  // 128-centroid halves (reduction)
+    constexpr int NQ = KMAX / QW;       // distance accumulator groups
+    const int nq = (npad + QW - 1) / QW;
 
     // ---- setup: constant operand parts, centroids, bounds, barriers, TMEM
     if (tid == 0) { misc[1] = 0u; misc[2] = 0u; }
@@ -270,7 +276,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
         for (int s = 0; s < XS; ++s) { mbar_init(&xfull[s], 1); mbar_init(&xempty[s], 256); }
         for (int a = 0; a < AS; ++a) { mbar_init(&afull[a], 128); mbar_init(&aempty[a], 1); }
         for (int b = 0; b < BS; ++b) mbar_init(&bempty[b], 1);
-        for (int b = 0; b < 2; ++b) { mbar_init(&dfull[b], 1); mbar_init(&dempty[b], 128); }
+        for (int b = 0; b < kMaxQ; ++b) { mbar_init(&dfull[b], 1); mbar_init(&dempty[b], 128); }
         for (int o = 0; o < OS; ++o) { mbar_init(&ofull[o], 128); mbar_init(&oempty[o], 1); }
         mbar_init(sdone, 1);
         dev::mbar_fence_init();
@@ -307,6 +313,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             const float a2 = nh_ - a0 - a1;
             n01 = bf2(a0, a1);
             n2 = bf2(a2, 0.f);
+
             atomicMax(&misc[1], __float_as_uint(m));  // non-negative floats order as their bits
             atomicMax(&misc[2], __float_as_uint(q));
         } else {
@@ -319,6 +326,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             sts_v4(sBD + sw_off(n, 80), z);
             n01 = bf2(-0x1p100f, 0.f);  // padding centroid: v = -2^100, never a candidate
             n2 = 0u;
+
         }
         sts_v4(sBD + sw_off(n, 96), make_uint4(n01, n2, 0, 0));
         sts_v4(sBD + sw_off(n, 112), make_uint4(0, 0, 0, 0));
@@ -360,18 +368,17 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             for (int64_t i = 0; i < nt; ++i) {
                 const int a = (int)(i % AS);
                 mbar_wait(&afull[a], (uint32_t)((i / AS) & 1));
-                for (int h = 0; h < nh; ++h) {
-                    const int hb = h;
-                    mbar_wait(&dempty[hb], (uint32_t)(i & 1) ^ 1u);
+                for (int g = 0; g < nq; ++g) {
+                    mbar_wait(&dempty[g], (uint32_t)(i & 1) ^ 1u);
                     tc_fence_after();
-                    const int wh = (npad - 128 * h) < 128 ? (npad - 128 * h) : 128;
-                    const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(wh >> 3) << 17) |
+                    const int wq = (npad - QW * g) < QW ? (npad - QW * g) : QW;
+                    const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(wq >> 3) << 17) |
                                            ((uint32_t)(TM >> 4) << 24);
 #pragma unroll
                     for (int k = 0; k < 4; ++k)
-                        mma_f16(tmem + 128u * hb, sdesc_sw128(sAD + a * kADBytes + k * 32),
-                                sdesc_sw128(sBD + h * 16384 + k * 32), idesc, k ? 1u : 0u);
-                    tc_commit(&dfull[hb]);
+                        mma_f16(tmem + (uint32_t)(QW * g), sdesc_sw128(sAD + a * kADBytes + k * 32),
+                                sdesc_sw128(sBD + g * QW * 128 + k * 32), idesc, k ? 1u : 0u);
+                    tc_commit(&dfull[g]);
                 }
                 tc_commit(&aempty[a]);
                 if (i >= 1) reduce(i - 1);
@@ -452,36 +459,37 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
                 xv[4 * j] = v.x; xv[4 * j + 1] = v.y; xv[4 * j + 2] = v.z; xv[4 * j + 3] = v.w;
             }
             mbar_arrive(&xempty[s]);
-            // pass 1 over both halves: maxima of the 4-column groups (64 registers), then the
-            // accumulators go back to the MMA warp
+            // pass 1 over the accumulator groups: maxima of the 4-column groups (64 registers); each
+            // accumulator goes back to the MMA warp as soon as it is read
             float gm[64];
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                if (h < nh) {
-                    mbar_wait(&dfull[h], (uint32_t)(i & 1));
+            for (int qg = 0; qg < NQ; ++qg) {
+                if (qg < nq) {
+                    mbar_wait(&dfull[qg], (uint32_t)(i & 1));
                     tc_fence_after();
                 }
-                const int nch = h < nh ? (((npad - 128 * h) < 128 ? (npad - 128 * h) : 128) / 32) : 0;
-                const uint32_t tb = tmem + ((uint32_t)(q * 32) << 16) + 128u * h;
+                const int ncq = qg < nq ? (((npad - QW * qg) < QW ? (npad - QW * qg) : QW) / 32) : 0;
+                const uint32_t tb = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(QW * qg);
 #pragma unroll
-                for (int ch = 0; ch < 4; ++ch) {
-                    if (ch < nch) {
+                for (int c = 0; c < QW / 32; ++c) {
+                    const int ch = qg * (QW / 32) + c;
+                    if (c < ncq) {
                         uint32_t v[32];
-                        tmem_ld<32>(tb + ch * 32, v);
+                        tmem_ld<32>(tb + c * 32, v);
                         tmem_wait();
 #pragma unroll
                         for (int g = 0; g < 8; ++g)
-                            gm[h * 32 + ch * 8 + g] =
+                            gm[ch * 8 + g] =
                                 max3(__uint_as_float(v[4 * g]), __uint_as_float(v[4 * g + 1]),
                                      fmaxf(__uint_as_float(v[4 * g + 2]), __uint_as_float(v[4 * g + 3])));
                     } else {
 #pragma unroll
-                        for (int g = 0; g < 8; ++g) gm[h * 32 + ch * 8 + g] = -0x1p120f;
+                        for (int g = 0; g < 8; ++g) gm[ch * 8 + g] = -0x1p120f;
                     }
                 }
-                if (h < nh) {  // this half's accumulator is consumed: the next tile's MMAs may start
+                if (qg < nq) {  // this accumulator is consumed: the next tile's MMAs may refill it
                     tc_fence_before();
-                    mbar_arrive(&dempty[h]);
+                    mbar_arrive(&dempty[qg]);
                 }
             }
             float vm[8];
@@ -596,7 +604,15 @@ cudaError_t kmeans_assign_tc(const float* x, const float* cen, int32_t* member, 
     if (p1 <= p0) return cudaSuccess;
     if (p1 - p0 > (int64_t)INT32_MAX - TM) return cudaErrorNotSupported;  // TMA row coordinates are int32
     const int npad = ((kc + 31) / 32) * 32;
-    cudaError_t e = cudaFuncSetAttribute(assign_tc, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemTC);
+    // accumulator group width (ACCMG_KMEANS_TC_QW: 32, 64 or 128 centroid columns; same-box A/B in
+    // profiles/r01/kmeans_tc.log: 128 = 22.9 ms, 64 = 29.4, 32 = 42.4 — more, narrower MMAs lose)
+    static int qw = -1;
+    if (qw < 0) {
+        const char* v = getenv("ACCMG_KMEANS_TC_QW");
+        qw = v ? atoi(v) : 128;
+    }
+    auto kern = qw == 64 ? assign_tc<64> : qw == 32 ? assign_tc<32> : assign_tc<128>;
+    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemTC);
     if (e != cudaSuccess) return e;
     const int64_t ntiles = (p1 - p0 + TM - 1) / TM;
     // s32 reduction accumulators: byte sums <= 255 per point, so at most 2^23 points (65536 tiles)
@@ -617,7 +633,7 @@ cudaError_t kmeans_assign_tc(const float* x, const float* cen, int32_t* member, 
            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
         return cudaErrorNotSupported;
-    assign_tc<<<(unsigned)blocks, kThreadsTC, kSmemTC, s>>>(xmap, cen, member, sums, counts, p0, p1, kc, npad, shift,
+    kern<<<(unsigned)blocks, kThreadsTC, kSmemTC, s>>>(xmap, cen, member, sums, counts, p0, p1, kc, npad, shift,
                                                             err_flag);
     return cudaGetLastError();
 }
