@@ -13,7 +13,8 @@ import re
 import numpy as np
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libaccmg.so")
+# ACCMG_LIBRARY: another in-tree build of the same library (same-box A/B measurements only)
+LIB_PATH = os.environ.get("ACCMG_LIBRARY") or os.path.join(_HERE, "libaccmg.so")
 HEADER = os.path.join(os.path.dirname(_HERE), "include", "accmg.h")
 
 if not os.path.exists(LIB_PATH):

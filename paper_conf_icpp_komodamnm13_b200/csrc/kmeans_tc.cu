@@ -81,7 +81,8 @@ constexpr int OFF_BAR = OFF_PC + (KMAX / 4) * kGrpBytes;
 constexpr int kMaxQ = 8;                // distance accumulator column groups (>= KMAX / QW)
 constexpr int kNumBars = 2 * XS + 2 * AS + BS + 2 * kMaxQ + 2 * OS + 1;
 constexpr int OFF_MISC = OFF_BAR + kNumBars * 8;    // tmem slot, Cinf bits, C2 bits
-constexpr int kSmemTC = OFF_MISC + 16 + 1024;       // + alignment slack
+constexpr int OFF_EQ = OFF_MISC + 16;               // float2 [BS][TM]: the point's E and Q (1 + 2^-17) + 2E
+constexpr int kSmemTC = OFF_EQ + BS * TM * 8 + 1024;  // + alignment slack
 static_assert(OFF_AB % 1024 == 0 && OFF_BD % 1024 == 0 && OFF_OH % 1024 == 0 && OFF_X % 1024 == 0, "align");
 static_assert(kSmemTC <= 227 * 1024, "smem");
 
@@ -390,6 +391,8 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
         // ---- converters: point row r
         const int r = tid - 64;
         const float scale = (float)(1 << shift);
+        const float Cinf = __uint_as_float(misc[1]);
+        const float C2 = __uint_as_float(misc[2]);
         int bad = 0;
         for (int64_t i = 0; i < nt; ++i) {
             const int s = (int)(i % XS), a = (int)(i % AS);
@@ -433,6 +436,15 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
                 for (int b = 0; b < 4; ++b)
                     sts_u8(base[4 * (j & 1) + b] + (uint32_t)((4 * j + b) * 128), u >> (8 * b));
             }
+            {  // the filter bound's per-point terms, for the epilogue (header: E, Dhat)
+                float L1 = 0.f, Q = 0.f;
+#pragma unroll
+                for (int j = 0; j < 16; ++j) { L1 += fabsf(xv[j]); Q = fmaf(xv[j], xv[j], Q); }
+                const float E = (0x1p-11f * (L1 * Cinf + C2)) * 1.001f + 0x1p-100f;
+                const float Qa = Q * (1.f + 0x1p-17f) + 2.f * E;
+                asm volatile("st.shared.v2.f32 [%0], {%1, %2};" ::"r"(sbase + OFF_EQ + (bs * TM + r) * 8), "f"(E), "f"(Qa)
+                             : "memory");
+            }
             fence_async_smem();
             mbar_arrive(&afull[a]);
         }
@@ -441,8 +453,6 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
         // ---- epilogue: point row r = TMEM lane
         const int q = warp & 3;
         const int r = q * 32 + lane;
-        const float Cinf = __uint_as_float(misc[1]);
-        const float C2 = __uint_as_float(misc[2]);
         int32_t pend[OS];
 #pragma unroll
         for (int o = 0; o < OS; ++o) pend[o] = -1;
@@ -498,11 +508,10 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
                 vm[u] = max3(max3(gm[8 * u], gm[8 * u + 1], gm[8 * u + 2]), max3(gm[8 * u + 3], gm[8 * u + 4], gm[8 * u + 5]),
                              fmaxf(gm[8 * u + 6], gm[8 * u + 7]));
             const float vmax = max3(max3(vm[0], vm[1], vm[2]), max3(vm[3], vm[4], vm[5]), fmaxf(vm[6], vm[7]));
-            float L1 = 0.f, Q = 0.f;
-#pragma unroll
-            for (int j = 0; j < 16; ++j) { L1 += fabsf(xv[j]); Q = fmaf(xv[j], xv[j], Q); }
-            const float E = (0x1p-11f * (L1 * Cinf + C2)) * 1.001f + 0x1p-100f;
-            const float Dhat = fmaxf(Q * (1.f + 0x1p-17f) - 2.f * vmax + 2.f * E, 0.f);
+            float E, Qa;  // from the converter (stage i % BS is recycled only after this tile's reduction)
+            asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(E), "=f"(Qa)
+                         : "r"(sbase + OFF_EQ + ((uint32_t)(i % BS) * TM + r) * 8) : "memory");
+            const float Dhat = fmaxf(Qa - 2.f * vmax, 0.f);
             const float T = (2.f * E + 0x1p-16f * Dhat) * 1.001f;
             // candidate group <=> its maximum >= vmax - T <=> > thr (next float below vmax - T);
             // the sign bits of thr - gm are funnel-shifted into masks (bit 31 - g <-> group g)
