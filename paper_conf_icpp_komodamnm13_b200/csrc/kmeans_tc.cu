@@ -200,6 +200,11 @@ __device__ __forceinline__ uint64_t add2(uint64_t a, uint64_t b) {
     asm("add.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
     return d;
 }
+__device__ __forceinline__ uint64_t sub2(uint64_t a, uint64_t b) {
+    uint64_t d;
+    asm("sub.rn.f32x2 %0, %1, %2;" : "=l"(d) : "l"(a), "l"(b));
+    return d;
+}
 __device__ __forceinline__ uint64_t fma2(uint64_t a, uint64_t b, uint64_t c) {
     uint64_t d;
     asm("fma.rn.f32x2 %0, %1, %2, %3;" : "=l"(d) : "l"(a), "l"(b), "l"(c));
@@ -517,10 +522,16 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             // the sign bits of thr - gm are funnel-shifted into masks (bit 31 - g <-> group g)
             const float thr = next_below(vmax - T);
             uint32_t mk0 = 0, mk1 = 0;
+            const uint64_t thr2 = pk2(thr, thr);
 #pragma unroll
-            for (int g = 0; g < 32; ++g) {
-                mk0 = __funnelshift_l(__float_as_uint(thr - gm[g]), mk0, 1);
-                mk1 = __funnelshift_l(__float_as_uint(thr - gm[32 + g]), mk1, 1);
+            for (int g = 0; g < 32; g += 2) {  // packed: two groups per FADD2 (each lane rounds alone)
+                float d0, d1, d2, d3;
+                upk2(sub2(thr2, pk2(gm[g], gm[g + 1])), d0, d1);
+                upk2(sub2(thr2, pk2(gm[32 + g], gm[32 + g + 1])), d2, d3);
+                mk0 = __funnelshift_l(__float_as_uint(d0), mk0, 1);
+                mk1 = __funnelshift_l(__float_as_uint(d2), mk1, 1);
+                mk0 = __funnelshift_l(__float_as_uint(d1), mk0, 1);
+                mk1 = __funnelshift_l(__float_as_uint(d3), mk1, 1);
             }
             // exact re-check of the candidate groups in ascending centroid order (strict <)
             float bd = __int_as_float(0x7f800000);
