@@ -9,7 +9,8 @@
 //     A = [x0 | x0 | x1 | 1 1 1], B = [c0 | c1 | c0 | h0 h1 h2] (bf16 pieces: x = x0 + x1 + e with
 //     |e| <= 2^-16 |x|, -|c|^2/2 = h0 + h1 + h2), four tcgen05.mma.kind::f16 (K = 64) give
 //     v = x0.c0 + x0.c1 + x1.c0 - |c|^2/2 in TMEM, fp32, one 128-column half of the centroids per
-//     accumulator (two accumulators: the epilogue of one half overlaps the MMAs of the next);
+//     accumulator; each half is handed back to the MMA warp as soon as the epilogue has read it,
+//     so the next tile's MMAs of that half overlap the epilogue's remaining work;
 //   * reductiontoarray: sums[c][(j, b)] = sum_p onehot[c][p] * byte_b(x[p][j] * 2^shift + 2^31) and
 //     counts[c] = sum_p onehot[c][p] * 1 — tcgen05.mma.kind::i8 (u8 x u8 -> s32, exact) with
 //     A = the one-hot assignment matrix [128 clusters][128 points] and B = the points' fixed-point
@@ -23,17 +24,20 @@
 //   T = 2E + 2^-16 Dhat, Dhat = Q (1 + 2^-17) - 2 vmax + 2E >= D(p, c^) (c^ = argmax v).
 // A non-candidate c has V(c^) - V(c) > 2^-16 Dhat, so D(c) - D(c^) > 2^-15 D(c^) >= eps (D(c) +
 // D(c^)) with the fmaf chain's relative error eps <= 18 * 2^-24 (non-negative terms): D_f(c) >
-// D_f(c^), it can neither win nor tie. Each 128-column half uses its own maximum (a smaller vmax
-// only enlarges T: the candidate set is a superset). Inputs are on the 2^-shift grid (W4).
+// D_f(c^), it can neither win nor tie. Inputs are on the 2^-shift grid (W4). CPU pins of this
+// reading: tests/test_kmeans_filter_bound.py.
 //
 // Warp roles (one CTA per SM, persistent over 128-point tiles):
-//   w0 producer: cp.async.bulk of the tile's fp32 rows (8 KiB) into an mbarrier ring;
+//   w0 producer: TMA load (64-byte swizzle) of the tile's fp32 rows (8 KiB) into an mbarrier ring;
 //   w1 MMA issuer (one thread): distance MMAs of tile i, then the reduction MMAs of tile i-1;
 //   w2-5 converters (one point per thread): bf16 pieces of x into the distance A operand, the
-//        fixed-point bytes into the reduction B operand, the 2^-shift grid check;
-//   w6-9 epilogue (one point per thread = TMEM lane): per half, pass 1 = 32-column maxima
-//        (3-input FMNMX), pass 2 = candidate masks of the columns >= threshold (sign bits
-//        funnel-shifted into a mask) and exact re-checks; member[p]; the point's one-hot byte.
+//        fixed-point bytes into the reduction B operand, the 2^-shift grid check, the point's
+//        bound terms E and Q(1 + 2^-17) + 2E for the epilogue;
+//   w6-9 epilogue (one point per thread = TMEM lane): pass 1 = maxima of 4-column groups (3-input
+//        FMNMX) over all k columns, then a candidate-group mask (sign bits of thr - max, packed
+//        FSUB2, funnel-shifted), the exact re-check of the candidate groups (packed FADD2 / FFMA2,
+//        each lane rounding like the scalar op), member[p] and the point's one-hot byte.
+// Same-box A/B measurements of the alternatives tried: profiles/r01/kmeans_tc.log.
 #include <cuda_bf16.h>
 
 #include <cstdlib>
