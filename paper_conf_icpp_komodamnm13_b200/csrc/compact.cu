@@ -395,7 +395,26 @@ write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const in
         }
         consumers_sync();
         T* tile_payload = payload + r.off_el;
-        if (r.dense) {
+        // the push-only case (nothing packed): replica by replica, a per-tile base pointer and
+        // 32-bit offsets instead of a 64-bit global index and a pointer-list loop per element (the
+        // stage is re-read from shared memory for each replica)
+        if (r.dense && !keep && push.n >= 1) {
+            for (int q = 0; q < NSC; ++q, ++seq) {
+                const int st = seq % NST;
+                dev::mbar_wait(&full[st], (seq / NST) & 1);
+                const T* V = reinterpret_cast<const T*>(ring + st * kStageBytes);
+                for (int d = 0; d < push.n; ++d) {
+                    T* const pd = static_cast<T*>(push.p[d]) + w0 * 32;
+#pragma unroll
+                    for (int j = warp; j < SCW; j += kConsumers / 32) {
+                        const int i = q * SCW + j;
+                        if ((W[kPad + i] >> lane) & 1u) pd[i * 32 + lane] = V[j * 32 + lane];
+                    }
+                }
+                __syncwarp();
+                if (lane == 0) dev::mbar_arrive(&empty[st]);
+            }
+        } else if (r.dense) {
             for (int q = 0; q < NSC; ++q, ++seq) {
                 const int st = seq % NST;
                 dev::mbar_wait(&full[st], (seq / NST) & 1);
