@@ -386,7 +386,8 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
                                            ((uint32_t)(TM >> 4) << 24);
 #pragma unroll
                     for (int k = 0; k < 4; ++k)
-                        mma_f16(tmem + (uint32_t)(QW * g), sdesc_sw128(sAD + a * kADBytes + k * 32),
+                        // A slices x0, x0, x1, 1 (slice 0 read twice) against B slices c0, c1, c0, h
+                        mma_f16(tmem + (uint32_t)(QW * g), sdesc_sw128(sAD + a * kADBytes + (k == 1 ? 0 : k * 32)),
                                 sdesc_sw128(sBD + g * QW * 128 + k * 32), idesc, k ? 1u : 0u);
                     tc_commit(&dfull[g]);
                 }
@@ -420,10 +421,9 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             split8(xv, h0, l0);
             split8(xv + 8, h1, l1);
             const uint32_t ad = sAD + a * kADBytes;
+            // slices 0 = x0, 2 = x1 (3 = the constant ones); the MMA reads slice 0 twice
             sts_v4(ad + sw_off(r, 0), h0);
             sts_v4(ad + sw_off(r, 16), h1);
-            sts_v4(ad + sw_off(r, 32), h0);
-            sts_v4(ad + sw_off(r, 48), h1);
             sts_v4(ad + sw_off(r, 64), l0);
             sts_v4(ad + sw_off(r, 80), l1);
             // fixed point x * 2^shift, biased to unsigned: u = v + 2^31; byte b of dim j -> row 4j + b
