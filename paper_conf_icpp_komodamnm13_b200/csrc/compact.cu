@@ -69,7 +69,20 @@ count_k(const uint32_t* __restrict__ l1, const uint32_t* __restrict__ l2, int64_
     }
     int64_t ns = 0, ne = 0, nel = 0;
     const int64_t ws = w0 + (int64_t)threadIdx.x * kWordsPerThread;
-    if (ws < w1) {
+    if (ws + kWordsPerThread <= w1 && (reinterpret_cast<uintptr_t>(l1 + ws) & 15) == 0) {
+        // full group: two 128-bit loads (coalesced across the warp) and the two neighbour words
+        static_assert(kWordsPerThread == 8, "two uint4 per thread");
+        const uint4 a = *reinterpret_cast<const uint4*>(l1 + ws);
+        const uint4 b = *reinterpret_cast<const uint4*>(l1 + ws + 4);
+        const uint32_t wv[10] = {ws >= 1 ? l1[ws - 1] : 0u, a.x, a.y, a.z, a.w, b.x, b.y, b.z, b.w,
+                                 ws + 8 < nwords ? l1[ws + 8] : 0u};
+#pragma unroll
+        for (int j = 1; j <= 8; ++j) {
+            ns += __popc(start_mask(wv[j], wv[j - 1]));
+            ne += __popc(end_mask(wv[j], wv[j + 1]));
+            nel += __popc(wv[j]);
+        }
+    } else if (ws < w1) {
         uint32_t prev = ws >= 1 ? l1[ws - 1] : 0u;  // count pass clears nothing: neighbours are stable
         uint32_t cur = l1[ws];
 #pragma unroll
