@@ -311,7 +311,10 @@ def main():
         line = {"impl": "reference", "metric": METRIC, "value": round(rate, 1), "unit": UNIT, "n_gpus": args.gpus,
                 "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "vs_baseline": None,
                 "dtype": "f32", "data": "synthetic",
-                "config": {"workload": f"C2: 2D 5-point Jacobi {args.size}x{args.size} fp32 (bounded sample on host cores)"},
+                # the accmg arm's workload; the bounded host sample is described in cpu_baseline.sample
+                "config": {"workload": f"C2: 2D 5-point Jacobi {args.size}x{args.size} fp32, row-block partition, "
+                                       + ("undeclared (dirty-bit tracking)" if args.undeclared else "declared halo h=1"),
+                           "n": args.size, "partitions": 1, "sweeps_per_step": 1, "parallelism": "oracle on host cores"},
                 "cpu_baseline": {"value": round(rate, 1), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
                 "e2e": {"value": round(rate, 1), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
         print(json.dumps(line), flush=True)
