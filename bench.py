@@ -118,9 +118,11 @@ def ncu_traffic(kernel_key: str):
 
 
 # ---- CPU oracle legs -----------------------------------------------------------------------------
-def oracle_jacobi_rate(n: int, target_s: float = 10.0):
+def oracle_jacobi_rate(n: int, target_s: float = 10.0, steps: int = 0, warmup: int = 0):
     """The oracle (oracle/oracle.c, as it stands) on a bounded sample of the C2 workload: full-width
-    row bands of the n x n field, repeated sweeps for ~target_s seconds, on all host cores."""
+    row bands of the n x n field, repeated sweeps for ~target_s seconds (or, with steps > 0, warmup
+    untimed sweeps then exactly `steps` timed sweeps: one step = one sweep of the band), on all
+    host cores."""
     import gen
     import oracle
     cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
@@ -130,12 +132,14 @@ def oracle_jacobi_rate(n: int, target_s: float = 10.0):
     # the oracle sweeps a square array; use a (rows+2) x n band embedded as its own field:
     # its interior rows are exactly C2 rows 1..rows (same arithmetic per point)
     out = band.copy()
+    for _ in range(warmup):
+        oracle.jacobi_sweep_rect(band, out, nthreads=cores)
     t0 = time.perf_counter()
     reps = 0
     while True:
         oracle.jacobi_sweep_rect(band, out, nthreads=cores)
         reps += 1
-        if time.perf_counter() - t0 > target_s:
+        if (steps > 0 and reps >= steps) or (steps <= 0 and time.perf_counter() - t0 > target_s):
             break
     dt = time.perf_counter() - t0
     upd = reps * rows * (n - 2)
@@ -307,7 +311,7 @@ def main():
     if args.impl == "reference":
         if rank != 0:
             return
-        rate, cores, sample = oracle_jacobi_rate(args.size, target_s=2.0)
+        rate, cores, sample = oracle_jacobi_rate(args.size, steps=max(args.steps, 1), warmup=args.warmup)
         line = {"impl": "reference", "metric": METRIC, "value": round(rate, 1), "unit": UNIT, "n_gpus": args.gpus,
                 "steps": args.steps, "warmup": args.warmup, "higher_is_better": True, "vs_baseline": None,
                 "dtype": "f32", "data": "synthetic",
