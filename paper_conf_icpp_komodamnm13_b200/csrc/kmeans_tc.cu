@@ -257,6 +257,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t ntiles = (p1 - p0 + TM - 1) / TM;
     const int64_t nt = blockIdx.x < ntiles ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
+    const uint32_t nt32 = (uint32_t)nt;
     const int nh = (npad + 127) / 128;  // 128-centroid halves (reduction)
     constexpr int NQ = KMAX / QW;       // distance accumulator groups
     const int nq = (npad + QW - 1) / QW;
@@ -350,8 +351,8 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
     if (warp == 0) {
         // ---- producer
         if (lane == 0) {
-            for (int64_t i = 0; i < nt; ++i) {
-                const int64_t t = blockIdx.x + i * gridDim.x;
+            for (uint32_t i = 0; i < nt32; ++i) {
+                const uint32_t t = blockIdx.x + i * gridDim.x;
                 const int s = (int)(i % XS);
                 mbar_wait_sleep(&xempty[s], (uint32_t)((i / XS) & 1) ^ 1u);
                 mbar_expect_tx(&xfull[s], kXBytes);  // rows past the end are zero-filled
@@ -362,7 +363,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
         // ---- MMA issuer (one thread)
         if (lane == 0) {
             const uint32_t idesc_sum = (2u << 4) | ((uint32_t)(kRows >> 3) << 17) | ((uint32_t)(TM >> 4) << 24);
-            auto reduce = [&](int64_t j) {
+            auto reduce = [&](uint32_t j) {
                 const int o = (int)(j % OS);
                 mbar_wait(&ofull[o], (uint32_t)((j / OS) & 1));
                 tc_fence_after();
@@ -375,7 +376,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
                 tc_commit(&oempty[o]);
                 tc_commit(&bempty[j % BS]);
             };
-            for (int64_t i = 0; i < nt; ++i) {
+            for (uint32_t i = 0; i < nt32; ++i) {
                 const int a = (int)(i % AS);
                 mbar_wait(&afull[a], (uint32_t)((i / AS) & 1));
                 for (int g = 0; g < nq; ++g) {
@@ -394,7 +395,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
                 tc_commit(&aempty[a]);
                 if (i >= 1) reduce(i - 1);
             }
-            if (nt > 0) reduce(nt - 1);
+            if (nt32 > 0) reduce(nt32 - 1);
             tc_commit(sdone);
         }
     } else if (warp < 6) {
@@ -404,7 +405,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
         const float Cinf = __uint_as_float(misc[1]);
         const float C2 = __uint_as_float(misc[2]);
         int bad = 0;
-        for (int64_t i = 0; i < nt; ++i) {
+        for (uint32_t i = 0; i < nt32; ++i) {
             const int s = (int)(i % XS), a = (int)(i % AS);
             mbar_wait(&xfull[s], (uint32_t)((i / XS) & 1));
             float xv[16];
@@ -465,11 +466,12 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
         int32_t pend[OS];
 #pragma unroll
         for (int o = 0; o < OS; ++o) pend[o] = -1;
-        for (int64_t i = 0; i < nt; ++i) {
-            const int64_t t = blockIdx.x + i * gridDim.x;
+        for (uint32_t i = 0; i < nt32; ++i) {
+            const uint32_t t = blockIdx.x + i * gridDim.x;
             const int s = (int)(i % XS);
-            const int64_t p = p0 + t * TM + r;
-            const bool valid = p < p1;
+            const uint32_t pr = t * TM + (uint32_t)r;  // row within the partition (< 2^31)
+            const int64_t p = p0 + pr;
+            const bool valid = pr < (uint32_t)(p1 - p0);
             mbar_wait(&xfull[s], (uint32_t)((i / XS) & 1));
             float xv[16];
 #pragma unroll
