@@ -90,3 +90,20 @@ def test_masked_writes_two_processes(tmp_path):
     _launch(2, 2, "masked", tmp_path)
     for r in range(2):
         assert np.array_equal(np.load(tmp_path / f"rank{r}_out.npy"), exp)
+
+
+@pytest.mark.parametrize("work", ["jacobi_decl", "jacobi_undecl"])
+def test_jacobi_three_processes(tmp_path, work):
+    """Three ranks (partitions 0-2 in three CUDA contexts): the middle rank pushes halos / dirty
+    elements to two IPC-mapped peers per loop; every rank bit-exact."""
+    N, S = 300, 6  # tests/mp_worker.py runs 6 sweeps of the 300 x 300 field
+    A0 = gen.jacobi_field(5, N)
+    oA, oB = A0.copy(), A0.copy()
+    oracle.jacobi_run(oA, oB, S)
+    stats = _launch(3, 1, work, tmp_path)
+    for r in range(3):
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_A.npy"), oA)
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_B.npy"), oB)
+    if work == "jacobi_undecl":
+        P = 3
+        assert sum(s["bytes_interpartition"] for s in stats) == S * (P - 1) * (16 * P + 16 * (N - 2) + 4 * (N - 2) ** 2)
