@@ -77,7 +77,8 @@ def test_scatter_two_processes(tmp_path):
     assert sum(s["write_misses"] for s in stats) == int(miss.sum())
 
 
-def test_masked_writes_two_processes(tmp_path):
+@pytest.mark.parametrize("world,V", [(2, 2), (3, 1), (3, 2)])
+def test_masked_writes_multi_process(tmp_path, world, V):
     """Irregular undeclared writes (isolated bits, runs across tiles and chunks) across processes:
     each rank's compaction pass pushes its dirty elements into the peer's replicas through the IPC
     mappings; every rank ends bit-exact. (NCCL cannot put two ranks on one GPU; its packed-buffer
@@ -87,8 +88,8 @@ def test_masked_writes_two_processes(tmp_path):
     exp = np.full(n, -1.0, dtype=np.float32)
     for seed, dens, run in ((22, 0.5, 1), (23, 0.3, 70001), (24, 0.9, 40)):
         oracle.masked_write(src, gen.write_mask(seed, n, dens, run), exp)
-    _launch(2, 2, "masked", tmp_path)
-    for r in range(2):
+    _launch(world, V, "masked", tmp_path)
+    for r in range(world):
         assert np.array_equal(np.load(tmp_path / f"rank{r}_out.npy"), exp)
 
 
