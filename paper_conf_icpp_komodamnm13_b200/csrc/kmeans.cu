@@ -94,7 +94,6 @@ assign_d(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __
     const float scale = (float)(1 << shift);
     const int64_t n = p1 - p0;
     const int64_t ngroups = (n + PPT - 1) / PPT;
-    const float4* nc4 = reinterpret_cast<const float4*>(s_nc);
     for (int64_t grp = (int64_t)blockIdx.x * NT + threadIdx.x; grp < ngroups; grp += (int64_t)gridDim.x * NT) {
         const int64_t pb = p0 + grp * PPT;
         uint64_t xp[NP][D];  // pair h = (x[pb+2h][j], x[pb+2h+1][j])
