@@ -126,7 +126,7 @@ def oracle_jacobi_rate(n: int, target_s: float = 10.0, steps: int = 0, warmup: i
     import gen
     import oracle
     cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
-    rows = 8190  # 8192 x n band: 1 GiB per array, far larger than any host cache
+    rows = min(8190, n - 2)  # 8192 x n band at C2: 1 GiB per array, far larger than any host cache
     band = gen.jacobi_field(2, n, 0, rows + 2)  # a band of the real field (rows 0..rows+1)
     band = np.ascontiguousarray(band)
     # the oracle sweeps a square array; use a (rows+2) x n band embedded as its own field:
