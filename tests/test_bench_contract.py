@@ -24,3 +24,28 @@ def test_reference_arm_json_line():
     assert d["cpu_baseline"]["kind"] == "oracle" and d["cpu_baseline"]["cores"] >= 1
     assert d["e2e"]["h2d_bytes_per_step"] == 0 and d["e2e"]["unit"] == d["unit"]
     assert "3 sweeps" in d["cpu_baseline"]["sample"]
+
+
+import pytest  # noqa: E402
+
+
+@pytest.mark.gpu
+def test_accmg_arm_json_line():
+    """The accmg arm at a small field: one JSON line with roofline, e2e, clocks, launches."""
+    from tests.gpu_util import need_gpu
+    need_gpu()
+    out = subprocess.run([sys.executable, os.path.join(ROOT, "bench.py"), "--size", "4096", "--steps", "5",
+                          "--warmup", "3", "--e2e-steps", "1", "--e2e-sweeps", "4"], cwd=ROOT, capture_output=True,
+                         text=True, timeout=600)
+    assert out.returncode == 0, out.stderr[-2000:]
+    lines = [l for l in out.stdout.splitlines() if l.strip()]
+    assert len(lines) == 1
+    d = json.loads(lines[0])
+    for k in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better", "scaling",
+              "vs_baseline", "dtype", "data", "config", "roofline", "clocks", "e2e", "gpu_launches", "cpu_baseline"):
+        assert k in d, k
+    assert d["steps"] == 5 and d["warmup"] == 3 and d["gpu_launches"] >= 5
+    r = d["roofline"]
+    assert r["bound"] == "hbm" and r["unit"] == "GB/s" and 0 < r["frac"] < 1.1 and r["peak"] > 0
+    assert d["e2e"]["h2d_bytes_per_step"] > 0 and d["e2e"]["d2h_bytes_per_step"] > 0
+    assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
