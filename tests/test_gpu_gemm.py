@@ -75,3 +75,17 @@ def test_large_sampled_rows():
     rows = np.unique(np.concatenate([np.arange(0, M, 97), [M - 1, 1023, 1024, 2047, 2048, 3071, 3072]]))
     R = oracle.gemm_rows_f64(Ab, Bb, rows)
     assert np.array_equal(C[rows], R.astype(np.float32))
+
+
+@pytest.mark.skipif(bool(__import__("os").environ.get("ACCMG_GEMM_IMPL")), reason="already a per-impl run")
+def test_two_sm_variant_bitexact():
+    """ACCMG_GEMM_IMPL=2 (tcgen05.mma.cta_group::2 CTA pairs), read once per process: the GEMM
+    tests in a child process."""
+    import os
+    import subprocess
+    import sys
+    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-p", "no:cacheprovider", "tests/test_gpu_gemm.py",
+                        "-k", "not two_sm_variant"], cwd=root, env=dict(os.environ, ACCMG_GEMM_IMPL="2"),
+                       capture_output=True, text=True, timeout=900)
+    assert r.returncode == 0, r.stdout[-3000:]
