@@ -486,7 +486,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
 #pragma unroll
             for (int qg = 0; qg < NQ; ++qg) {
                 if (qg < nq) {
-                    mbar_wait(&dfull[qg], (uint32_t)(i & 1));
+                    mbar_wait_sleep(&dfull[qg], (uint32_t)(i & 1));
                     tc_fence_after();
                 }
                 const int ncq = qg < nq ? (((npad - QW * qg) < QW ? (npad - QW * qg) : QW) / 32) : 0;
