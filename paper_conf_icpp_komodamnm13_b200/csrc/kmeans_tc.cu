@@ -365,7 +365,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             const uint32_t idesc_sum = (2u << 4) | ((uint32_t)(kRows >> 3) << 17) | ((uint32_t)(TM >> 4) << 24);
             auto reduce = [&](uint32_t j) {
                 const int o = (int)(j % OS);
-                mbar_wait(&ofull[o], (uint32_t)((j / OS) & 1));
+                mbar_wait_sleep(&ofull[o], (uint32_t)((j / OS) & 1));
                 tc_fence_after();
                 const uint32_t b = sAB + (uint32_t)(j % BS) * kABBytes;
                 for (int h = 0; h < nh; ++h)
@@ -378,9 +378,9 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             };
             for (uint32_t i = 0; i < nt32; ++i) {
                 const int a = (int)(i % AS);
-                mbar_wait(&afull[a], (uint32_t)((i / AS) & 1));
+                mbar_wait_sleep(&afull[a], (uint32_t)((i / AS) & 1));
                 for (int g = 0; g < nq; ++g) {
-                    mbar_wait(&dempty[g], (uint32_t)(i & 1) ^ 1u);
+                    mbar_wait_sleep(&dempty[g], (uint32_t)(i & 1) ^ 1u);
                     tc_fence_after();
                     const int wq = (npad - QW * g) < QW ? (npad - QW * g) : QW;
                     const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(wq >> 3) << 17) |
