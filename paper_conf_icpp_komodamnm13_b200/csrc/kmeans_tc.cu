@@ -407,7 +407,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
         int bad = 0;
         for (uint32_t i = 0; i < nt32; ++i) {
             const int s = (int)(i % XS), a = (int)(i % AS);
-            mbar_wait(&xfull[s], (uint32_t)((i / XS) & 1));
+            mbar_wait_sleep(&xfull[s], (uint32_t)((i / XS) & 1));
             float xv[16];
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
