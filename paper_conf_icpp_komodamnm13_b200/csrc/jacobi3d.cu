@@ -80,7 +80,7 @@ jacobi3d_tma(const __grid_constant__ CUtensorMap map, float* __restrict__ dst, i
     dev::mbar_wait(&bar[1], 0);
     for (int64_t i = ps; i < pe; ++i) {
         const int q = (int)(i - ps) + 2;  // plane i+1
-        dev::mbar_wait(&bar[q % kStages], (uint32_t)((q / kStages) & 1));
+        dev::mbar_wait_sleep(&bar[q % kStages], (uint32_t)((q / kStages) & 1));
         const float* P0 = tile[(q - 2) % kStages];
         const float* P1 = tile[(q - 1) % kStages];
         const float* P2 = tile[q % kStages];
