@@ -305,9 +305,27 @@ def run_e2e(args, A, WL, torch, stream, dist, ws, rank, local, declared):
                     "sync_to_host_owned of the result, max over ranks; per-rank bytes"}
 
 
+def free_port() -> int:
+    import socket
+    with socket.socket(socket.AF_INET, socket.SOCK_STREAM) as s:
+        s.bind(("127.0.0.1", 0))
+        return s.getsockname()[1]
+
+
+def self_launch(n: int) -> int:
+    """`python bench.py --gpus N` without torchrun: re-run this script as N ranks (one process per
+    GPU, rank r on device r % device_count) through torch.distributed.run on 127.0.0.1. Rank 0's
+    JSON line is the only stdout line; the exit code is torchrun's."""
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={n}",
+           "--master-addr", "127.0.0.1", "--master-port", str(free_port()), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.call(cmd)
+
+
 def main():
     args = parse()
     ws, rank, local = dist_env()
+    if args.impl == "accmg" and args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        sys.exit(self_launch(args.gpus))
     if args.impl == "reference":
         if rank != 0:
             return
@@ -325,7 +343,7 @@ def main():
         return
     out = run_accmg(args)
     if rank == 0:
-        if not args.no_cpu_baseline:
+        if not args.no_cpu_baseline and ws == 1:  # the host baseline is taken at N = 1 only
             rate, cores, sample = oracle_jacobi_rate(args.size, target_s=10.0)
             out["cpu_baseline"] = {"value": round(rate, 1), "unit": UNIT, "cores": cores, "kind": "oracle",
                                    "sample": sample}

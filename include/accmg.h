@@ -70,7 +70,8 @@ typedef struct accmg_config {
                                   (planning and byte accounting without any CUDA call; loop bodies
                                   are not executed) */
     int64_t dirty_chunk_bytes; /* second-level dirty-bit chunk (L135: "we experimentally choose 1MB");
-                                  bytes of array data per chunk bit; 0 = 1<<20; power of two >= 128 */
+                                  bytes of array data per chunk bit; 0 = 1<<20; a power of two >= 256
+                                  (ACCMG_EINVAL otherwise) */
     int32_t exchange_mode;     /* ACCMG_XCHG_* */
     int32_t debug_checks;      /* 1 = check declared-write disjointness (G14) and dirty-set
                                   disjointness (L62), keep per-loop bitmap snapshots for the
@@ -164,7 +165,9 @@ typedef struct accmg_access {
  *   partition's write window (L137 §IV.D.2); a miss appends (index, value) to the partition's
  *   system buffer, and after the kernel the buffered writes are completed in the owner's replica
  *   (the partition whose window holds the index) — L137, L163. Indices must be distinct (L62) and
- *   lie in some partition's window of dst.
+ *   lie in some partition's window of dst: a record whose index no window holds (negative, >= m,
+ *   or in a gap between windows) is dropped, and the next synchronising call (sync_to_host,
+ *   barrier, get_stats) returns ACCMG_EDATA.
  * ACCMG_BODY_TEST_SPARSE_WRITE: bounds ndim=1 rows [0,R); descs [in R (fp32 R*C), out W (fp32 R*C)];
  *   rows i with i % period == 0: out[i][j] = in[i][j] + 1.0f for all j (exercises L2 chunk skipping).
  * ACCMG_BODY_TEST_MASKED_WRITE: bounds ndim=1 [0,n); descs [in R (fp32 n), mask R (uint8 n),

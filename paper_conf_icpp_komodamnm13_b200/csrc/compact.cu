@@ -16,6 +16,7 @@
 // clears L1 as it goes). HBM-bound: per dirty element 1/8 B bitmap + esize read + esize written,
 // + 16 B per run.
 #include "kernels.h"
+#include "tma_host.h"
 #include "tma_dev.cuh"
 #include "track.cuh"
 
@@ -476,7 +477,8 @@ cudaError_t launch_write_pipe_st(uint32_t* l1, int64_t nwords, int64_t extent, i
                                  uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s, int keep) {
     auto kern = write_pipe_k<T, NST>;
     const size_t smem = (size_t)NST * kStageBytes;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int per_sm = 1;
+    cudaError_t e = kernel_prep(kern, kConsumers + 32, smem, &per_sm);
     if (e != cudaSuccess) return e;
     static int flat = -1;  // ACCMG_COMPACT_IMPL=2: gather path only (measurement)
     if (flat < 0) {
@@ -484,10 +486,7 @@ cudaError_t launch_write_pipe_st(uint32_t* l1, int64_t nwords, int64_t extent, i
         flat = (v && atoi(v) == 2) ? 1 : 0;
     }
     const int aligned = !flat && (reinterpret_cast<uintptr_t>(values) % 16) == 0;
-    int dev = 0, sms = 148, per_sm = 1;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, kConsumers + 32, smem);
+    const int sms = sm_count_cached();
     int64_t grid = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
     if (grid > ntiles) grid = ntiles;
     kern<<<(unsigned)grid, kConsumers + 32, smem, s>>>(l1, nwords, extent, tile_counts, tile_offs, tile_edges, ntiles,

@@ -417,15 +417,13 @@ gemm2_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ 
 
 bool make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t row_bytes, uint32_t box_in,
               uint32_t box_out) {
-    auto fn = tma_encode_fn();
-    if (!fn) return false;
     cuuint64_t dims[2] = {inner, outer};
     cuuint64_t strides[1] = {row_bytes};
     cuuint32_t box[2] = {box_in, box_out};
     cuuint32_t es[2] = {1, 1};
-    return fn(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
-              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
-              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) == CUDA_SUCCESS;
+    return tma_encode_tiled(m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
+                            CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                            CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
 }
 
 }  // namespace
@@ -455,7 +453,7 @@ cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M,
     if (impl == 2) {
         // CTA pairs: A map boxes are 128 rows (each CTA loads its half of the 256-row tile)
         const size_t smem = 1024 + (size_t)kStages2 * kStage2Bytes + 256;
-        cudaError_t e = cudaFuncSetAttribute(gemm2_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaError_t e = kernel_prep(gemm2_kernel, kThreads, smem);
         if (e != cudaSuccess) return e;
         const int64_t tiles = ((m1 - m0 + BM2 - 1) / BM2) * (N / BN2);
         int64_t pairs = sms / 2;
@@ -478,7 +476,7 @@ cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M,
         return cudaGetLastError();
     }
     const size_t smem = 1024 + (size_t)kStages * kStageBytes + 256;
-    cudaError_t e = cudaFuncSetAttribute(gemm_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = kernel_prep(gemm_kernel, kThreads, smem);
     if (e != cudaSuccess) return e;
     const int64_t tiles = ((m1 - m0 + BM - 1) / BM) * (N / BN);
     const int grid = (int)(tiles < sms ? tiles : sms);

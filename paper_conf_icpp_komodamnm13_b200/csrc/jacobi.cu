@@ -195,7 +195,9 @@ cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, i
         cudaError_t e = jacobi2d_tma(src, dst, rows, cols, r0, r1, c0, c1, src_lo, src_hi, t, s, launches, push);
         if (e != cudaErrorNotSupported) return e;  // shapes the TMA variant does not take fall through
     }
-    const bool vec4 = (cols % 4 == 0) && ((reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) % 16 == 0);
+    uintptr_t align = reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst);
+    for (int i = 0; i < push.n; ++i) align |= reinterpret_cast<uintptr_t>(push.dst[i]);  // pushed rows are stored alike
+    const bool vec4 = (cols % 4 == 0) && align % 16 == 0;
     cudaError_t e = vec4 ? launch_rows<4>(src, dst, rows, cols, r0, r1, c0, c1, t, push, s)
                          : launch_rows<1>(src, dst, rows, cols, r0, r1, c0, c1, t, push, s);
     if (launches) *launches += 1;

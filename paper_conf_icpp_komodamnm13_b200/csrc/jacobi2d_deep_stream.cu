@@ -262,11 +262,9 @@ cudaError_t launch_h(const CUtensorMap& map, float* dst, int64_t cols, int64_t r
     auto kern = t.l1 ? deep_stream_k<H, true> : deep_stream_k<H, false>;
     constexpr int kWarps = Cfg<H>::NW;
     const size_t smem = (size_t)kWarps * kStages * kStageBytes;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = kernel_prep(kern, kWarps * 32, smem);
     if (e != cudaSuccess) return e;
-    int dev = 0, nsm = 148;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
+    const int nsm = sm_count_cached();
     // segment length: items are equal, so time ~ waves x rows per item = ceil(items / resident
     // warps) x (seg + 2h); pick the segment count minimising that (short partitions — 4096 rows of
     // C2 at P = 8 — would otherwise run 1.3 waves of 512-row items)
@@ -301,8 +299,6 @@ cudaError_t jacobi2d_deep_stream(const float* src, float* dst, int64_t rows, int
         (reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) % 16 != 0)
         return cudaErrorNotSupported;
     if (r1 <= r0 || c1 <= c0) return cudaSuccess;
-    auto fn = tma_encode_fn();
-    if (!fn) return cudaErrorNotSupported;
     const int64_t row_lo = (src_lo + cols - 1) / cols, row_hi = src_hi / cols;
     if (row_lo > std::max<int64_t>(r0 - h, 0) || row_hi < std::min<int64_t>(r1 + h, rows)) return cudaErrorInvalidValue;
     const int hc = h <= 4 ? 4 : 8;
@@ -311,9 +307,9 @@ cudaError_t jacobi2d_deep_stream(const float* src, float* dst, int64_t rows, int
     cuuint64_t strides[1] = {(cuuint64_t)cols * 4};
     cuuint32_t box[2] = {(cuuint32_t)W, (cuuint32_t)RS};
     cuuint32_t es[2] = {1, 1};
-    if (fn(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(src) + row_lo * cols, dims, strides, box, es,
-           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    if (!tma_encode_tiled(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(src) + row_lo * cols, dims,
+                          strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                          CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE))
         return cudaErrorNotSupported;
     const int64_t cbase = (c0 / 4) * 4;
     const int TK = W - 2 * hc;

@@ -128,11 +128,9 @@ cudaError_t jacobi2d_tma(const float* src, float* dst, int64_t rows, int64_t col
                          const HaloPush& push) {
     (void)rows;
     if (r1 <= r0 || c1 <= c0) return cudaSuccess;
-    if (cols % 4 != 0 || (reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) % 16 != 0 ||
-        cols >= (1ll << 31))
-        return cudaErrorNotSupported;
-    auto fn = tma_encode_fn();
-    if (!fn) return cudaErrorNotSupported;
+    uintptr_t align = reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst);
+    for (int i = 0; i < push.n; ++i) align |= reinterpret_cast<uintptr_t>(push.dst[i]);  // 128-bit pushes too
+    if (cols % 4 != 0 || align % 16 != 0 || cols >= (1ll << 31)) return cudaErrorNotSupported;
     // the map covers only the whole rows of src's allocation (row coordinates relative to row_lo)
     const int64_t row_lo = (src_lo + cols - 1) / cols, row_hi = src_hi / cols;
     if (r0 - 1 < row_lo || r1 + 1 > row_hi) return cudaErrorInvalidValue;
@@ -141,22 +139,20 @@ cudaError_t jacobi2d_tma(const float* src, float* dst, int64_t rows, int64_t col
     cuuint64_t strides[1] = {(cuuint64_t)cols * 4};
     cuuint32_t box[2] = {BOXK, BOXR};
     cuuint32_t es[2] = {1, 1};
-    if (fn(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(src) + row_lo * cols, dims, strides, box, es,
-           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    if (!tma_encode_tiled(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(src) + row_lo * cols, dims,
+                          strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                          CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE))
         return cudaErrorNotSupported;
     const int64_t cbase = (c0 / 4) * 4;
     const size_t smem = (size_t)kStages * kStageFloats * 4;
     auto kern = t.l1 ? jacobi2d_tma_k<true> : jacobi2d_tma_k<false>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    int per_sm = 1;
+    cudaError_t e = kernel_prep(kern, 256, smem, &per_sm);
     if (e != cudaSuccess) return e;
     // rows per CTA (32 x tpc): the grid runs in waves of (resident CTAs per SM x SMs); pick tpc so
     // that waves x (rows + 2 halo rows) per CTA is smallest -- a 4095-row partition (C2 at P = 8)
     // runs 10 waves of 256-row CTAs with the last one 23 % full, but 15 full waves of 160 rows
-    int dev = 0, nsm = 148, per_sm = 1;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&nsm, cudaDevAttrMultiProcessorCount, dev);
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, 256, smem);
+    const int nsm = sm_count_cached();
     const int64_t strips = (c1 - cbase + TK - 1) / TK, slots = (int64_t)nsm * (per_sm > 0 ? per_sm : 1);
     int tpc = kMaxTiles;
     int64_t best = -1;

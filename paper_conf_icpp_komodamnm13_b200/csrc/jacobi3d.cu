@@ -137,7 +137,7 @@ cudaError_t launch3d(const CUtensorMap& map, float* dst, int64_t n1, int64_t n2,
               (unsigned)((i1 - i0 + SEG - 1) / SEG));
     const size_t smem = Geo<TJ, NS>::kSmem;
     auto kern = t.l1 ? jacobi3d_tma<true, TJ, SEG, NS> : jacobi3d_tma<false, TJ, SEG, NS>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    cudaError_t e = kernel_prep(kern, 256, smem);
     if (e != cudaSuccess) return e;
     kern<<<grid, 256, smem, s>>>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, kbase, plane_lo, t);
     if (launches) *launches += 1;
@@ -153,8 +153,6 @@ cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64
     if (n2 % 4 != 0 || (reinterpret_cast<uintptr_t>(src) | reinterpret_cast<uintptr_t>(dst)) % 16 != 0 ||
         n0 >= (1ll << 31) || n1 >= (1ll << 31) || n2 >= (1ll << 31))
         return cudaErrorNotSupported;
-    auto fn = tma_encode_fn();
-    if (!fn) return cudaErrorNotSupported;
     // the tensor map covers only the planes of src's allocation ([src_lo, src_hi) elements), so
     // the TMA unit never addresses memory outside it; plane coordinates are relative to plane_lo
     const int64_t pl = n1 * n2;
@@ -170,9 +168,9 @@ cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64
     }
     cuuint32_t box[3] = {BOXK, (cuuint32_t)((vbox == 1 || vbox == 3 || vbox == 6) ? 34 : 18), 1};
     cuuint32_t es[3] = {1, 1, 1};
-    if (fn(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(src) + plane_lo * pl, dims, strides, box, es,
-           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    if (!tma_encode_tiled(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(src) + plane_lo * pl, dims,
+                          strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                          CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE))
         return cudaErrorNotSupported;
     // tile variant (ACCMG_J3D_VARIANT): 0 = 16 rows x 32 planes, 4 stages; 1 = 32 x 32; 2 = 16 x 64;
     // 3 = 32 x 64; 4 / 5 = 16 x 32 with 6 / 8 stages; 6 = 32 x 32, 6 stages; 7 = 16 x 64, 6 stages.

@@ -104,9 +104,11 @@ cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M,
 cudaError_t scatter_body(const float* src, const int32_t* idx, float* dst, int64_t i0, int64_t i1, int64_t wlo,
                          int64_t whi, uint64_t* recs, int64_t* count, cudaStream_t s, int64_t* launches);
 // Completes buffered writes in the owners' replicas: record (e, v) goes to dsts.p[h] where h is
-// the window with bounds[h] <= e < bounds[h+1] (nb windows, ascending). count = device counter.
+// the window [bounds[h], his[h]) holding e (nb windows, ascending). count = device counter. A record
+// no window holds is dropped and sets *bad.
 cudaError_t apply_misses(const uint64_t* recs, const int64_t* count, int64_t cap, const PtrList& dsts,
-                         const int64_t* bounds_dev, int nb, int64_t* total, cudaStream_t s, int64_t* launches);
+                         const int64_t* bounds_dev, const int64_t* his_dev, int nb, int64_t* total, int* bad,
+                         cudaStream_t s, int64_t* launches);
 
 // ---- coherence: compaction of dirty runs, scatter into peer replicas -------------------------
 constexpr int kTileWords = 2048;   // bitmap words per compaction tile (65536 elements)

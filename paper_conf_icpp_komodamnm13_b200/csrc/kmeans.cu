@@ -19,6 +19,7 @@
 #include <cstdlib>
 
 #include "kernels.h"
+#include "tma_host.h"
 #include "track.cuh"
 
 namespace accmg {
@@ -287,10 +288,9 @@ cudaError_t launch_assign_c16(const float* x, const float* cen, int32_t* member,
     cudaError_t e = cudaMemcpyToSymbolAsync(c_cen, cen, (size_t)kc * 16 * sizeof(float), 0, cudaMemcpyDeviceToDevice, s);
     if (e != cudaSuccess) return e;
     const size_t smem = (size_t)kc * 16 * 8 + (size_t)kc * 8;
-    e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
     int per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem);
+    e = kernel_prep(kern, NT, smem, &per_sm);
+    if (e != cudaSuccess) return e;
     const int64_t groups = (p1 - p0 + 2 * NP - 1) / (2 * NP);
     int64_t blocks = (groups + NT - 1) / NT;
     const int64_t cap = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
@@ -305,13 +305,10 @@ cudaError_t launch_assign16(const float* x, const float* cen, int32_t* member, i
     auto kern = assign_d<16, NP, CU, NT, MINB>;
     const size_t smem = (size_t)kc * 16 * 8 + (size_t)kc * 8 + (size_t)kc * 16 * 4;
     if (smem > 200 * 1024) return cudaErrorNotSupported;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
-    if (e != cudaSuccess) return e;
     // all of the unified L1/shared capacity as shared memory, so several blocks fit per SM
-    e = cudaFuncSetAttribute(kern, cudaFuncAttributePreferredSharedMemoryCarveout, cudaSharedmemCarveoutMaxShared);
-    if (e != cudaSuccess) return e;
     int per_sm = 0;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, kern, NT, smem);
+    cudaError_t e = kernel_prep(kern, NT, smem, &per_sm, true);
+    if (e != cudaSuccess) return e;
     const int64_t groups = (p1 - p0 + 2 * NP - 1) / (2 * NP);
     int64_t blocks = (groups + NT - 1) / NT;
     const int64_t cap = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
@@ -489,7 +486,7 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
     } else {
         const size_t smem = (((size_t)kc * d * 4 + 15) / 16) * 16 + (size_t)kc * d * 8 + (size_t)kc * 8;
         if (smem > 200 * 1024) return cudaErrorNotSupported;
-        cudaError_t e = cudaFuncSetAttribute(assign_generic, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+        cudaError_t e = kernel_prep(assign_generic, kThreads, smem);
         if (e != cudaSuccess) return e;
         int64_t blocks = (p1 - p0 + kThreads - 1) / kThreads;
         if (blocks > (int64_t)sms * 4) blocks = (int64_t)sms * 4;

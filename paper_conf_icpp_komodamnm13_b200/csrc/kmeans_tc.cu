@@ -40,6 +40,7 @@
 // Same-box A/B measurements of the alternatives tried: profiles/r01/kmeans_tc.log.
 #include <cuda_bf16.h>
 
+#include <cstdio>
 #include <cstdlib>
 
 #include "kernels.h"
@@ -53,7 +54,9 @@ namespace {
 using dev::mbar_arrive;
 using dev::mbar_expect_tx;
 using dev::mbar_init;
+#ifndef KM_DEBUG_HANG
 using dev::mbar_wait;
+#endif
 using dev::smem_u32;
 
 constexpr int TM = 128;                 // points per tile (distance MMA M, reduction MMA K)
@@ -62,14 +65,22 @@ constexpr int XS = 4;                   // fp32 point-tile stages
 constexpr int AS = 2;                   // distance A operand stages (freed by the distance MMAs)
 constexpr int BS = 4;                   // reduction B operand stages (freed by the reduction MMAs)
 constexpr int OS = 2;                   // one-hot stages
-constexpr int kRows = 80;               // reduction B rows: 16 dims x 4 bytes, counts, 15 zero
+constexpr int kRows = 64;               // reduction B rows: 16 dims x 4 bytes (counts: shared atomics)
 constexpr int kXBytes = TM * 64;        // 8 KiB
 constexpr int kADBytes = TM * 128;      // 16 KiB
-constexpr int kABBytes = kRows * 128;   // 10 KiB
+constexpr int kABBytes = kRows * 128;   // 8 KiB
 constexpr int kOHBytes = KMAX * 128;    // 32 KiB (two 128-cluster halves)
-constexpr int kThreadsTC = 320;
+constexpr int QW = 128;                 // centroid columns per distance accumulator (one MMA N)
+constexpr int NDB = 3;                  // distance accumulators: a ring of three 128-column halves
+// warps (sub-partition = warp % 4): 0 producer, 2-5 converters, 6-13 epilogue (two sets of four:
+// warp % 4 is the TMEM lane quarter), 15 / 1 distance-MMA issuers (centroid halves 0 / 1), 14
+// reduction-MMA issuer. A tcgen05.mma holds back its issuing sub-partition's other warps while it
+// runs (scripts/km_trace.cu: the epilogue warp beside the MMA issuer lagged ~1000 cycles per tile),
+// so the three MMA streams sit on the three sub-partitions the producer does not use
+constexpr int kThreadsTC = 512;
+constexpr int kRedWarp = 14;
 constexpr int kTmemCols = 512;
-constexpr uint32_t kColSum = 256;       // reduction accumulators: half h at 256 + 80 h
+constexpr uint32_t kColSum = NDB * QW;  // reduction accumulators: cluster half h at 384 + 64 h
 
 constexpr int OFF_AD = 0;
 constexpr int OFF_AB = OFF_AD + AS * kADBytes;
@@ -82,12 +93,16 @@ constexpr int OFF_X = OFF_OH + OS * kOHBytes;
 constexpr int kGrpBytes = 272;
 constexpr int OFF_PC = OFF_X + XS * kXBytes;
 constexpr int OFF_BAR = OFF_PC + (KMAX / 4) * kGrpBytes;
-constexpr int kMaxQ = 8;                // distance accumulator column groups (>= KMAX / QW)
-constexpr int kNumBars = 2 * XS + 2 * AS + BS + 2 * kMaxQ + 2 * OS + 1;
+constexpr int kNumBars = 2 * XS + 2 * AS + BS + 2 * NDB + 2 * OS + 1;
 constexpr int OFF_MISC = OFF_BAR + kNumBars * 8;    // tmem slot, Cinf bits, C2 bits
 constexpr int OFF_EQ = OFF_MISC + 16;               // float2 [BS][TM]: the point's E and Q (1 + 2^-17) + 2E
-constexpr int kSmemTC = OFF_EQ + BS * TM * 8 + 1024;  // + alignment slack
+// epilogue half exchange, double-buffered by tile parity: maxima [2][2][TM], verdicts [2][2][TM];
+// half-1 winner of a re-check (d [TM], c [TM])
+constexpr int OFF_EX = OFF_EQ + BS * TM * 8;
+constexpr int OFF_CNT = OFF_EX + 10 * TM * 4;       // int32 [KMAX]: the CTA's cluster counts
+constexpr int kSmemTC = OFF_CNT + KMAX * 4 + 1024;  // + alignment slack
 static_assert(OFF_AB % 1024 == 0 && OFF_BD % 1024 == 0 && OFF_OH % 1024 == 0 && OFF_X % 1024 == 0, "align");
+static_assert(kColSum + 2 * kRows <= kTmemCols, "tmem");
 static_assert(kSmemTC <= 227 * 1024, "smem");
 
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
@@ -103,6 +118,27 @@ __device__ __forceinline__ void mma_f16(uint32_t d, uint64_t da, uint64_t db, ui
         "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
         "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
         "l"(da), "l"(db), "r"(idesc), "r"(acc)
+        : "memory");
+}
+// warp-collective forms: every lane executes them with the same operands, one elected lane issues
+__device__ __forceinline__ void mma_f16_elect(uint32_t d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p, e;\n\tsetp.ne.b32 p, %4, 0;\n\telect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
+        "l"(da), "l"(db), "r"(idesc), "r"(acc)
+        : "memory");
+}
+__device__ __forceinline__ void mma_i8_elect(uint32_t d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
+    asm volatile(
+        "{\n\t.reg .pred p, e;\n\tsetp.ne.b32 p, %4, 0;\n\telect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.mma.cta_group::1.kind::i8 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
+        "l"(da), "l"(db), "r"(idesc), "r"(acc)
+        : "memory");
+}
+__device__ __forceinline__ void tc_commit_elect(uint64_t* bar) {
+    asm volatile(
+        "{\n\t.reg .pred e;\n\telect.sync _|e, 0xffffffff;\n\t"
+        "@e tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];\n\t}" ::"r"(smem_u32(bar))
         : "memory");
 }
 __device__ __forceinline__ void mma_i8(uint32_t d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
@@ -128,6 +164,23 @@ __device__ __forceinline__ uint32_t sw_off(uint32_t m, uint32_t kbyte) {
 }
 // wait with a suspend-time hint: a warp that waits for a free stage sleeps instead of spinning on
 // issue slots the converter / epilogue warps of its SM sub-partition need
+#ifdef KM_DEBUG_HANG  // waits that report themselves and trap after ~2^26 polls (debug builds only)
+__device__ __forceinline__ void mbar_wait_dbg(uint64_t* bar, uint32_t parity, int line) {
+    for (uint32_t it = 0;; ++it) {
+        uint32_t ok;
+        asm volatile("{\n\t.reg .pred p;\n\tmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\tselp.u32 %0, 1, 0, p;\n\t}"
+                     : "=r"(ok) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+        if (ok) return;
+        if (it == (1u << 24)) {
+            printf("hang: block %d warp %d lane %d line %d bar %u parity %u\n", blockIdx.x, threadIdx.x / 32,
+                   threadIdx.x % 32, line, smem_u32(bar) & 0xFFFF, parity);
+            __trap();
+        }
+    }
+}
+#define mbar_wait_sleep(b, p) mbar_wait_dbg(b, p, __LINE__)
+#define mbar_wait(b, p) mbar_wait_dbg(b, p, __LINE__)
+#else
 __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) {
     asm volatile(
         "{\n\t.reg .pred p;\n"
@@ -137,6 +190,7 @@ __device__ __forceinline__ void mbar_wait_sleep(uint64_t* bar, uint32_t parity) 
         "r"(parity), "r"(20000u)
         : "memory");
 }
+#endif
 __device__ __forceinline__ void sts_u8(uint32_t addr, uint32_t v) {
     asm volatile("st.shared.u8 [%0], %1;" ::"r"(addr), "r"(v) : "memory");
 }
@@ -227,11 +281,46 @@ __device__ __forceinline__ float next_below(float a) {
     return __int_as_float(a > 0.f ? b - 1 : b + 1);
 }
 
-// QW: width (centroid columns) of each distance accumulator; each has its own full / empty
-// barriers, so the MMAs of the next tile refill a group as soon as the epilogue has read it
-template <int QW>
+#ifdef KM_PROGRESS  // per-warp progress in mapped host memory (scripts/km_hang.cu); debug builds only
+__device__ unsigned* g_prog;
+#define KPR(EV, T)                                                                                     \
+    do {                                                                                             \
+        if ((threadIdx.x & 31) == 0 && blockIdx.x < 4096)                                            \
+            *(volatile unsigned*)&g_prog[blockIdx.x * 16 + (threadIdx.x >> 5)] = ((EV) << 24) | (T);  \
+    } while (0)
+#else
+#define KPR(EV, T)
+#endif
+#ifndef KTR_EPI
+#define KTR_EPI 6  // epilogue warp whose events the trace records (its half-1 partner: KTR_EPI + 4)
+#endif
+#ifdef KM_TRACE  // per-role timeline of CTA 0 (scripts/km_trace.cu); compiled out of the product
+__device__ unsigned long long g_km_trace[64][32];
+#define KTR(W, EV)                                                                                   \
+    do {                                                                                             \
+        if (blockIdx.x == 0 && warp == (W) && lane == 0 && i >= 200 && i < 264)                      \
+            g_km_trace[i - 200][EV] = clock64();                                                     \
+    } while (0)
+#else
+#define KTR(W, EV)
+#endif
+
+constexpr int kProdWarp = 0, kMmaWarp = 15, kMmaWarp1 = 1;
+
+__device__ __forceinline__ void named_bar(uint32_t id, uint32_t n) {
+    // non-aligned form: a warp may arrive diverged (after data-dependent re-check loops)
+    __syncwarp();
+    asm volatile("barrier.sync %0, %1;" ::"r"(id), "r"(n) : "memory");
+}
+
+// Two epilogue warps per TMEM lane quarter, one per 128-centroid half: a single warp's tcgen05.ld
+// + wait::ld sustains ~32 B/cycle (scripts/tmem_bw.cu), so one warp would need ~1000 cycles per
+// tile for the 128 KiB of distances. The distance accumulators form a ring of three 128-column
+// buffers (half h of tile i in buffer (nq i + h) mod 3), so the MMAs of the next tile's first half
+// run while the epilogue still reads this tile's two halves.
 __global__ void __launch_bounds__(kThreadsTC, 1)
-assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ cen, int32_t* __restrict__ member,
+assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg, const float* __restrict__ cen,
+          int32_t* __restrict__ member,
           int64_t* __restrict__ sums, int64_t* __restrict__ counts, int64_t p0, int64_t p1, int kc, int npad,
           int shift, int* err) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
@@ -248,23 +337,23 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
     uint64_t* aempty = afull + AS;
     uint64_t* bempty = aempty + AS;
     uint64_t* dfull = bempty + BS;
-    uint64_t* dempty = dfull + kMaxQ;
-    uint64_t* ofull = dempty + kMaxQ;
+    uint64_t* dempty = dfull + NDB;
+    uint64_t* ofull = dempty + NDB;
     uint64_t* oempty = ofull + OS;
     uint64_t* sdone = oempty + OS;
     uint32_t* misc = reinterpret_cast<uint32_t*>(smem + OFF_MISC);  // [0] tmem, [1] Cinf bits, [2] C2 bits
 
+    constexpr int kThreads = kThreadsTC;
     const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
     const int64_t ntiles = (p1 - p0 + TM - 1) / TM;
     const int64_t nt = blockIdx.x < ntiles ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
     const uint32_t nt32 = (uint32_t)nt;
     const int nh = (npad + 127) / 128;  // 128-centroid halves (reduction)
-    constexpr int NQ = KMAX / QW;       // distance accumulator groups
-    const int nq = (npad + QW - 1) / QW;
+    const int nq = nh;                  // distance accumulator halves per tile
 
     // ---- setup: constant operand parts, centroids, bounds, barriers, TMEM
     if (tid == 0) { misc[1] = 0u; misc[2] = 0u; }
-    for (int i = tid; i < npad * 16; i += kThreadsTC) {
+    for (int i = tid; i < npad * 16; i += kThreads) {
         const int c = i >> 4, j = i & 15;
         const float v = c < kc ? -cen[i] : 0.f;
         asm volatile("st.shared.f32 [%0], %1;" ::"r"(sPC + (c >> 2) * kGrpBytes + ((c >> 1) & 1) * 128 + j * 8 +
@@ -272,33 +361,30 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
                      "f"(v)
                      : "memory");
     }
-    for (uint32_t i = tid; i < OS * kOHBytes / 16; i += kThreadsTC) sts_v4(sOH + i * 16, make_uint4(0, 0, 0, 0));
-    for (int i = tid; i < AS * TM; i += kThreadsTC) {  // distance A, slice 3 = [1 1 1 0 ...]
+    for (uint32_t i = tid; i < OS * kOHBytes / 16; i += kThreads) sts_v4(sOH + i * 16, make_uint4(0, 0, 0, 0));
+    for (int i = tid; i < AS * TM; i += kThreads) {  // distance A, slice 3 = [1 1 1 0 ...]
         const uint32_t base = sAD + (i / TM) * kADBytes, r = i % TM;
         sts_v4(base + sw_off(r, 96), make_uint4(0x3F803F80u, 0x00003F80u, 0, 0));
         sts_v4(base + sw_off(r, 112), make_uint4(0, 0, 0, 0));
     }
-    for (int i = tid; i < BS * 16 * 8; i += kThreadsTC) {  // reduction B rows 64 (= 1) and 65..79 (= 0)
-        const int a = i / 128, row = 64 + (i % 128) / 8, ch = i % 8;
-        const uint32_t v = row == 64 ? 0x01010101u : 0u;
-        sts_v4(sAB + a * kABBytes + row * 128 + ch * 16, make_uint4(v, v, v, v));
-    }
+    for (int i = tid; i < KMAX; i += kThreads) reinterpret_cast<int*>(smem + OFF_CNT)[i] = 0;
     if (tid == 0) {
-        for (int s = 0; s < XS; ++s) { mbar_init(&xfull[s], 1); mbar_init(&xempty[s], 256); }
-        for (int a = 0; a < AS; ++a) { mbar_init(&afull[a], 128); mbar_init(&aempty[a], 1); }
+        for (int s = 0; s < XS; ++s) { mbar_init(&xfull[s], 1); mbar_init(&xempty[s], 128); }  // the converters
+        for (int a = 0; a < AS; ++a) { mbar_init(&afull[a], 128); mbar_init(&aempty[a], nq); }  // nq issuers
         for (int b = 0; b < BS; ++b) mbar_init(&bempty[b], 1);
-        for (int b = 0; b < kMaxQ; ++b) { mbar_init(&dfull[b], 1); mbar_init(&dempty[b], 128); }
+        for (int b = 0; b < NDB; ++b) { mbar_init(&dfull[b], 1); mbar_init(&dempty[b], 128); }
         for (int o = 0; o < OS; ++o) { mbar_init(&ofull[o], 128); mbar_init(&oempty[o], 1); }
         mbar_init(sdone, 1);
         dev::mbar_fence_init();
     }
+    KPR(1, 0);
     if (warp == 1) {
         asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(misc)),
                      "r"(kTmemCols));
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     __syncthreads();
-    for (int n = tid; n < npad; n += kThreadsTC) {  // distance B rows [c0 | c1 | c0 | h0 h1 h2 0 ...]
+    for (int n = tid; n < npad; n += kThreads) {  // distance B rows [c0 | c1 | c0 | h0 h1 h2 0 ...]
         float c[16];
         float q = 0.f, m = 0.f;
 #pragma unroll
@@ -344,61 +430,87 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
     }
     fence_async_smem();  // operands written by generic-proxy stores are read by tcgen05.mma
     tc_fence_before();
+    KPR(2, 0);
     __syncthreads();
     tc_fence_after();
+    KPR(3, 0);
     const uint32_t tmem = misc[0];
 
-    if (warp == 0) {
+    if (warp == kProdWarp) {
         // ---- producer
         if (lane == 0) {
             for (uint32_t i = 0; i < nt32; ++i) {
                 const uint32_t t = blockIdx.x + i * gridDim.x;
                 const int s = (int)(i % XS);
                 mbar_wait_sleep(&xempty[s], (uint32_t)((i / XS) & 1) ^ 1u);
+                KTR(kProdWarp, 25);
+                KPR(4, i);
                 mbar_expect_tx(&xfull[s], kXBytes);  // rows past the end are zero-filled
                 dev::tma_load_2d(&xmap, &xfull[s], smem + OFF_X + s * kXBytes, 0, (int)(t * TM));
             }
         }
-    } else if (warp == 1) {
-        // ---- MMA issuer (one thread)
-        if (lane == 0) {
-            const uint32_t idesc_sum = (2u << 4) | ((uint32_t)(kRows >> 3) << 17) | ((uint32_t)(TM >> 4) << 24);
-            auto reduce = [&](uint32_t j) {
-                const int o = (int)(j % OS);
-                mbar_wait_sleep(&ofull[o], (uint32_t)((j / OS) & 1));
-                tc_fence_after();
-                const uint32_t b = sAB + (uint32_t)(j % BS) * kABBytes;
-                for (int h = 0; h < nh; ++h)
+    } else if (warp == kMmaWarp || warp == kMmaWarp1) {
+        // ---- distance-MMA issuers, one per 128-centroid half (tcgen05.mma occupies the issuing
+        // sub-partition while it runs, so the three MMA streams sit on three sub-partitions). The
+        // whole warp runs the loop and one elected lane issues each tcgen05 instruction;
+        // descriptors are the stage bases plus the 16-byte-unit offsets of the slices
+        const int h = warp == kMmaWarp ? 0 : 1;
+        const uint64_t dAD = sdesc_sw128(sAD), dBD = sdesc_sw128(sBD);
+        const int wq = (npad - QW * h) < QW ? (npad - QW * h) : QW;
+        const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(wq >> 3) << 17) |
+                               ((uint32_t)(TM >> 4) << 24);
+        const uint64_t bd = dBD + (uint64_t)((h * QW * 128) >> 4);
+        for (uint32_t i = 0; i < nt32 && h < nq; ++i) {
+            const int a = (int)(i % AS);
+            mbar_wait_sleep(&afull[a], (uint32_t)((i / AS) & 1));
+            KTR(kMmaWarp, 4);
+            KPR(5, i);
+            const uint64_t ad = dAD + (uint64_t)((a * kADBytes) >> 4);
+            const uint32_t u = (uint32_t)nq * i + (uint32_t)h, db = u % NDB;  // ring slot and its use count
+            mbar_wait_sleep(&dempty[db], ((u / NDB) & 1u) ^ 1u);
+            KTR(kMmaWarp, 5);
+            KTR(kMmaWarp1, 6);
+            KPR(6, i);
+            tc_fence_after();
 #pragma unroll
-                    for (int k = 0; k < 4; ++k)
-                        mma_i8(tmem + kColSum + 80u * h, sdesc_sw128(sOH + o * kOHBytes + h * 16384 + k * 32),
-                               sdesc_sw128(b + k * 32), idesc_sum, (j | k) ? 1u : 0u);
-                tc_commit(&oempty[o]);
-                tc_commit(&bempty[j % BS]);
-            };
-            for (uint32_t i = 0; i < nt32; ++i) {
-                const int a = (int)(i % AS);
-                mbar_wait_sleep(&afull[a], (uint32_t)((i / AS) & 1));
-                for (int g = 0; g < nq; ++g) {
-                    mbar_wait_sleep(&dempty[g], (uint32_t)(i & 1) ^ 1u);
-                    tc_fence_after();
-                    const int wq = (npad - QW * g) < QW ? (npad - QW * g) : QW;
-                    const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(wq >> 3) << 17) |
-                                           ((uint32_t)(TM >> 4) << 24);
-#pragma unroll
-                    for (int k = 0; k < 4; ++k)
-                        // A slices x0, x0, x1, 1 (slice 0 read twice) against B slices c0, c1, c0, h
-                        mma_f16(tmem + (uint32_t)(QW * g), sdesc_sw128(sAD + a * kADBytes + (k == 1 ? 0 : k * 32)),
-                                sdesc_sw128(sBD + g * QW * 128 + k * 32), idesc, k ? 1u : 0u);
-                    tc_commit(&dfull[g]);
-                }
-                tc_commit(&aempty[a]);
-                if (i >= 1) reduce(i - 1);
-            }
-            if (nt32 > 0) reduce(nt32 - 1);
-            tc_commit(sdone);
+            for (int k = 0; k < 4; ++k)
+                // A slices x0, x0, x1, 1 (slice 0 read twice) against B slices c0, c1, c0, h
+                mma_f16_elect(tmem + QW * db, ad + (uint64_t)((k == 1 ? 0 : k * 32) >> 4),
+                              bd + (uint64_t)((k * 32) >> 4), idesc, k ? 1u : 0u);
+            tc_commit_elect(&dfull[db]);
+            tc_commit_elect(&aempty[a]);
+            KPR(7, i);
+            KTR(kMmaWarp, 13);
+            KTR(kMmaWarp1, 14);
         }
-    } else if (warp < 6) {
+    } else if (warp == kRedWarp) {
+        // ---- reductiontoarray MMAs (u8 one-hot x byte planes -> s32), one tile behind the
+        // epilogue's one-hot bytes
+        const uint32_t idesc_sum = (2u << 4) | ((uint32_t)(kRows >> 3) << 17) | ((uint32_t)(TM >> 4) << 24);
+        const uint64_t dAB = sdesc_sw128(sAB), dOH = sdesc_sw128(sOH);
+        for (uint32_t j = 0; j < nt32; ++j) {
+            const int o = (int)(j % OS);
+            mbar_wait_sleep(&ofull[o], (uint32_t)((j / OS) & 1));
+            {
+                const uint32_t i = j + 1;
+                KTR(kRedWarp, 7);
+            }
+            KPR(8, j);
+            tc_fence_after();
+            const uint64_t b = dAB + (uint64_t)(((j % BS) * kABBytes) >> 4);
+            const uint64_t oh = dOH + (uint64_t)((o * kOHBytes) >> 4);
+            for (int h = 0; h < nh; ++h)
+#pragma unroll
+                for (int k = 0; k < 4; ++k)
+                    mma_i8_elect(tmem + kColSum + (uint32_t)(kRows * h), oh + (uint64_t)((h * 16384 + k * 32) >> 4),
+                                 b + (uint64_t)((k * 32) >> 4), idesc_sum, (j | k) ? 1u : 0u);
+            tc_commit_elect(&oempty[o]);
+            tc_commit_elect(&bempty[j % BS]);
+            KPR(9, j);
+        }
+        tc_commit_elect(sdone);
+        KPR(10, 0);
+    } else if (warp >= 2 && warp < 6) {
         // ---- converters: point row r
         const int r = tid - 64;
         const float scale = (float)(1 << shift);
@@ -408,16 +520,21 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
         for (uint32_t i = 0; i < nt32; ++i) {
             const int s = (int)(i % XS), a = (int)(i % AS);
             mbar_wait_sleep(&xfull[s], (uint32_t)((i / XS) & 1));
+            KTR(2, 0);
+            KPR(11, i);
             float xv[16];
 #pragma unroll
             for (int j = 0; j < 4; ++j) {
                 const float4 v = lds_f4(sX + s * kXBytes + r * 64 + ((j ^ ((r >> 1) & 3)) << 4));
                 xv[4 * j] = v.x; xv[4 * j + 1] = v.y; xv[4 * j + 2] = v.z; xv[4 * j + 3] = v.w;
             }
-            mbar_arrive(&xempty[s]);
             mbar_wait_sleep(&aempty[a], (uint32_t)((i / AS) & 1) ^ 1u);
+            KTR(2, 1);
+            KPR(12, i);
             const int bs = (int)(i % BS);
             mbar_wait_sleep(&bempty[bs], (uint32_t)((i / BS) & 1) ^ 1u);
+            KTR(2, 2);
+            KPR(13, i);
             uint4 h0, l0, h1, l1;
             split8(xv, h0, l0);
             split8(xv + 8, h1, l1);
@@ -427,6 +544,10 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             sts_v4(ad + sw_off(r, 16), h1);
             sts_v4(ad + sw_off(r, 64), l0);
             sts_v4(ad + sw_off(r, 80), l1);
+            // the stage is released only after instructions that consume the loaded values (the
+            // arrive alone does not wait for the shared-memory loads to return their data, and the
+            // producer refills the stage as soon as all converters have arrived)
+            mbar_arrive(&xempty[s]);
             // fixed point x * 2^shift, biased to unsigned: u = v + 2^31; byte b of dim j -> row 4j + b
             // row m = 4j + b has swizzle phase m & 7 = 4 (j & 1) + b: eight per-thread base addresses,
             // the row offset m * 128 is the store's immediate (st.shared.u8 keeps the low byte)
@@ -434,18 +555,22 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             uint32_t base[8];
 #pragma unroll
             for (int k = 0; k < 8; ++k) base[k] = ab + ((((uint32_t)r >> 4) ^ (uint32_t)k) << 4) + ((uint32_t)r & 15u);
+            // grid check without branches: v = x 2^shift must equal rint(v) (every float of magnitude
+            // >= 2^23 is an integer) and |v| < 2^31; the largest |v - rint(v)| and |v| of the point
+            // are tested once
+            float fr = 0.f, vm = 0.f;
 #pragma unroll
             for (int j = 0; j < 16; ++j) {
                 const float v = xv[j] * scale;  // exact: power-of-two scaling
-                const float av = fabsf(v);
-                const float m = copysignf(8388608.0f, v);
-                const bool ok = av < 2147483648.0f && (av >= 8388608.0f || __fsub_rn(__fadd_rn(v, m), m) == v);
-                bad |= !ok;
-                const uint32_t u = (uint32_t)__float2int_rn(v) ^ 0x80000000u;
+                const float rv = rintf(v);
+                fr = fmaxf(fr, fabsf(v - rv));  // exact difference (Sterbenz)
+                vm = fmaxf(vm, fabsf(v));
+                const uint32_t u = (uint32_t)__float2int_rn(rv) ^ 0x80000000u;
 #pragma unroll
                 for (int b = 0; b < 4; ++b)
                     sts_u8(base[4 * (j & 1) + b] + (uint32_t)((4 * j + b) * 128), u >> (8 * b));
             }
+            bad |= (fr != 0.f) | !(vm < 2147483648.0f);
             {  // the filter bound's per-point terms, for the epilogue (header: E, Dhat)
                 float L1 = 0.f, Q = 0.f;
 #pragma unroll
@@ -457,125 +582,230 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             }
             fence_async_smem();
             mbar_arrive(&afull[a]);
+            KTR(2, 3);
+            KPR(14, i);
         }
         if (bad) atomicOr(err, 1);
-    } else {
-        // ---- epilogue: point row r = TMEM lane
+    } else if (warp >= 6 && warp < 14) {
+        // ---- epilogue, orthogonal groupings: point row r = TMEM lane; warp set `half` reads the
+        // 128 columns of centroids [128 half, 128 half + 128). Local column l = 16 b + a: the
+        // b-groups (16 consecutive columns, 8 per half) and the a-groups (columns with the same
+        // l mod 16, 16 per half) partition the columns two ways and (a, b) names one column, so
+        // when exactly one a-group and one b-group reach the threshold the candidate set is that
+        // single column: the argmin is proved without any re-check (the common case for separated
+        // clusters). Otherwise every 4-column group of the product set (candidate b-groups x
+        // quarters holding candidate a-groups) is re-checked with the exact fmaf chain.
         const int q = warp & 3;
         const int r = q * 32 + lane;
+        const int half = (warp - 6) >> 2;
+        float* exv0 = reinterpret_cast<float*>(smem + OFF_EX);  // [parity][half][TM] half maxima
+        int* exs0 = reinterpret_cast<int*>(exv0 + 4 * TM);      // [parity][half][TM] local verdicts
+        float* exd = exv0 + 8 * TM;                              // [TM] half-1 winner distance (re-check)
+        int* exi = reinterpret_cast<int*>(exv0 + 9 * TM);        // [TM] half-1 winner index (re-check)
+        int* s_cnt = reinterpret_cast<int*>(smem + OFF_CNT);   // the CTA's cluster counts
         int32_t pend[OS];
 #pragma unroll
         for (int o = 0; o < OS; ++o) pend[o] = -1;
+        const bool have = half < nq;  // this half holds centroids
+        const int ncq = have ? (((npad - QW * half) < QW ? (npad - QW * half) : QW) / 32) : 0;
+        const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16);
         for (uint32_t i = 0; i < nt32; ++i) {
             const uint32_t t = blockIdx.x + i * gridDim.x;
             const int s = (int)(i % XS);
             const uint32_t pr = t * TM + (uint32_t)r;  // row within the partition (< 2^31)
             const int64_t p = p0 + pr;
             const bool valid = pr < (uint32_t)(p1 - p0);
-            mbar_wait(&xfull[s], (uint32_t)((i / XS) & 1));
-            float xv[16];
+            KTR(KTR_EPI, 9);
+            KTR(KTR_EPI + 4, 21);
+            KPR(15, i);
+            float am[16], bm[8];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
-                const float4 v = lds_f4(sX + s * kXBytes + r * 64 + ((j ^ ((r >> 1) & 3)) << 4));
-                xv[4 * j] = v.x; xv[4 * j + 1] = v.y; xv[4 * j + 2] = v.z; xv[4 * j + 3] = v.w;
-            }
-            mbar_arrive(&xempty[s]);
-            // pass 1 over the accumulator groups: maxima of the 4-column groups (64 registers); each
-            // accumulator goes back to the MMA warp as soon as it is read
-            float gm[64];
+            for (int a = 0; a < 16; ++a) am[a] = -0x1p120f;
 #pragma unroll
-            for (int qg = 0; qg < NQ; ++qg) {
-                if (qg < nq) {
-                    mbar_wait_sleep(&dfull[qg], (uint32_t)(i & 1));
-                    tc_fence_after();
-                }
-                const int ncq = qg < nq ? (((npad - QW * qg) < QW ? (npad - QW * qg) : QW) / 32) : 0;
-                const uint32_t tb = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(QW * qg);
+            for (int b = 0; b < 8; ++b) bm[b] = -0x1p120f;
+            if (have) {
+                const uint32_t u = (uint32_t)nq * i + (uint32_t)half, db = u % NDB;
+                mbar_wait_sleep(&dfull[db], (u / NDB) & 1u);
+                tc_fence_after();
+                KTR(KTR_EPI, 11);
+                KTR(KTR_EPI + 4, 22);
+                KPR(16, i);
+                const uint32_t tb = tq + QW * db;
+#ifdef KM_ONE_LD
+                constexpr int kLd = 1;
+#else
+                constexpr int kLd = 2;  // 32-column chunks per tcgen05.wait::ld
+#endif
 #pragma unroll
-                for (int c = 0; c < QW / 32; ++c) {
-                    const int ch = qg * (QW / 32) + c;
-                    if (c < ncq) {
-                        uint32_t v[32];
-                        tmem_ld<32>(tb + c * 32, v);
-                        tmem_wait();
+                for (int c2 = 0; c2 < 4; c2 += kLd) {
+                    uint32_t v[2][32];
+                    if (c2 < ncq) tmem_ld<32>(tb + c2 * 32, v[0]);
+                    if (kLd == 2 && c2 + 1 < ncq) tmem_ld<32>(tb + (c2 + 1) * 32, v[1]);
+                    tmem_wait();
 #pragma unroll
-                        for (int g = 0; g < 8; ++g)
-                            gm[ch * 8 + g] =
-                                max3(__uint_as_float(v[4 * g]), __uint_as_float(v[4 * g + 1]),
-                                     fmaxf(__uint_as_float(v[4 * g + 2]), __uint_as_float(v[4 * g + 3])));
-                    } else {
+                    for (int e = 0; e < kLd; ++e) {
+                        const int c = c2 + e;
+                        if (c < ncq) {
+#define VF(k) __uint_as_float(v[e][k])
+                            bm[2 * c] = max3(max3(max3(VF(0), VF(1), VF(2)), max3(VF(3), VF(4), VF(5)),
+                                                  max3(VF(6), VF(7), VF(8))),
+                                             max3(VF(9), VF(10), VF(11)), max3(VF(12), VF(13), fmaxf(VF(14), VF(15))));
+                            bm[2 * c + 1] = max3(max3(max3(VF(16), VF(17), VF(18)), max3(VF(19), VF(20), VF(21)),
+                                                      max3(VF(22), VF(23), VF(24))),
+                                                 max3(VF(25), VF(26), VF(27)), max3(VF(28), VF(29), fmaxf(VF(30), VF(31))));
 #pragma unroll
-                        for (int g = 0; g < 8; ++g) gm[ch * 8 + g] = -0x1p120f;
+                            for (int a = 0; a < 16; ++a) am[a] = max3(am[a], VF(a), VF(16 + a));
+#undef VF
+                        }
                     }
                 }
-                if (qg < nq) {  // this accumulator is consumed: the next tile's MMAs may refill it
-                    tc_fence_before();
-                    mbar_arrive(&dempty[qg]);
-                }
+                tc_fence_before();
+                mbar_arrive(&dempty[db]);  // the ring slot may take another half
+            } else {
+                // a half without centroids still reads the converter's E, Q terms of this tile:
+                // order it after them through the other half's accumulator (waiting only)
+                mbar_wait_sleep(&dfull[i % NDB], (i / NDB) & 1u);
             }
-            float vm[8];
-#pragma unroll
-            for (int u = 0; u < 8; ++u)
-                vm[u] = max3(max3(gm[8 * u], gm[8 * u + 1], gm[8 * u + 2]), max3(gm[8 * u + 3], gm[8 * u + 4], gm[8 * u + 5]),
-                             fmaxf(gm[8 * u + 6], gm[8 * u + 7]));
-            const float vmax = max3(max3(vm[0], vm[1], vm[2]), max3(vm[3], vm[4], vm[5]), fmaxf(vm[6], vm[7]));
+            KTR(KTR_EPI, 12);
+            KTR(KTR_EPI + 4, 23);
+            // this half's own threshold, from its own maximum vh: thr_h <= the global threshold
+            // (a smaller maximum only raises Dhat), so its local candidates include the global ones
+            const float vh = max3(max3(bm[0], bm[1], bm[2]), max3(bm[3], bm[4], bm[5]), fmaxf(bm[6], bm[7]));
             float E, Qa;  // from the converter (stage i % BS is recycled only after this tile's reduction)
             asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(E), "=f"(Qa)
                          : "r"(sbase + OFF_EQ + ((uint32_t)(i % BS) * TM + r) * 8) : "memory");
-            const float Dhat = fmaxf(Qa - 2.f * vmax, 0.f);
-            const float T = (2.f * E + 0x1p-16f * Dhat) * 1.001f;
-            // candidate group <=> its maximum >= vmax - T <=> > thr (next float below vmax - T);
-            // the sign bits of thr - gm are funnel-shifted into masks (bit 31 - g <-> group g)
-            const float thr = next_below(vmax - T);
-            uint32_t mk0 = 0, mk1 = 0;
-            const uint64_t thr2 = pk2(thr, thr);
+            auto thr_of = [&](float vm) {  // candidate <=> value >= vm - T <=> > thr (next float below)
+                const float Dhat = fmaxf(Qa - 2.f * vm, 0.f);
+                const float T = (2.f * E + 0x1p-16f * Dhat) * 1.001f;
+                return next_below(vm - T);
+            };
+            const float thr_h = thr_of(vh);
+            KTR(KTR_EPI, 15);
+            // sign bits of thr - max (packed FSUB2, each lane rounds alone) funnel-shifted into masks
+            const uint64_t thr2 = pk2(thr_h, thr_h);
+            uint32_t mA0 = 0, mA1 = 0, mB = 0;  // bit 15 - a (a < 8 in mA0 << 8) / 7 - b
 #pragma unroll
-            for (int g = 0; g < 32; g += 2) {  // packed: two groups per FADD2 (each lane rounds alone)
+            for (int a = 0; a < 8; a += 2) {  // two independent funnel chains for the a-groups
                 float d0, d1, d2, d3;
-                upk2(sub2(thr2, pk2(gm[g], gm[g + 1])), d0, d1);
-                upk2(sub2(thr2, pk2(gm[32 + g], gm[32 + g + 1])), d2, d3);
-                mk0 = __funnelshift_l(__float_as_uint(d0), mk0, 1);
-                mk1 = __funnelshift_l(__float_as_uint(d2), mk1, 1);
-                mk0 = __funnelshift_l(__float_as_uint(d1), mk0, 1);
-                mk1 = __funnelshift_l(__float_as_uint(d3), mk1, 1);
+                upk2(sub2(thr2, pk2(am[a], am[a + 1])), d0, d1);
+                upk2(sub2(thr2, pk2(am[8 + a], am[9 + a])), d2, d3);
+                mA0 = __funnelshift_l(__float_as_uint(d0), mA0, 1);
+                mA1 = __funnelshift_l(__float_as_uint(d2), mA1, 1);
+                mA0 = __funnelshift_l(__float_as_uint(d1), mA0, 1);
+                mA1 = __funnelshift_l(__float_as_uint(d3), mA1, 1);
             }
-            // exact re-check of the candidate groups in ascending centroid order (strict <)
+            const uint32_t mA = (mA0 << 8) | mA1;
+#pragma unroll
+            for (int b = 0; b < 8; b += 2) {
+                float d0, d1;
+                upk2(sub2(thr2, pk2(bm[b], bm[b + 1])), d0, d1);
+                mB = __funnelshift_l(__float_as_uint(d0), mB, 1);
+                mB = __funnelshift_l(__float_as_uint(d1), mB, 1);
+            }
+            // local verdict: 0 none, 1 + c single candidate c (global index: the half's maximum), -1 several
+            int verdict = 0;
+            if (mB) {
+                if (__popc(mA) == 1 && __popc(mB) == 1)
+                    verdict = 1 + 128 * half + 16 * (7 - (31 - __clz(mB))) + (15 - (31 - __clz(mA)));
+                else
+                    verdict = -1;
+            }
+            KTR(KTR_EPI, 16);
+            // one exchange per tile: both halves' maxima and local verdicts (slots by tile parity: a
+            // warp reaches the next tile's write before its partner has read this tile's values)
+            float* exv = exv0 + (i & 1) * 2 * TM;
+            int* exs = exs0 + (i & 1) * 2 * TM;
+            exv[half * TM + r] = vh;
+            exs[half * TM + r] = verdict;
+            KPR(17, i);
+            named_bar(1 + q, 64);
+            KPR(18, i);
+            KTR(KTR_EPI, 18);
+            KTR(KTR_EPI + 4, 24);
+            const float m0 = exv[r], m1 = exv[TM + r];
+            const int v0 = exs[r], v1 = exs[TM + r];
+            // global threshold (the same in both warps); a half has global candidates only if its
+            // maximum exceeds it, and then they are among its local ones: the argmin is unique when
+            // exactly one half does and that half's local verdict is a single column
+            const float thr = thr_of(fmaxf(m0, m1));
+            const bool in0 = m0 > thr, in1 = m1 > thr;
+            const bool unique = in0 != in1 && (in0 ? v0 : v1) > 0;
             float bd = __int_as_float(0x7f800000);
-            int bi = 0;
-            while (mk0 | mk1) {
-                int G;
-                if (mk0) { G = __clz(mk0); mk0 &= ~(0x80000000u >> G); }
-                else { G = 32 + __clz(mk1); mk1 &= ~(0x80000000u >> (G - 32)); }
-                const uint32_t gb = sPC + G * kGrpBytes;
-                uint64_t acc0 = 0ull, acc1 = 0ull;  // (4G, 4G+1), (4G+2, 4G+3)
+            int bi = unique ? (in0 ? v0 : v1) - 1 : 0;
+            if (__any_sync(0xffffffffu, !unique)) {  // warp-uniform in both warps of the pair
+                if (!unique && mB && (half == 0 ? in0 : in1)) {
+                    // the point's coordinates (global memory: the tile's stage may be recycled)
+                    float xv[16];
+                    const float4* xp = reinterpret_cast<const float4*>(xg + (valid ? p : p0) * 16);
 #pragma unroll
-                for (int j = 0; j < 16; j += 2) {
-                    const float4 c0 = lds_f4(gb + j * 8);
-                    const float4 c1 = lds_f4(gb + 128 + j * 8);
-                    const uint64_t xa = pk2(xv[j], xv[j]), xb = pk2(xv[j + 1], xv[j + 1]);
-                    uint64_t d = add2(xa, pk2(c0.x, c0.y));
-                    acc0 = fma2(d, d, acc0);
-                    d = add2(xa, pk2(c1.x, c1.y));
-                    acc1 = fma2(d, d, acc1);
-                    d = add2(xb, pk2(c0.z, c0.w));
-                    acc0 = fma2(d, d, acc0);
-                    d = add2(xb, pk2(c1.z, c1.w));
-                    acc1 = fma2(d, d, acc1);
+                    for (int j = 0; j < 4; ++j) {
+                        const float4 v = xp[j];
+                        xv[4 * j] = v.x; xv[4 * j + 1] = v.y; xv[4 * j + 2] = v.z; xv[4 * j + 3] = v.w;
+                    }
+                    // 4-column groups of the product set, ascending: b-group lb, quarter qq of it
+                    uint32_t quarters = 0;  // quarter k holds a-groups 4k..4k+3 (bits 15-4k..12-4k)
+#pragma unroll
+                    for (int k = 0; k < 4; ++k) quarters |= ((mA >> (12 - 4 * k)) & 0xFu) ? (1u << k) : 0u;
+                    uint32_t mb = mB;
+                    while (mb) {
+                        const int lb = __clz(mb) - 24;  // bit 7 - lb
+                        mb &= ~(0x80u >> lb);
+                        uint32_t qs = quarters;
+                        while (qs) {
+                            const int qq = __ffs(qs) - 1;
+                            qs &= qs - 1;
+                            const int G = 32 * half + 4 * lb + qq;  // global 4-centroid group
+                            const uint32_t gb = sPC + G * kGrpBytes;
+                            uint64_t acc0 = 0ull, acc1 = 0ull;  // (4G, 4G+1), (4G+2, 4G+3)
+#pragma unroll
+                            for (int j = 0; j < 16; j += 2) {
+                                const float4 c0 = lds_f4(gb + j * 8);
+                                const float4 c1 = lds_f4(gb + 128 + j * 8);
+                                const uint64_t xa = pk2(xv[j], xv[j]), xb = pk2(xv[j + 1], xv[j + 1]);
+                                uint64_t d = add2(xa, pk2(c0.x, c0.y));
+                                acc0 = fma2(d, d, acc0);
+                                d = add2(xa, pk2(c1.x, c1.y));
+                                acc1 = fma2(d, d, acc1);
+                                d = add2(xb, pk2(c0.z, c0.w));
+                                acc0 = fma2(d, d, acc0);
+                                d = add2(xb, pk2(c1.z, c1.w));
+                                acc1 = fma2(d, d, acc1);
+                            }
+                            float dd[4];
+                            upk2(acc0, dd[0], dd[1]);
+                            upk2(acc1, dd[2], dd[3]);
+#pragma unroll
+                            for (int e = 0; e < 4; ++e) {
+                                const int c = 4 * G + e;
+                                if (c < kc && dd[e] < bd) { bd = dd[e]; bi = c; }
+                            }
+                        }
+                    }
                 }
-                float dd[4];
-                upk2(acc0, dd[0], dd[1]);
-                upk2(acc1, dd[2], dd[3]);
-#pragma unroll
-                for (int e = 0; e < 4; ++e) {
-                    const int c = 4 * G + e;
-                    if (c < kc && dd[e] < bd) { bd = dd[e]; bi = c; }
+                // half 1 hands its winner to half 0; the lower half wins ties (lower indices)
+                if (half == 1) { exd[r] = bd; exi[r] = bi; }
+                KPR(19, i);
+                named_bar(1 + q, 64);
+                KPR(20, i);
+                if (half == 0 && !unique) {
+                    const float d1 = exd[r];
+                    if (d1 < bd) { bd = d1; bi = exi[r]; }
                 }
             }
-            if (valid) member[p] = bi;
+            KTR(KTR_EPI, 17);
+            // member[] and the reductiontoarray count (the sums go through the MMA): half 1 when the
+            // winner is proved unique (both halves know it), half 0 after a re-check
+            if (valid && unique == (half == 1)) {
+                member[p] = bi;
+                atomicAdd(&s_cnt[bi], 1);
+            }
+            if (half == 1) continue;
             // the point's one-hot byte (cluster row bi, point column r); the byte this thread set
             // in this stage OS tiles ago is cleared first
             const int o = (int)(i % OS);
+            KPR(21, i);
             mbar_wait(&oempty[o], (uint32_t)((i / OS) & 1) ^ 1u);
+            KTR(KTR_EPI, 19);
             int32_t& pd = (o == 0) ? pend[0] : pend[1];
             if (pd >= 0) sts_u8(sOH + o * kOHBytes + (uint32_t)pd, 0u);
             if (valid) {
@@ -587,20 +817,29 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
             }
             fence_async_smem();
             mbar_arrive(&ofull[o]);
+            KPR(22, i);
+            KTR(KTR_EPI, 20);
+            KTR(7, 26);
+            KTR(8, 27);
+            KTR(9, 28);
         }
-        // reduction accumulators: lane = cluster (h*128 + r), columns 4j+b = byte sums, 64 = count
+        // reduction accumulators: lane = cluster (h*128 + r), columns 4j+b = byte sums; counts
+        // from the shared atomics (every epilogue warp has passed its last tile: named barrier)
+        KPR(23, 0);
+        named_bar(5, 256);
+        KPR(24, 0);
         mbar_wait(sdone, 0);
+        KPR(25, 0);
         tc_fence_after();
-        for (int h = 0; h < nh; ++h) {
-            uint32_t v0[32], v1[32], v2[16];
-            const uint32_t tb = tmem + ((uint32_t)(q * 32) << 16) + kColSum + 80u * h;
-            tmem_ld<32>(tb, v0);
-            tmem_ld<32>(tb + 32, v1);
-            tmem_ld<16>(tb + 64, v2);
+        for (int h = half; h < nh; h += 2) {
+            uint32_t v0[32], v1[32];
+            const uint32_t tb2 = tq + kColSum + (uint32_t)(kRows * h);
+            tmem_ld<32>(tb2, v0);
+            tmem_ld<32>(tb2 + 32, v1);
             tmem_wait();
             const int c = 128 * h + r;
-            const uint64_t cnt = v2[0];
-            if (c < kc && cnt) {
+            const uint64_t cnt = c < kc ? (uint64_t)s_cnt[c] : 0ull;
+            if (cnt) {
 #pragma unroll
                 for (int j = 0; j < 16; ++j) {
                     const uint32_t* w = j < 8 ? &v0[4 * j] : &v1[4 * (j - 8)];
@@ -614,11 +853,41 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ ce
         }
     }
     tc_fence_before();
+    KPR(26, 0);
     __syncthreads();
+    KPR(27, 0);
     tc_fence_after();
     if (warp == 1) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
 }
 
+}  // namespace
+
+#ifdef KM_PROGRESS
+static unsigned* h_prog = nullptr;
+#endif
+}  // namespace k
+}  // namespace accmg
+#ifdef KM_PROGRESS
+// debug builds only: per-warp progress of the first 4096 CTAs in mapped host memory
+extern "C" int accmg_km_progress_init(void) {
+    if (cudaHostAlloc(&accmg::k::h_prog, 4096 * 16 * 4, cudaHostAllocMapped) != cudaSuccess) return -1;
+    memset(accmg::k::h_prog, 0xff, 4096 * 16 * 4);
+    unsigned* d = nullptr;
+    cudaHostGetDevicePointer(&d, accmg::k::h_prog, 0);
+    return cudaMemcpyToSymbol(accmg::k::g_prog, &d, sizeof(d)) == cudaSuccess ? 0 : -2;
+}
+extern "C" void accmg_km_progress_dump(int nctas) {
+    for (int b = 0; b < nctas; ++b) {
+        printf("cta %3d:", b);
+        for (int w = 0; w < 16; ++w) printf(" %08x", accmg::k::h_prog[b * 16 + w]);
+        printf("\n");
+    }
+    fflush(stdout);
+}
+#endif
+namespace accmg {
+namespace k {
+namespace {
 }  // namespace
 
 int kmeans_tc_supported(const float* x, int d, int kc) {
@@ -630,15 +899,7 @@ cudaError_t kmeans_assign_tc(const float* x, const float* cen, int32_t* member, 
     if (p1 <= p0) return cudaSuccess;
     if (p1 - p0 > (int64_t)INT32_MAX - TM) return cudaErrorNotSupported;  // TMA row coordinates are int32
     const int npad = ((kc + 31) / 32) * 32;
-    // accumulator group width (ACCMG_KMEANS_TC_QW: 32, 64 or 128 centroid columns; same-box A/B in
-    // profiles/r01/kmeans_tc.log: 128 = 22.9 ms, 64 = 29.4, 32 = 42.4 — more, narrower MMAs lose)
-    static int qw = -1;
-    if (qw < 0) {
-        const char* v = getenv("ACCMG_KMEANS_TC_QW");
-        qw = v ? atoi(v) : 128;
-    }
-    auto kern = qw == 64 ? assign_tc<64> : qw == 32 ? assign_tc<32> : assign_tc<128>;
-    cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, kSmemTC);
+    cudaError_t e = kernel_prep(assign_tc, kThreadsTC, kSmemTC);
     if (e != cudaSuccess) return e;
     const int64_t ntiles = (p1 - p0 + TM - 1) / TM;
     // s32 reduction accumulators: byte sums <= 255 per point, so at most 2^23 points (65536 tiles)
@@ -648,18 +909,16 @@ cudaError_t kmeans_assign_tc(const float* x, const float* cen, int32_t* member, 
     if (blocks < need) blocks = need;
     // point tiles by TMA: [rows][16] fp32 from p0, 128-row boxes, 64-byte swizzle (the per-row
     // float4 reads of the converter and epilogue threads hit 8 distinct bank groups)
-    auto fn = tma_encode_fn();
-    if (!fn) return cudaErrorNotSupported;
     CUtensorMap xmap;
     cuuint64_t dims[2] = {16, (cuuint64_t)(p1 - p0)};
     cuuint64_t strides[1] = {64};
     cuuint32_t box[2] = {16, TM};
     cuuint32_t es[2] = {1, 1};
-    if (fn(&xmap, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(x) + p0 * 16, dims, strides, box, es,
-           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B, CU_TENSOR_MAP_L2_PROMOTION_L2_128B,
-           CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE) != CUDA_SUCCESS)
+    if (!tma_encode_tiled(&xmap, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<float*>(x) + p0 * 16, dims, strides,
+                          box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B,
+                          CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE))
         return cudaErrorNotSupported;
-    kern<<<(unsigned)blocks, kThreadsTC, kSmemTC, s>>>(xmap, cen, member, sums, counts, p0, p1, kc, npad, shift,
+    assign_tc<<<(unsigned)blocks, kThreadsTC, kSmemTC, s>>>(xmap, x, cen, member, sums, counts, p0, p1, kc, npad, shift,
                                                             err_flag);
     return cudaGetLastError();
 }

@@ -77,7 +77,8 @@ struct accmg_region_s {
     std::vector<uint8_t*> gdev;      // P
     std::vector<int64_t*> gpartial;  // P
     int64_t* acc = nullptr;          // local reduction accumulator (P2P mode)
-    std::vector<void*> opened;       // IPC mappings to close
+    std::vector<void*> opened;       // IPC mappings of the peers' replicas (re-opened when a hull grows)
+    std::vector<void*> opened_partial;  // IPC mappings of the peers' reduction partials (opened once)
 };
 
 namespace {
@@ -128,9 +129,24 @@ struct State {
     int64_t* d_miss_total = nullptr;
     std::vector<Prof> prof;
     std::vector<cudaEvent_t> ev_free;
+    // deferred accounting of undeclared loops whose sizes the host does not need to launch the
+    // propagation (fused push): the compaction totals are copied into pinned slots on the stream
+    // and booked at the next synchronising call, so the loop never waits for the device
+    struct Acct {
+        int64_t esize, ce;
+        int slot;
+    };
+    std::vector<Acct> pend;
+    int64_t* h_acct = nullptr;  // kAcctSlots x 4 int64 (pinned)
 };
+constexpr int kAcctSlots = 4096;
 
 State S;
+
+// pinned host staging S.h_pin (int64 slots): [0, kPinMiss) compaction sizes / all-gathered sizes
+// (4 per region and partition: up to 16 regions x 64 partitions, plus the all-gather's copy), then
+// 128 window bounds of the write-miss completion
+constexpr int64_t kPinMiss = 4 * 16 * 64 * 2;
 
 int fail(int code, const std::string& msg, bool sticky) {
     if (sticky && !S.sticky) S.sticky = code;
@@ -283,7 +299,36 @@ struct ProfScope {
     }
 };
 
+// Bytes of one partition's packet of undeclared writes (runs, elements, dirty chunks), delivered to
+// the P-1 other partitions (reading W8; booked by the sending process).
+void book_packet(int64_t runs, int64_t elems, int64_t chunks, int64_t es, int64_t ce, bool multi) {
+    const int64_t hdr = 16 + 16 * runs, pay = es * elems;
+    S.st.bytes_undeclared_headers += (S.P - 1) * hdr;
+    S.st.bytes_undeclared_payload += (S.P - 1) * pay;
+    S.st.bytes_interpartition += (S.P - 1) * (hdr + pay);
+    S.st.bytes_paper_protocol += (S.P - 1) * chunks * (ce * es + ce / 8);
+    if (multi) S.st.bytes_remote += (int64_t)(S.W - 1 + (S.nccl_all ? 1 : 0)) * (hdr + pay);
+    if (S.p2p) S.st.bytes_remote += (int64_t)(S.P - S.V) * (hdr + pay);
+}
+
+// Books the deferred packets (one stream synchronisation for all loops since the last call).
+int flush_acct() {
+    if (S.pend.empty()) return 0;
+    CUDA_TRY(cudaStreamSynchronize(S.stream));
+    for (auto& a : S.pend) {
+        const int64_t* v = S.h_acct + 4 * a.slot;
+        if (v[3] != v[0]) {
+            S.pend.clear();
+            return fail(ACCMG_ECUDA, "compaction: run starts != run ends", true);
+        }
+        book_packet(v[0], v[1], v[2], a.esize, a.ce, false);
+    }
+    S.pend.clear();
+    return 0;
+}
+
 int collect_prof() {
+    TRY(flush_acct());
     if (S.prof.empty()) return 0;
     CUDA_TRY(cudaStreamSynchronize(S.stream));
     for (auto& p : S.prof) {
@@ -339,6 +384,11 @@ int ensure_alloc(accmg_region_s* r, const std::vector<IntervalSet>& need, int64_
         r->dev[li] = nbase;
     }
     if (changed && S.p2p) {
+        // drain this process's stream first: the hull copies above must be complete before a peer
+        // can reach the new replica (it may pull from or push into it right after the exchange),
+        // and the previous loop's pulls and pushes through the old mappings must be finished
+        // before those mappings close (every rank takes this branch: the tables are global)
+        CUDA_TRY(cudaStreamSynchronize(S.stream));
         for (auto p : r->opened) cudaIpcCloseMemHandle(p);
         r->opened.clear();
         std::vector<void*> mine(r->abase.begin(), r->abase.end()), all;
@@ -399,7 +449,7 @@ int run_xfers(const std::vector<Xfer>& xs) {
                 return fail(ACCMG_ESTATE, "data loader: range valid on no partition and not on the host copy", false);
         }
     }
-    if (S.dry) return 0;
+    if (S.dry || xs.empty()) return 0;
     ProfScope ps(2);
     bool any_nccl = false;
     // device-to-device pulls of this phase (same-GPU replicas, or peers' replicas mapped through IPC
@@ -789,6 +839,11 @@ k::PtrList push_list(accmg_region_s* r, int li) {
 }
 
 int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
+    // with the fused push nothing on the host needs the packet sizes before the write pass (the
+    // packed buffer is not materialised): the loop does not synchronise, the sizes are booked later
+    const bool fused = !S.use_nccl && k::compact_can_push();
+    const bool deferred = fused && !S.cfg.debug_checks && !S.chunks;
+    if (deferred && S.pend.size() + regs.size() * S.V > (size_t)kAcctSlots) TRY(flush_acct());
     // 1. per local replica: (debug snapshot), count, scan
     {
         ProfScope ps(1);
@@ -826,10 +881,24 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
                                                    S.stream, &S.st.kernel_launches));
         }
     }
+    if (deferred) {
+        ProfScope ps(1);
+        for (auto* r : regs)
+            for (int li = 0; li < S.V; ++li) {
+                Trk& t = r->trk[li];
+                const int slot = (int)S.pend.size();
+                CUDA_TRY(cudaMemcpyAsync(S.h_acct + 4 * slot, t.totals, 32, cudaMemcpyDeviceToHost, S.stream));
+                S.pend.push_back({r->esize, chunk_elems(r), slot});
+                CUDA_TRY(k::compact_write(t.l1, t.nwords, r->extent, t.ntiles, t.tile_counts, t.tile_offs, t.tile_edges,
+                                          r->dev[li], (int)r->esize, nullptr, 0, push_list(r, li), S.stream,
+                                          &S.st.kernel_launches, 0));
+                t.has_packed = false;
+            }
+        return 0;
+    }
     // 2. sizes to the host (one synchronisation for all regions); with the P2P transport (or one
     // process) the write pass also pushes every dirty element into the other replicas, so the
     // packed buffer is not re-read by a separate scatter pass
-    const bool fused = !S.use_nccl && k::compact_can_push();
     int slot = 0;
     for (auto* r : regs)
         for (int li = 0; li < S.V; ++li, ++slot)
@@ -918,19 +987,11 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
     }
     // accounting (by the sending process): every packet is delivered to the P-1 other partitions
     // (reading W8)
-    for (size_t ri = 0; ri < regs.size(); ++ri) {
-        const int64_t es = regs[ri]->esize, ce = chunk_elems(regs[ri]);
-        for (int g = 0; g < S.P; ++g) {
-            if (!local(g)) continue;
-            const int64_t hdr = 16 + 16 * runs[ri * S.P + g], pay = es * elems[ri * S.P + g];
-            S.st.bytes_undeclared_headers += (S.P - 1) * hdr;
-            S.st.bytes_undeclared_payload += (S.P - 1) * pay;
-            S.st.bytes_interpartition += (S.P - 1) * (hdr + pay);
-            S.st.bytes_paper_protocol += (S.P - 1) * chunks[ri * S.P + g] * (ce * es + ce / 8);
-            if (multi) S.st.bytes_remote += (int64_t)(S.W - 1 + (S.nccl_all ? 1 : 0)) * (hdr + pay);
-            if (S.p2p) S.st.bytes_remote += (int64_t)(S.P - S.V) * (hdr + pay);
-        }
-    }
+    for (size_t ri = 0; ri < regs.size(); ++ri)
+        for (int g = 0; g < S.P; ++g)
+            if (local(g))
+                book_packet(runs[ri * S.P + g], elems[ri * S.P + g], chunks[ri * S.P + g], regs[ri]->esize,
+                            chunk_elems(regs[ri]), multi);
     // 4. exchange + scatter
     ProfScope ps(2);
     if (!multi) {
@@ -1012,11 +1073,18 @@ int merge_reduce(accmg_region_s* r) {
 // Device-side precondition failures of bodies (d_flag[1]) surface at the next synchronising call.
 int check_data_flag() {
     if (S.dry) return 0;
-    CUDA_TRY(cudaMemcpyAsync(S.h_pin, S.d_flag, 2 * sizeof(int), cudaMemcpyDeviceToHost, S.stream));
+    TRY(flush_acct());
+    CUDA_TRY(cudaMemcpyAsync(S.h_pin, S.d_flag, 3 * sizeof(int), cudaMemcpyDeviceToHost, S.stream));
     CUDA_TRY(cudaStreamSynchronize(S.stream));
-    if (((int*)S.h_pin)[1]) {
-        CUDA_TRY(cudaMemsetAsync(S.d_flag + 1, 0, sizeof(int), S.stream));
-        return fail(ACCMG_EDATA, "kmeans: a point is not on the 2^-shift fixed-point grid (|x*2^shift| < 2^31)", false);
+    const int* f = (const int*)S.h_pin;
+    const int grid = f[1], scat = f[2];
+    if (grid || scat) {
+        CUDA_TRY(cudaMemsetAsync(S.d_flag + 1, 0, 2 * sizeof(int), S.stream));
+        CUDA_TRY(cudaStreamSynchronize(S.stream));
+        if (grid)
+            return fail(ACCMG_EDATA, "kmeans: a point is not on the 2^-shift fixed-point grid (|x*2^shift| < 2^31)", false);
+        return fail(ACCMG_EDATA, "scatter: an index lies in no partition's write window (negative, >= m, or a gap); "
+                                 "its write was dropped", false);
     }
     return 0;
 }
@@ -1025,7 +1093,9 @@ void free_region(accmg_region_s* r) {
     if (!S.dry) {
         cudaStreamSynchronize(S.stream);
         for (auto p : r->opened) cudaIpcCloseMemHandle(p);
+        for (auto p : r->opened_partial) cudaIpcCloseMemHandle(p);
         r->opened.clear();
+        r->opened_partial.clear();
         if (S.p2p) {  // nobody frees memory a peer may still have mapped
             std::string err;
             S.boot.barrier(&err);
@@ -1110,10 +1180,12 @@ int accmg_init(const accmg_config* cfg) {
     TRY(dmalloc((void**)&S.scratch, 2 * k::kScatterBlocks * 8, true));
     TRY(dmalloc((void**)&S.d_sizes, (size_t)4 * 8 * 16 * S.P * (S.W + 1), true));
     TRY(dmalloc((void**)&S.d_flag, 16, true));
-    TRY(dmalloc((void**)&S.d_miss, sizeof(int64_t) * 4 * 64, true));
-    S.d_miss_total = S.d_miss + 3 * 64;
-    CUDA_TRY(cudaMemsetAsync(S.d_miss, 0, sizeof(int64_t) * 4 * 64, S.stream));
-    CUDA_TRY(cudaHostAlloc((void**)&S.h_pin, (size_t)4 * 8 * 16 * S.P * (S.W + 1) + 64, cudaHostAllocDefault));
+    // [V] per-loop miss counters, [64) window starts at 2*64, ends at 3*64, running total at 4*64
+    TRY(dmalloc((void**)&S.d_miss, sizeof(int64_t) * 5 * 64, true));
+    S.d_miss_total = S.d_miss + 4 * 64;
+    CUDA_TRY(cudaMemsetAsync(S.d_miss, 0, sizeof(int64_t) * 5 * 64, S.stream));
+    CUDA_TRY(cudaHostAlloc((void**)&S.h_pin, (size_t)(kPinMiss + 128) * 8, cudaHostAllocDefault));
+    CUDA_TRY(cudaHostAlloc((void**)&S.h_acct, (size_t)kAcctSlots * 4 * 8, cudaHostAllocDefault));
     CUDA_TRY(cudaMemsetAsync(S.d_flag, 0, 16, S.stream));
     if (S.p2p) {
         std::string err;
@@ -1162,6 +1234,7 @@ int accmg_finalize(void) {
         for (auto p : S.miss_recs) dfree(p, 0, true);
         dfree(S.recv, 0, true);
         if (S.h_pin) cudaFreeHost(S.h_pin);
+        if (S.h_acct) cudaFreeHost(S.h_acct);
         for (auto& p : S.prof) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
         for (auto e : S.ev_free) cudaEventDestroy(e);
         if (S.comm) S.nccl->CommDestroy(S.comm);
@@ -1348,7 +1421,7 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
                 if (S.p2p && fresh) {  // same loop on every rank: publish the partials
                     TRY(dmalloc((void**)&r->acc, r->extent * 8, true));
                     std::vector<void*> mine(r->partial.begin(), r->partial.end()), all;
-                    TRY(exchange_ptrs(mine, all, r->opened));
+                    TRY(exchange_ptrs(mine, all, r->opened_partial));
                     r->gpartial.resize(S.P);
                     for (int g = 0; g < S.P; ++g) r->gpartial[g] = static_cast<int64_t*>(all[g]);
                 }
@@ -1379,20 +1452,23 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
             // the partition whose declared write window holds the index
             ProfScope ps(2);
             accmg_region_s* r = descs[2].region;
-            std::vector<int64_t> starts(S.P, 0);
+            // window bounds staged through pinned memory: [0, 64) starts, [64, 128) ends
+            int64_t* wb = S.h_pin + kPinMiss;
             int nb = 0;
             k::PtrList dl{};
             for (int g = 0; g < S.P; ++g) {
                 IntervalSet w = window(descs[2], ca[g], cb[g], r->extent);
                 if (w.empty()) continue;
-                starts[nb++] = w.items()[0].lo;
+                wb[nb] = w.items()[0].lo;
+                wb[64 + nb] = w.items()[0].hi;
+                ++nb;
                 dl.p[dl.n++] = S.p2p ? (void*)r->gdev[g] : (void*)r->dev[lidx(g)];
             }
-            CUDA_TRY(cudaMemcpyAsync(S.d_miss + 2 * 64, starts.data(), sizeof(int64_t) * nb, cudaMemcpyHostToDevice,
-                                     S.stream));
+            CUDA_TRY(cudaMemcpyAsync(S.d_miss + 2 * 64, wb, sizeof(int64_t) * 128, cudaMemcpyHostToDevice, S.stream));
             for (int li = 0; li < S.V; ++li)
-                CUDA_TRY(k::apply_misses(S.miss_recs[li], S.d_miss + li, S.miss_cap, dl, S.d_miss + 2 * 64, nb,
-                                         S.d_miss_total, S.stream, &S.st.kernel_launches));
+                CUDA_TRY(k::apply_misses(S.miss_recs[li], S.d_miss + li, S.miss_cap, dl, S.d_miss + 2 * 64,
+                                         S.d_miss + 3 * 64, nb, S.d_miss_total, S.d_flag + 2, S.stream,
+                                         &S.st.kernel_launches));
         }
         if (!tracked_regs.empty()) TRY(propagate_dirty(tracked_regs));
         for (int i = 0; i < n_descs; ++i)
@@ -1494,9 +1570,9 @@ int accmg_get_stats(accmg_stats* out) {
     if (!S.dry) {
         TRY(collect_prof());
         TRY(check_data_flag());
-        int64_t misses = 0;
-        CUDA_TRY(cudaMemcpy(&misses, S.d_miss_total, sizeof(int64_t), cudaMemcpyDeviceToHost));
-        S.st.write_misses = misses - S.miss_base;
+        CUDA_TRY(cudaMemcpyAsync(S.h_pin, S.d_miss_total, sizeof(int64_t), cudaMemcpyDeviceToHost, S.stream));
+        CUDA_TRY(cudaStreamSynchronize(S.stream));
+        S.st.write_misses = S.h_pin[0] - S.miss_base;
         S.st.bytes_write_miss = S.st.write_misses * 12;  // int64 index + fp32 value delivered
     }
     *out = S.st;
@@ -1508,7 +1584,10 @@ int accmg_reset_stats(void) {
     GUARD();
     if (!S.dry) {
         TRY(collect_prof());
-        CUDA_TRY(cudaMemcpy(&S.miss_base, S.d_miss_total, sizeof(int64_t), cudaMemcpyDeviceToHost));
+        // the miss counter is written on the library stream (non-blocking): read it there
+        CUDA_TRY(cudaMemcpyAsync(S.h_pin, S.d_miss_total, sizeof(int64_t), cudaMemcpyDeviceToHost, S.stream));
+        CUDA_TRY(cudaStreamSynchronize(S.stream));
+        S.miss_base = S.h_pin[0];
     }
     const int64_t u = S.st.device_bytes_user, sy = S.st.device_bytes_system;
     S.st = accmg_stats{};

@@ -1,8 +1,10 @@
 """One rank of a multi-process (one process per GPU) run, used by tests/test_gpu_multiproc.py.
 
-usage: python tests/mp_worker.py RANK WORLD V UID_HEX WORKLOAD OUTDIR [EXCHANGE_MODE]
+usage: python tests/mp_worker.py RANK WORLD V UID_HEX WORKLOAD OUTDIR [EXCHANGE_MODE [DEVICE]]
 Runs the workload through the C ABI with world_size = WORLD, num_partitions = WORLD * V, and
 saves its host arrays (after sync_to_host) and its stats under OUTDIR/rank<R>_*.npy/.json.
+DEVICE defaults to 0; the launching test passes rank % device_count (one process per GPU on a
+multi-GPU box, ranks sharing the GPU on a one-GPU box).
 """
 import json
 import os
@@ -23,7 +25,8 @@ def main():
     uid = bytes.fromhex(sys.argv[4])
     work, out = sys.argv[5], sys.argv[6]
     mode = int(sys.argv[7]) if len(sys.argv) > 7 else A.XCHG_AUTO
-    A.accmg_init(num_partitions=world * V, world_size=world, rank=rank, device=0, nccl_unique_id=uid,
+    device = int(sys.argv[8]) if len(sys.argv) > 8 else 0
+    A.accmg_init(num_partitions=world * V, world_size=world, rank=rank, device=device, nccl_unique_id=uid,
                  exchange_mode=mode, dirty_chunk_bytes=8192)
     res = {}
     if work in ("jacobi_decl", "jacobi_undecl"):
@@ -33,6 +36,14 @@ def main():
         per = WL.jacobi_run(Ah, Bh, S, declared=(work == "jacobi_decl"), per_loop_stats=True)
         res = {"A": Ah, "B": Bh}
         loops = {k: sum(p[k] for p in per) for k in per[0]}
+    elif work == "jacobi_decl_sync":
+        # no stats call between the loops and sync_to_host: nothing synchronises the stream before
+        # the hull growth of the non-owned copy-out (ensure_alloc ordering)
+        N, S = 2048, 4
+        Ah = gen.jacobi_field(6, N)
+        Bh = Ah.copy()
+        WL.jacobi_run(Ah, Bh, S, declared=True)
+        res = {"A": Ah, "B": Bh}
     elif work == "kmeans":
         x = gen.kmeans_points(5, 20000, 16, 32, gen.KM_OVERLAP)
         cen, mem = WL.kmeans_run(x, 32, 5)
@@ -60,7 +71,7 @@ def main():
         A.accmg_sync_to_host(regs[2])
         res = {"dst": dst}
     st = A.accmg_get_stats()
-    if work.startswith("jacobi"):
+    if work in ("jacobi_decl", "jacobi_undecl"):
         st = {"total": st, **loops}
     A.accmg_finalize()
     for k, v in res.items():

@@ -24,10 +24,19 @@ def _gpu():
     need_gpu()
 
 
-def _launch(world, V, work, tmp_path, mode=0):
+def _device_count():
+    import torch
+    return torch.cuda.device_count()
+
+
+def _launch(world, V, work, tmp_path, mode=0, devices=None):
+    """One process per rank; rank r runs on devices[r] (default r % device_count: one GPU per rank
+    on a multi-GPU box, all ranks on the one GPU otherwise)."""
     uid = os.urandom(128).hex()
+    nd = _device_count()
+    devices = devices or [r % nd for r in range(world)]
     procs = [subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "mp_worker.py"), str(r), str(world), str(V),
-                               uid, work, str(tmp_path), str(mode)], cwd=ROOT)
+                               uid, work, str(tmp_path), str(mode), str(devices[r])], cwd=ROOT)
              for r in range(world)]
     for p in procs:
         assert p.wait(timeout=600) == 0
@@ -113,3 +122,50 @@ def test_jacobi_three_processes(tmp_path, work):
     if work == "jacobi_undecl":
         P = 3
         assert sum(s["bytes_interpartition"] for s in stats) == S * (P - 1) * (16 * P + 16 * (N - 2) + 4 * (N - 2) ** 2)
+
+
+@pytest.mark.parametrize("work", ["jacobi_decl", "jacobi_undecl", "kmeans", "masked"])
+def test_two_physical_gpus(tmp_path, work):
+    """Ranks 0 and 1 on devices 0 and 1: replicas mapped across GPUs through CUDA IPC, halo rows
+    posted into the peer's HBM over NVLink by the Jacobi body, dirty elements pushed by the
+    compaction pass, reduction partials read over NVLink, and the flag barrier across devices.
+    Every rank bit-exact against the oracle."""
+    if _device_count() < 2:
+        pytest.skip(f"needs 2 physical GPUs, this box has {_device_count()} (the one-GPU runs above cover the same code "
+                    "path with both ranks on one device)")
+    _launch(2, 1, work, tmp_path, devices=[0, 1])
+    if work.startswith("jacobi"):
+        N, S = 300, 6
+        A0 = gen.jacobi_field(5, N)
+        oA, oB = A0.copy(), A0.copy()
+        oracle.jacobi_run(oA, oB, S)
+        exp = {"A": oA, "B": oB}
+    elif work == "kmeans":
+        x = gen.kmeans_points(5, 20000, 16, 32, gen.KM_OVERLAP)
+        ocen, omem = oracle.kmeans_run(x, 32, 5)
+        exp = {"cen": ocen, "mem": omem}
+    else:
+        n = (1 << 20) + 4321
+        src = (gen.u_fill(21, 0, n) >> np.uint64(40)).astype(np.float32) * np.float32(2.0 ** -24)
+        out = np.full(n, -1.0, dtype=np.float32)
+        for seed, dens, run in ((22, 0.5, 1), (23, 0.3, 70001), (24, 0.9, 40)):
+            oracle.masked_write(src, gen.write_mask(seed, n, dens, run), out)
+        exp = {"out": out}
+    for r in range(2):
+        for k, v in exp.items():
+            assert np.array_equal(np.load(tmp_path / f"rank{r}_{k}.npy"), v), (r, k)
+
+
+@pytest.mark.parametrize("world,V", [(2, 1), (3, 2)])
+def test_sync_to_host_right_after_loops(tmp_path, world, V):
+    """A 2048^2 declared Jacobi run whose non-owned sync_to_host follows the last loop directly (no
+    stats call to synchronise the stream): the replica hulls grow to the full extent there, so the
+    hull copies and the previous loop's pushes must complete before the new replicas are published."""
+    N, S = 2048, 4
+    A0 = gen.jacobi_field(6, N)
+    oA, oB = A0.copy(), A0.copy()
+    oracle.jacobi_run(oA, oB, S)
+    _launch(world, V, "jacobi_decl_sync", tmp_path)
+    for r in range(world):
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_A.npy"), oA)
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_B.npy"), oB)

@@ -48,3 +48,29 @@ def test_identity_has_no_misses_and_repeats():
     idx = np.arange(n, dtype=np.int32)
     got, st = _run(src, idx, 4, reps=3)
     assert np.array_equal(got, src) and st["write_misses"] == 0
+
+
+@pytest.mark.parametrize("bad", [-1, -(2 ** 31), 70000, 2 ** 31 - 1])
+@pytest.mark.parametrize("P", [1, 3])
+def test_index_outside_every_window_is_edata(bad, P):
+    """An index no partition's write window holds (negative, or >= n when dst has m > n elements) has
+    no owner: the record is dropped (no write past any replica) and the next synchronising call
+    fails with ACCMG_EDATA; every other write still lands."""
+    from paper_conf_icpp_komodamnm13_b200 import accmg as A
+    from paper_conf_icpp_komodamnm13_b200 import workloads as WL
+    n, m = 65536, 65536 + 4096
+    src = np.arange(n, dtype=np.float32) + 1
+    idx = gen.permutation(12, n)
+    idx[777] = bad
+    dst = np.zeros(m, np.float32)
+    with runtime(num_partitions=P) as acc:
+        rs, ri, rd = acc.accmg_region_create(src), acc.accmg_region_create(idx), acc.accmg_region_create(dst)
+        WL.scatter_loop(rs, ri, rd, n, m)
+        with pytest.raises(A.AccmgError) as ei:
+            acc.accmg_sync_to_host(rd)
+        assert ei.value.code == A.EDATA and "scatter" in str(ei.value)
+        acc.accmg_sync_to_host(rd)  # the flag is cleared once reported
+    exp = np.zeros(m, np.float32)
+    ok = np.arange(n) != 777
+    exp[idx[ok]] = src[ok]
+    assert np.array_equal(dst, exp)
