@@ -193,6 +193,9 @@ def run_accmg(args):
     for s in range(args.warmup):
         WL.jacobi_sweep(rA, rB, s, N, declared)
     barrier()
+    # timed region: no per-phase events between the loops (consecutive bodies overlap their launch
+    # with the previous body's tail: programmatic dependent launch)
+    A.accmg_set_profile(False)
     A.accmg_reset_stats()
     e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     with ClockSampler(dev) as clk:
@@ -204,6 +207,14 @@ def run_accmg(args):
         barrier()
     ms = e0.elapsed_time(e1)
     st = A.accmg_get_stats()
+    # the body kernel's own duration: the same loops again, bracketed per body by the library's
+    # CUDA events on its stream (profile mode)
+    A.accmg_set_profile(True)
+    A.accmg_reset_stats()
+    for s in range(args.warmup + args.steps, args.warmup + 2 * args.steps):
+        WL.jacobi_sweep(rA, rB, s, N, declared)
+    barrier()
+    stp = A.accmg_get_stats()
     t = torch.tensor([ms], dtype=torch.float64)
     tb = torch.tensor([st["bytes_interpartition"], st["kernel_launches"]], dtype=torch.float64)
     if dist:
@@ -215,7 +226,7 @@ def run_accmg(args):
 
     # roofline of the dominant kernel (the Jacobi body): algorithmic 8 B per point update
     peaks, peak_src = measured_peaks()
-    body_ms = st["ms_body"] / max(st["body_launches"], 1)
+    body_ms = stp["ms_body"] / max(stp["body_launches"], 1)
     rows_g = b - a
     alg_bytes = 8 * rows_g * (N - 2)
     achieved = alg_bytes / (body_ms / 1e3) / 1e9
@@ -225,6 +236,8 @@ def run_accmg(args):
             "frac": round(achieved / peaks["hbm_gbs"], 4), "traffic": traffic,
             "peak_source": peak_src, "kernel": "jacobi2d_tma_k (TMA-staged tiles)", "algorithmic_bytes_per_launch": alg_bytes,
             "avg_launch_ms": round(body_ms, 4),
+            "avg_launch_method": "CUDA events around each body launch on the library stream, in a second pass of "
+                                 "the same number of loops (the timed pass runs without per-launch events)",
             # also against the 8 TB/s HBM3e specification the north star quotes
             "frac_of_spec_8000GBs": round(achieved / 8000.0, 4)}
     bytes_loop = float(tb[0]) / max(st["loops"], 1)
@@ -259,33 +272,71 @@ def run_accmg(args):
     return out
 
 
+def gpu_numa_cpus(dev: int):
+    """CPUs of the NUMA node the GPU hangs off (sysfs), or None."""
+    try:
+        import pynvml
+        pynvml.nvmlInit()
+        bus = pynvml.nvmlDeviceGetPciInfo(pynvml.nvmlDeviceGetHandleByIndex(dev)).busId
+        bus = bus.decode() if isinstance(bus, bytes) else bus
+        bus = bus.lower()[-12:]  # domain:bus:device.function, 0000:xx:yy.z
+        node = int(open(f"/sys/bus/pci/devices/{bus}/numa_node").read())
+        if node < 0:
+            return None
+        cpus = set()
+        for part in open(f"/sys/devices/system/node/node{node}/cpulist").read().strip().split(","):
+            lo, _, hi = part.partition("-")
+            cpus.update(range(int(lo), int(hi or lo) + 1))
+        return cpus & os.sched_getaffinity(0) or None
+    except Exception:
+        return None
+
+
 def run_e2e(args, A, WL, torch, stream, dist, ws, rank, local, declared):
+    """End to end through the C ABI: per step region_create + copy-in (the first loop's data loader
+    pulls this rank's windows from pinned host memory) + the sweeps + sync_to_host_owned of the result
+    + region_destroy, host wall clock, max over ranks. Host buffers are pinned (cudaHostAlloc through
+    torch) and allocated and generated by threads of the GPU's NUMA node."""
     N = args.size
     a, b = A.accmg_chunk(1, N - 1, ws, rank)
     r0, r1 = (a - 1, b + 1) if declared else (0, N)
-    Ah = np.empty((N, N), dtype=np.float32)
-    Bh = np.empty((N, N), dtype=np.float32)
-    import gen
-    gen.jacobi_field(2, N, r0, r1, out=Ah[r0:r1])
-    Bh[r0:r1] = Ah[r0:r1]
-    A0 = Ah[r0:r1].copy()
-    cr = torch.cuda.cudart()
-    for arr in (Ah, Bh):  # pin this rank's rows
-        nb = (r1 - r0) * N * 4
-        assert int(cr.cudaHostRegister(arr[r0:r1].ctypes.data, nb, 0)) == 0
-    times, h2d, d2h = [], 0, 0
+    old_aff = os.sched_getaffinity(0)
+    near = gpu_numa_cpus(local)
+    if near:
+        os.sched_setaffinity(0, near)
+    try:
+        import gen
+        pin = [torch.empty(((r1 - r0), N), dtype=torch.float32, pin_memory=True) for _ in range(2)]
+        pa, pb = pin[0].numpy(), pin[1].numpy()
+        gen.jacobi_field(2, N, r0, r1, out=pa)
+        pb[...] = pa
+        A0 = pa.copy()
+        # the rank's rows of the region arrays live in the pinned buffers: numpy views with the
+        # full-extent geometry, the region's host pointer is the (virtual) element 0
+        base = pa.ctypes.data - r0 * N * 4
+        Ah = np.ndarray((N, N), dtype=np.float32, buffer=(ctypes_buf(base, N * N * 4)))
+        Bh = np.ndarray((N, N), dtype=np.float32, buffer=(ctypes_buf(pb.ctypes.data - r0 * N * 4, N * N * 4)))
+    finally:
+        os.sched_setaffinity(0, old_aff)
+    times, ph, h2d, d2h = [], [], 0, 0
     for step in range(args.e2e_steps + 1):  # first is warm-up
-        Ah[r0:r1] = A0
-        Bh[r0:r1] = A0
+        pa[...] = A0
+        pb[...] = A0
         stream.synchronize()
         if dist:
             dist.barrier()
         A.accmg_reset_stats()
         t0 = time.perf_counter()
         rA, rB = A.accmg_region_create(Ah), A.accmg_region_create(Bh)
-        for s in range(args.e2e_sweeps):
+        WL.jacobi_sweep(rA, rB, 0, N, declared)   # copy-in (data loader) + sweep 1
+        A.accmg_barrier()
+        t1 = time.perf_counter()
+        for s in range(1, args.e2e_sweeps):
             WL.jacobi_sweep(rA, rB, s, N, declared)
+        A.accmg_barrier()
+        t2 = time.perf_counter()
         A.accmg_sync_to_host_owned(rA)            # the result (even sweep count: A)
+        t3 = time.perf_counter()
         st = A.accmg_get_stats()
         A.accmg_region_destroy(rA)
         A.accmg_region_destroy(rB)
@@ -295,14 +346,27 @@ def run_e2e(args, A, WL, torch, stream, dist, ws, rank, local, declared):
             dist.all_reduce(tt, op=dist.ReduceOp.MAX)
         if step > 0:
             times.append(float(tt.item()))
+            sweep = (t2 - t1) / max(args.e2e_sweeps - 1, 1)
+            ph.append((t1 - t0 - sweep, t2 - t1 + sweep, t3 - t2, time.perf_counter() - t3))
             h2d, d2h = st["bytes_h2d"], st["bytes_d2h"]
-    for arr in (Ah, Bh):
-        cr.cudaHostUnregister(arr[r0:r1].ctypes.data)
     t = float(np.median(times))
+    cin, comp, cout, rest = (float(np.median([p[i] for p in ph])) for i in range(4))
+    del Ah, Bh, pa, pb, pin
     return {"value": round((N - 2) ** 2 * args.e2e_sweeps / t, 1), "unit": UNIT, "h2d_bytes_per_step": h2d,
             "d2h_bytes_per_step": d2h, "sweeps_per_step": args.e2e_sweeps, "seconds_per_step": round(t, 4),
-            "note": "host wall clock per step: region_create (copy-in from pinned host) + sweeps + "
-                    "sync_to_host_owned of the result, max over ranks; per-rank bytes"}
+            "phases_s": {"copy_in": round(cin, 4), "sweeps": round(comp, 4), "copy_out": round(cout, 4),
+                         "stats_destroy": round(rest, 4)},
+            "h2d_GBs": round(h2d / cin / 1e9, 2) if cin > 0 else None,
+            "d2h_GBs": round(d2h / cout / 1e9, 2) if cout > 0 else None,
+            "host_numa_bound": bool(near),
+            "note": "host wall clock per step: region_create + copy-in from pinned host (data loader of the "
+                    "first loop) + sweeps + sync_to_host_owned of the result + region_destroy, max over ranks; "
+                    "per-rank bytes; copy_in = first loop minus one sweep"}
+
+
+def ctypes_buf(addr: int, nbytes: int):
+    import ctypes
+    return (ctypes.c_uint8 * nbytes).from_address(addr)
 
 
 def free_port() -> int:

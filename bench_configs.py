@@ -137,18 +137,24 @@ def kmeans_cfg(n, iters, P, check):
         A.accmg_finalize()
     its = iters - 1
     ms_assign = st["ms_body"] / its  # body time includes the (tiny) update loop
-    lane_ops = 2.0 * n * k * d
     out = {"config": "c4", "P": P, "n": n, "iters_timed": its, "iters_per_s": n * its / t,
-           "ms_per_iteration": t / its * 1e3, **per_loop(st, 2 * its), "gen_s": tgen,
-           "fp32_lane_ops_per_s": lane_ops / (ms_assign / 1e3)}
-    # FP32 lane peak at the clock: 148 SMs x 128 lanes x 1.965 GHz = 3.72e13 lane-ops/s (FFMA2 packs
-    # two lanes into one instruction, not two ops into one lane; scripts/fp32_micro.cu measures
-    # 3.69e13 for the FADD2+FFMA2 pair the distance uses)
-    out["frac_of_fp32_lane_peak_1965MHz"] = out["fp32_lane_ops_per_s"] / (148 * 128 * 1.965e9)
-    # tensor-core assign (default, kmeans_tc.cu): HBM-bound streaming of the points (64 B read +
-    # 4 B member written per point); the FP32 figures above are then "equivalent" lane-ops
+           "ms_per_iteration": t / its * 1e3, **per_loop(st, 2 * its), "gen_s": tgen}
+    impl = os.environ.get("ACCMG_KMEANS_IMPL", "0")
+    # HBM view: 64 B of point coordinates read + 4 B of assignment written per point
     out["assign_hbm_gbs"] = n * (d * 4 + 4) / (ms_assign / 1e3) / 1e9
     out["assign_frac_of_measured_hbm"] = out["assign_hbm_gbs"] / pk["hbm_gbs"]
+    if impl == "0":
+        # tensor-pipe view of the tcgen05 formulation (kmeans_tc.cu): per 128-point tile 8 distance
+        # MMAs (M=128, N=128, K=16 bf16: 64 cycles each) + 8 reductiontoarray MMAs (M=128, N=64,
+        # K=32 u8: 32 cycles each) = 768 tensor cycles per tile per SM at 1.965 GHz
+        tiles = -(-n // 128)
+        t_tensor = tiles / 148 * 768 / 1.965e9
+        out["assign_tensor_bound_ms"] = t_tensor * 1e3
+        out["assign_frac_of_tensor_bound"] = t_tensor / (ms_assign / 1e3)
+    else:
+        # FP32-pipe kernels: 2 k d lane-ops per point (1 sub + 1 fma) against 148 SMs x 128 lanes
+        out["fp32_lane_ops_per_s"] = 2.0 * n * k * d / (ms_assign / 1e3)
+        out["frac_of_fp32_lane_peak_1965MHz"] = out["fp32_lane_ops_per_s"] / (148 * 128 * 1.965e9)
     out["kmeans_impl"] = os.environ.get("ACCMG_KMEANS_IMPL", "0")
     if check:
         ok = np.array_equal(member, lab)

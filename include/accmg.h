@@ -271,6 +271,11 @@ int accmg_barrier(void);
 int accmg_get_stats(accmg_stats* out);
 int accmg_reset_stats(void);
 
+/* Turns the per-phase CUDA-event timing of accmg_config.profile on (1) or off (0) for the loops
+   launched from now on. The events sit between consecutive kernels on the library stream, so they
+   also stop a loop body from overlapping its launch with the previous body's tail. */
+int accmg_set_profile(int on);
+
 /* Text of the sticky error (or the last argument error); never NULL. */
 const char* accmg_last_error(void);
 

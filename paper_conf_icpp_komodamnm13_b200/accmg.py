@@ -112,6 +112,7 @@ _SIGS = {
     "accmg_barrier": [],
     "accmg_get_stats": [ctypes.POINTER(accmg_stats)],
     "accmg_reset_stats": [],
+    "accmg_set_profile": [_i32],
     "accmg_chunk": [_i64, _i64, _i32, _i32, _p64, _p64],
     "accmg_debug_dirty_bitmap": [_vp, _i32, _vp, _i64],
     "accmg_debug_chunk_bits": [_vp, _i32, _vp, _i64],
@@ -246,6 +247,10 @@ def accmg_get_stats() -> dict:
 
 def accmg_reset_stats() -> None:
     _check(_lib.accmg_reset_stats(), "accmg_reset_stats")
+
+
+def accmg_set_profile(on: bool) -> None:
+    _check(_lib.accmg_set_profile(1 if on else 0), "accmg_set_profile")
 
 
 def accmg_last_error() -> str:

@@ -45,10 +45,17 @@ jacobi2d_tma_k(const __grid_constant__ CUtensorMap map, float* __restrict__ dst,
     const int64_t rs = r0 + (int64_t)blockIdx.y * (RB * tpc);
     if (rs >= r1) return;
     const int ntiles = (int)((((r1 - rs) < RB * tpc ? (r1 - rs) : RB * tpc) + RB - 1) / RB);
+    // programmatic dependent launch: the next loop's body may be scheduled while this grid drains
+    // (its CTAs wait here, after their setup, until this grid has completed and flushed), so the
+    // launch latency between consecutive sweeps overlaps the tail of the previous one
+    asm volatile("griddepcontrol.launch_dependents;" ::: "memory");
     if (tid == 0) {
         for (int s = 0; s < kStages; ++s) dev::mbar_init(&bar[s], 1);
         dev::mbar_fence_init();
         dev::tma_prefetch_desc(&map);
+    }
+    asm volatile("griddepcontrol.wait;" ::: "memory");  // src (and dst) are the previous loop's arrays
+    if (tid == 0) {
         for (int m = 0; m < kStages && m < ntiles; ++m) {
             dev::mbar_expect_tx(&bar[m], kTileBytes);
             dev::tma_load_2d(&map, &bar[m], tiles + m * kStageFloats, (int)(k0 - 4), (int)(rs + RB * m - 1 - row_lo));
@@ -164,8 +171,18 @@ cudaError_t jacobi2d_tma(const float* src, float* dst, int64_t rows, int64_t col
             tpc = q;
         }
     }
-    dim3 grid((unsigned)strips, (unsigned)((r1 - r0 + RB * tpc - 1) / (RB * tpc)));
-    kern<<<grid, 256, smem, s>>>(map, dst, cols, r0, r1, c0, c1, cbase, row_lo, tpc, t, push);
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3((unsigned)strips, (unsigned)((r1 - r0 + RB * tpc - 1) / (RB * tpc)));
+    cfg.blockDim = dim3(256);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    at[0].val.programmaticStreamSerializationAllowed = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    e = cudaLaunchKernelEx(&cfg, kern, map, dst, cols, r0, r1, c0, c1, cbase, row_lo, tpc, t, push);
+    if (e != cudaSuccess) return e;
     if (launches) *launches += 1;
     return cudaGetLastError();
 }

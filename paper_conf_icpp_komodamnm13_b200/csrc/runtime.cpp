@@ -1596,6 +1596,13 @@ int accmg_reset_stats(void) {
     return 0;
 }
 
+int accmg_set_profile(int on) {
+    GUARD();
+    if (on != 0 && on != 1) return fail(ACCMG_EINVAL, "set_profile: 0 or 1", false);
+    S.cfg.profile = on;
+    return 0;
+}
+
 const char* accmg_last_error(void) { return S.err.c_str(); }
 
 void* accmg_stream(void) { return S.init ? (void*)S.stream : nullptr; }
