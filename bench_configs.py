@@ -139,11 +139,11 @@ def kmeans_cfg(n, iters, P, check):
     ms_assign = st["ms_body"] / its  # body time includes the (tiny) update loop
     out = {"config": "c4", "P": P, "n": n, "iters_timed": its, "iters_per_s": n * its / t,
            "ms_per_iteration": t / its * 1e3, **per_loop(st, 2 * its), "gen_s": tgen}
-    impl = os.environ.get("ACCMG_KMEANS_IMPL", "0")
+    impl = "tc" if k <= 256 else "fp32"
     # HBM view: 64 B of point coordinates read + 4 B of assignment written per point
     out["assign_hbm_gbs"] = n * (d * 4 + 4) / (ms_assign / 1e3) / 1e9
     out["assign_frac_of_measured_hbm"] = out["assign_hbm_gbs"] / pk["hbm_gbs"]
-    if impl == "0":
+    if impl == "tc":
         # tensor-pipe view of the tcgen05 formulation (kmeans_tc.cu): per 128-point tile 8 distance
         # MMAs (M=128, N=128, K=16 bf16: 64 cycles each) + 8 reductiontoarray MMAs (M=128, N=64,
         # K=32 u8: 32 cycles each) = 768 tensor cycles per tile per SM at 1.965 GHz
@@ -155,7 +155,7 @@ def kmeans_cfg(n, iters, P, check):
         # FP32-pipe kernels: 2 k d lane-ops per point (1 sub + 1 fma) against 148 SMs x 128 lanes
         out["fp32_lane_ops_per_s"] = 2.0 * n * k * d / (ms_assign / 1e3)
         out["frac_of_fp32_lane_peak_1965MHz"] = out["fp32_lane_ops_per_s"] / (148 * 128 * 1.965e9)
-    out["kmeans_impl"] = os.environ.get("ACCMG_KMEANS_IMPL", "0")
+    out["kmeans_impl"] = impl
     if check:
         ok = np.array_equal(member, lab)
         # closed form: centroids are the exact means of the generated clusters

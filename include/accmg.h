@@ -139,6 +139,8 @@ typedef struct accmg_access {
  * ACCMG_BODY_GEMM_BF16_F32: bounds ndim=2 [0,M) x [0,N);
  *   descs [A R (bf16 M*K, declared stride=K), B R (bf16 K*N, undeclared), C W (fp32 M*N, declared
  *   stride=N)]; C[i][j] = sum_k A[i][k]*B[k][j], fp32 accumulation on tcgen05 tensor cores.
+ *   Shapes: N % 8 == 0 and K % 64 == 0 (else ACCMG_EUNSUPPORTED); any M. The k order of every
+ *   element is ascending in blocks of 64 (no split-K), independent of the partition count.
  * ACCMG_BODY_KMEANS_ASSIGN: bounds ndim=1 [0,n);
  *   descs [x R (fp32 n*d, declared stride=d), centroids R (fp32 k*d), member W (int32 n, declared
  *   stride=1), sums REDUCE_SUM (int64 k*d), counts REDUCE_SUM (int64 k)];

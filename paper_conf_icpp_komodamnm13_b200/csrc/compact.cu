@@ -164,88 +164,7 @@ scan_k(const int64_t* __restrict__ tile_counts, int64_t ntiles, int64_t* __restr
     }
 }
 
-template <typename T>
-__global__ void __launch_bounds__(kThreads)
-write_k(uint32_t* __restrict__ l1, int64_t nwords, const int64_t* __restrict__ tile_counts,
-        const int64_t* __restrict__ tile_offs, const uint32_t* __restrict__ tile_edges, int64_t ntiles,
-        const T* __restrict__ values, uint8_t* __restrict__ packed, int64_t n_runs) {
-    const int64_t t = blockIdx.x;
-    if (tile_counts[3 * t + 2] == 0) return;  // clean tile (no dirty element)
-    const int64_t w0 = t * kTileWords;
-    const int64_t nw = (w0 + kTileWords < nwords ? w0 + kTileWords : nwords) - w0;
-    __shared__ uint32_t sw[kTileWords + 2];
-    __shared__ int64_t woff[3][kThreads / 32];
-    const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-    for (int64_t i = tid; i < nw; i += kThreads) {
-        sw[i + 1] = l1[w0 + i];
-        l1[w0 + i] = 0u;  // clear as we go (this tile's words are read by this block only)
-    }
-    if (tid == 0) {
-        sw[0] = t > 0 ? tile_edges[2 * (t - 1) + 1] : 0u;
-        sw[nw + 1] = t + 1 < ntiles ? tile_edges[2 * (t + 1)] : 0u;
-    }
-    __syncthreads();
-    // per-warp counts over its 256 words (lane-contiguous groups of 8)
-    const int64_t wb = (int64_t)warp * (kTileWords / (kThreads / 32));  // 256 words per warp
-    int64_t cs = 0, ce = 0, cel = 0;
-    for (int j = 0; j < 8; ++j) {
-        const int64_t i = wb + lane * 8 + j;
-        if (i < nw) {
-            const uint32_t w = sw[i + 1];
-            cs += __popc(start_mask(w, sw[i]));
-            ce += __popc(end_mask(w, sw[i + 2]));
-            cel += __popc(w);
-        }
-    }
-    cs = warp_sum(cs); ce = warp_sum(ce); cel = warp_sum(cel);
-    if (lane == 0) { woff[0][warp] = cs; woff[1][warp] = ce; woff[2][warp] = cel; }
-    __syncthreads();
-    int64_t os = tile_offs[3 * t], oe = tile_offs[3 * t + 1], oel = tile_offs[3 * t + 2];
-    for (int i = 0; i < warp; ++i) { os += woff[0][i]; oe += woff[1][i]; oel += woff[2][i]; }
-    int64_t* run_start = reinterpret_cast<int64_t*>(packed + 16);
-    int64_t* run_end = run_start + n_runs;
-    T* payload = reinterpret_cast<T*>(packed + 16 + 16 * n_runs);
-    // 8 groups of 32 words, one word per lane, in element order
-    for (int g = 0; g < 8; ++g) {
-        const int64_t i = wb + g * 32 + lane;
-        const bool ok = i < nw;
-        const uint32_t w = ok ? sw[i + 1] : 0u;
-        if (__ballot_sync(dev::kFull, w != 0u) == 0u) continue;
-        const uint32_t sm = ok ? start_mask(w, sw[i]) : 0u;
-        const uint32_t em = ok ? end_mask(w, sw[i + 2]) : 0u;
-        const int64_t gw = w0 + i;
-        const int ps = __popc(sm), pe = __popc(em), pel = __popc(w);
-        const int is = warp_incl_scan(ps), ie = warp_incl_scan(pe), iel = warp_incl_scan(pel);
-        int64_t ks = os + is - ps, ke = oe + ie - pe;
-        for (uint32_t m = sm; m; m &= m - 1) run_start[ks++] = gw * 32 + (__ffs(m) - 1);
-        for (uint32_t m = em; m; m &= m - 1) run_end[ke++] = gw * 32 + __ffs(m);
-        const int rel_el = iel - pel;  // this lane's word: first payload slot relative to oel
-        // payload: word by word, lanes = element bits; all 32 words of the group are loaded before
-        // any is stored (32 coalesced 128-byte loads in flight per warp: the gather is
-        // latency-bound otherwise)
-        const int64_t gbase = w0 + wb + g * 32;
-#pragma unroll 1
-        for (int q0 = 0; q0 < 32; q0 += 32) {
-            uint32_t wq[32];
-            int bq[32];
-            T v[32];
-#pragma unroll
-            for (int u = 0; u < 32; ++u) {
-                wq[u] = __shfl_sync(dev::kFull, w, q0 + u);
-                bq[u] = __shfl_sync(dev::kFull, rel_el, q0 + u);
-                v[u] = ((wq[u] >> lane) & 1u) ? values[(gbase + q0 + u) * 32 + lane] : T(0);
-            }
-#pragma unroll
-            for (int u = 0; u < 32; ++u)
-                if ((wq[u] >> lane) & 1u) payload[oel + bq[u] + __popc(wq[u] & ((1u << lane) - 1u))] = v[u];
-        }
-        os += __shfl_sync(dev::kFull, is, 31);
-        oe += __shfl_sync(dev::kFull, ie, 31);
-        oel += __shfl_sync(dev::kFull, iel, 31);
-    }
-}
-
-// Pass 3, default (impl 0): persistent, warp-specialised. Same output as write_k.
+// Pass 3: persistent, warp-specialised.
 // Measured: a one-tile-per-block kernel spends most of a tile's life in dependent global loads
 // (tile counts -> bitmap words -> offsets, ~5 us each under full HBM load) before any payload
 // moves, so it capped at ~4 TB/s whatever the ring depth. Here each block walks its tiles
@@ -480,12 +399,7 @@ cudaError_t launch_write_pipe_st(uint32_t* l1, int64_t nwords, int64_t extent, i
     int per_sm = 1;
     cudaError_t e = kernel_prep(kern, kConsumers + 32, smem, &per_sm);
     if (e != cudaSuccess) return e;
-    static int flat = -1;  // ACCMG_COMPACT_IMPL=2: gather path only (measurement)
-    if (flat < 0) {
-        const char* v = getenv("ACCMG_COMPACT_IMPL");
-        flat = (v && atoi(v) == 2) ? 1 : 0;
-    }
-    const int aligned = !flat && (reinterpret_cast<uintptr_t>(values) % 16) == 0;
+    const int aligned = (reinterpret_cast<uintptr_t>(values) % 16) == 0;
     const int sms = sm_count_cached();
     int64_t grid = (int64_t)sms * (per_sm > 0 ? per_sm : 1);
     if (grid > ntiles) grid = ntiles;
@@ -494,28 +408,15 @@ cudaError_t launch_write_pipe_st(uint32_t* l1, int64_t nwords, int64_t extent, i
     return cudaGetLastError();
 }
 
-// Ring depth: ACCMG_COMPACT_STAGES. Measured (C5, P = 2 and 8, profiles/r01/compact_pipe.log):
-// more blocks per SM beat deeper rings -- 3 stages (4 blocks/SM) 1.59 ms per loop, 6: 1.71,
-// 10: 1.71, 24 (1 block/SM): 2.09; the one-tile-per-block kernel was 2.37 and write_k 2.21.
+// Ring depth 3 (4 blocks per SM). Measured (C5, P = 2 and 8, profiles/r01/compact_pipe.log): more
+// blocks per SM beat deeper rings -- 3 stages 1.59 ms per loop, 6: 1.71, 10: 1.71, 24 (1 block per
+// SM): 2.09; a one-tile-per-block kernel was 2.37 and a ballot-group write pass 2.21.
 template <typename T>
 cudaError_t launch_write_stream(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
                                 const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
                                 uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s, int keep) {
-    static int st = -1;
-    if (st < 0) {
-        const char* v = getenv("ACCMG_COMPACT_STAGES");
-        st = v ? atoi(v) : 3;
-    }
-    switch (st) {
-        case 2: return launch_write_pipe_st<T, 2>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
-        case 6: return launch_write_pipe_st<T, 6>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
-        case 8: return launch_write_pipe_st<T, 8>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
-        case 4: return launch_write_pipe_st<T, 4>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
-        case 10: return launch_write_pipe_st<T, 10>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
-        case 16: return launch_write_pipe_st<T, 16>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
-        case 24: return launch_write_pipe_st<T, 24>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
-        default: return launch_write_pipe_st<T, 3>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep);
-    }
+    return launch_write_pipe_st<T, 3>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed,
+                                      n_runs, push, s, keep);
 }
 
 // ---- scatter of packed runs ----------------------------------------------------------------------
@@ -712,52 +613,20 @@ cudaError_t compact_scan(const int64_t* tile_counts, int64_t ntiles, int64_t* ti
     return cudaGetLastError();
 }
 
-static int compact_impl() {
-    static int impl = -1;  // ACCMG_COMPACT_IMPL: 0 = write_pipe_k (default), 1 = write_k (ballot groups)
-    if (impl < 0) {
-        const char* v = getenv("ACCMG_COMPACT_IMPL");
-        impl = v ? atoi(v) : 0;
-    }
-    return impl;
-}
-
-bool compact_can_push() {
-    static int fused = -1;  // ACCMG_FUSED_PUSH=0: separate scatter pass (measurement)
-    if (fused < 0) {
-        const char* v = getenv("ACCMG_FUSED_PUSH");
-        fused = v ? atoi(v) : 1;
-    }
-    return fused != 0 && compact_impl() != 1;
-}
-
 cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
                           const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
                           int esize, uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s,
                           int64_t* launches, int keep) {
-    dim3 g((unsigned)ntiles);
-    const int impl = compact_impl();
-    if (push.n > 0 && impl == 1) return cudaErrorNotSupported;
-    if (impl != 1) {
-        cudaError_t e;
-        switch (esize) {
-            case 1: e = launch_write_stream<uint8_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
-            case 2: e = launch_write_stream<uint16_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
-            case 4: e = launch_write_stream<uint32_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
-            case 8: e = launch_write_stream<uint64_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
-            default: return cudaErrorInvalidValue;
-        }
-        if (launches) *launches += 1;
-        return e;
-    }
+    cudaError_t e;
     switch (esize) {
-        case 1: write_k<uint8_t><<<g, kThreads, 0, s>>>(l1, nwords, tile_counts, tile_offs, tile_edges, ntiles, (const uint8_t*)values, packed, n_runs); break;
-        case 2: write_k<uint16_t><<<g, kThreads, 0, s>>>(l1, nwords, tile_counts, tile_offs, tile_edges, ntiles, (const uint16_t*)values, packed, n_runs); break;
-        case 4: write_k<uint32_t><<<g, kThreads, 0, s>>>(l1, nwords, tile_counts, tile_offs, tile_edges, ntiles, (const uint32_t*)values, packed, n_runs); break;
-        case 8: write_k<uint64_t><<<g, kThreads, 0, s>>>(l1, nwords, tile_counts, tile_offs, tile_edges, ntiles, (const uint64_t*)values, packed, n_runs); break;
+        case 1: e = launch_write_stream<uint8_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
+        case 2: e = launch_write_stream<uint16_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
+        case 4: e = launch_write_stream<uint32_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
+        case 8: e = launch_write_stream<uint64_t>(l1, nwords, extent, ntiles, tile_counts, tile_offs, tile_edges, values, packed, n_runs, push, s, keep); break;
         default: return cudaErrorInvalidValue;
     }
     if (launches) *launches += 1;
-    return cudaGetLastError();
+    return e;
 }
 
 cudaError_t scatter_packed(const uint8_t* packed, int64_t n_runs, const PtrList& dsts, int esize,

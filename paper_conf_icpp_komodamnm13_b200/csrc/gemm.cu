@@ -4,7 +4,8 @@
 // C are the partition's declared windows, B is replicated.
 //
 // This is a real contraction, so it runs on the 5th-generation tensor cores:
-//   * persistent kernel, one CTA per SM, 128 x 256 output tiles, K-steps of 64;
+//   * persistent kernel, one CTA per SM, 128 x 256 output tiles (the last n-block may be partial:
+//     N % 8 == 0), K-steps of 64;
 //   * warp 0 = TMA producer: A tile [128 rows][64 k] (K-major) and B tile [64 k][256 n]
 //     (N-major, four 64-column boxes), both 128-byte swizzled, into a 4-stage smem ring guarded by
 //     full/empty mbarriers;
@@ -104,7 +105,7 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     const int num_m = (int)((m1 - m0 + BM - 1) / BM);
-    const int num_n = (int)(N / BN);
+    const int num_n = (int)((N + BN - 1) / BN);  // the last n-block may be partial (N % 8 == 0)
     const int64_t num_tiles = (int64_t)num_m * num_n;
     const int nk = (int)(K / BK);
 
@@ -192,6 +193,9 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
             const int64_t row = m0 + (int64_t)mb * BM + q * 32 + lane;
             float* crow = C + row * N + (int64_t)nb * BN;
             const bool ok = row < m1;
+            // columns of this tile inside C (a partial last n-block: the TMA zero-filled B's columns
+            // past N, their accumulators are not stored)
+            const int ncols = (int)((N - (int64_t)nb * BN) < BN ? (N - (int64_t)nb * BN) : BN);
 #pragma unroll 1
             for (int c = 0; c < BN / 32; ++c) {
                 uint32_t v[32];
@@ -210,8 +214,9 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
                     float4* dst = reinterpret_cast<float4*>(crow + c * 32);
 #pragma unroll
                     for (int j = 0; j < 8; ++j)
-                        dst[j] = make_float4(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]),
-                                             __uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3]));
+                        if (c * 32 + 4 * j < ncols)
+                            dst[j] = make_float4(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]),
+                                                 __uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3]));
                 }
             }
             tc_fence_before();
@@ -225,195 +230,6 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
     if (warp == 1) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
 }
 
-
-// ---- 2-SM variant: CTA pairs (cluster of 2) share one tcgen05.mma.cta_group::2, M = 256 -----------
-// Each CTA of the pair holds its 128 rows of A and its 128 columns of B (so each SM reads half the
-// B bytes per MMA from shared memory — the operand path that bounds the 1-CTA kernel, ncu
-// sm__mem_tensor_cycles_active 84 %) and gets its 128 accumulator rows in its own TMEM. The leader
-// CTA (rank 0) issues the MMAs; both CTAs' TMA loads complete on the leader's full barrier; MMA
-// completion is multicast to both CTAs' empty / tmem-full barriers; the peer's epilogue releases
-// the accumulator on the leader's tmem-empty barrier through its cluster address.
-constexpr int BM2 = 256, BN2 = 256;
-constexpr int kA2Bytes = 128 * BK * 2;            // 16 KiB: this CTA's 128 rows of A
-constexpr int kB2Bytes = BK * 128 * 2;            // 16 KiB: this CTA's 128 columns of B
-constexpr int kStage2Bytes = kA2Bytes + kB2Bytes; // 32 KiB
-constexpr int kStages2 = 6;
-constexpr uint32_t kIdesc2 = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(BN2 >> 3) << 17) |
-                             ((uint32_t)(BM2 >> 4) << 24);
-constexpr uint32_t kPeerBitMask = 0xFEFFFFFFu;   // shared::cluster address bit of the CTA rank
-
-__device__ __forceinline__ uint32_t cluster_rank() {
-    uint32_t r;
-    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
-    return r;
-}
-__device__ __forceinline__ void cluster_sync_all() {
-    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
-}
-__device__ __forceinline__ void tma_load_2d_2sm(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1) {
-    asm volatile(
-        "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%2, %3}], [%4];" ::"r"(
-            smem_u32(dst)),
-        "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_u32(bar) & kPeerBitMask)
-        : "memory");
-}
-__device__ __forceinline__ void tc_commit_mc(uint64_t* bar, uint16_t mask) {
-    asm volatile("tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
-                     smem_u32(bar)),
-                 "h"(mask)
-                 : "memory");
-}
-__device__ __forceinline__ void tc_mma2(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
-    const uint32_t z = 0;
-    asm volatile(
-        "{\n\t.reg .pred p;\n\t"
-        "setp.ne.b32 p, %4, 0;\n\t"
-        "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, {%5, %5, %5, %5, %5, %5, %5, %5}, p;\n\t}" ::"r"(tmem_d),
-        "l"(da), "l"(db), "r"(idesc), "r"(acc), "r"(z)
-        : "memory");
-}
-__device__ __forceinline__ void mbar_arrive_remote(uint64_t* bar, uint32_t rank) {
-    uint32_t ra;
-    asm volatile("mapa.shared::cluster.u32 %0, %1, %2;" : "=r"(ra) : "r"(smem_u32(bar)), "r"(rank));
-    asm volatile("mbarrier.arrive.release.cluster.shared::cluster.b64 _, [%0];" ::"r"(ra) : "memory");
-}
-
-__global__ void __launch_bounds__(kThreads, 1)
-gemm2_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ CUtensorMap map_b,
-             float* __restrict__ C, int64_t N, int64_t K, int64_t m0, int64_t m1, int64_t row_lo) {
-    extern __shared__ __align__(1024) unsigned char smem_raw[];
-    unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
-    uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages2 * kStage2Bytes);
-    uint64_t* empty = full + kStages2;
-    uint64_t* tfull = empty + kStages2;
-    uint64_t* tempty = tfull + 2;
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
-
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    const uint32_t rank = cluster_rank();
-    const bool leader = rank == 0;
-    const int num_m = (int)((m1 - m0 + BM2 - 1) / BM2);
-    const int num_n = (int)(N / BN2);
-    const int64_t num_tiles = (int64_t)num_m * num_n;
-    const int nk = (int)(K / BK);
-    const int64_t pair = blockIdx.x >> 1, npairs = gridDim.x >> 1;
-
-    if (warp == 0 && lane == 0) {
-        for (int s = 0; s < kStages2; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
-        for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 256); }
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_a)) : "memory");
-        asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_b)) : "memory");
-    }
-    if (warp == 1) {
-        asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(smem_u32(tmem_slot)),
-                     "r"(kTmemCols));
-        asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
-    }
-    tc_fence_before();
-    cluster_sync_all();  // both CTAs' barriers initialised and TMEM allocated
-    tc_fence_after();
-    const uint32_t tmem = *tmem_slot;
-
-    if (warp == 0) {
-        if (lane == 0) {
-            int stage = 0;
-            uint32_t phase = 0;
-            for (int64_t t = pair; t < num_tiles; t += npairs) {
-                int mb, nb;
-                tile_coords(t, num_m, num_n, mb, nb);
-                const int row = (int)(m0 + (int64_t)mb * BM2 + 128 * rank);
-                const int col = nb * BN2 + 128 * (int)rank;
-                for (int kb = 0; kb < nk; ++kb) {
-                    mbar_wait(&empty[stage], phase ^ 1);
-                    unsigned char* sa = smem + stage * kStage2Bytes;
-                    unsigned char* sb = sa + kA2Bytes;
-                    if (leader) mbar_expect_tx(&full[stage], 2 * kStage2Bytes);
-                    tma_load_2d_2sm(&map_a, &full[stage], sa, kb * BK, row - (int)row_lo);
-#pragma unroll
-                    for (int j = 0; j < 2; ++j)
-                        tma_load_2d_2sm(&map_b, &full[stage], sb + j * (BK * 128), col + 64 * j, kb * BK);
-                    if (++stage == kStages2) { stage = 0; phase ^= 1; }
-                }
-            }
-        }
-    } else if (warp == 1) {
-        if (leader) {
-            int stage = 0;
-            uint32_t phase = 0;
-            int acc = 0;
-            uint32_t acc_phase = 0;
-            for (int64_t t = pair; t < num_tiles; t += npairs) {
-                mbar_wait(&tempty[acc], acc_phase ^ 1);
-                tc_fence_after();
-                const uint32_t d = tmem + (uint32_t)(acc * BN2);
-                for (int kb = 0; kb < nk; ++kb) {
-                    mbar_wait(&full[stage], phase);
-                    tc_fence_after();
-                    if (lane == 0) {
-                        const uint32_t sa = smem_u32(smem + stage * kStage2Bytes);
-                        const uint32_t sb = sa + kA2Bytes;
-#pragma unroll
-                        for (int k = 0; k < BK / 16; ++k) {
-                            const uint64_t da = sdesc(sa + k * 32, 16, 1024);
-                            const uint64_t db = sdesc(sb + k * 2048, BK * 128, 1024);
-                            tc_mma2(d, da, db, kIdesc2, (kb | k) ? 1u : 0u);
-                        }
-                        tc_commit_mc(&empty[stage], 0x3);
-                    }
-                    __syncwarp();
-                    if (++stage == kStages2) { stage = 0; phase ^= 1; }
-                }
-                if (lane == 0) tc_commit_mc(&tfull[acc], 0x3);
-                __syncwarp();
-                if (++acc == 2) { acc = 0; acc_phase ^= 1; }
-            }
-        }
-    } else {
-        const int q = warp & 3;
-        int acc = 0;
-        uint32_t acc_phase = 0;
-        for (int64_t t = pair; t < num_tiles; t += npairs) {
-            int mb, nb;
-            tile_coords(t, num_m, num_n, mb, nb);
-            mbar_wait(&tfull[acc], acc_phase);
-            tc_fence_after();
-            const int64_t row = m0 + (int64_t)mb * BM2 + 128 * rank + q * 32 + lane;
-            float* crow = C + row * N + (int64_t)nb * BN2;
-            const bool ok = row < m1;
-#pragma unroll 1
-            for (int c = 0; c < BN2 / 32; ++c) {
-                uint32_t v[32];
-                const uint32_t taddr = tmem + ((uint32_t)(q * 32) << 16) + (uint32_t)(acc * BN2 + c * 32);
-                asm volatile(
-                    "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
-                    "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
-                    : "=r"(v[0]), "=r"(v[1]), "=r"(v[2]), "=r"(v[3]), "=r"(v[4]), "=r"(v[5]), "=r"(v[6]), "=r"(v[7]),
-                      "=r"(v[8]), "=r"(v[9]), "=r"(v[10]), "=r"(v[11]), "=r"(v[12]), "=r"(v[13]), "=r"(v[14]),
-                      "=r"(v[15]), "=r"(v[16]), "=r"(v[17]), "=r"(v[18]), "=r"(v[19]), "=r"(v[20]), "=r"(v[21]),
-                      "=r"(v[22]), "=r"(v[23]), "=r"(v[24]), "=r"(v[25]), "=r"(v[26]), "=r"(v[27]), "=r"(v[28]),
-                      "=r"(v[29]), "=r"(v[30]), "=r"(v[31])
-                    : "r"(taddr));
-                asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
-                if (ok) {
-                    float4* dst = reinterpret_cast<float4*>(crow + c * 32);
-#pragma unroll
-                    for (int j = 0; j < 8; ++j)
-                        dst[j] = make_float4(__uint_as_float(v[4 * j]), __uint_as_float(v[4 * j + 1]),
-                                             __uint_as_float(v[4 * j + 2]), __uint_as_float(v[4 * j + 3]));
-                }
-            }
-            tc_fence_before();
-            if (leader) mbar_arrive(&tempty[acc]);
-            else mbar_arrive_remote(&tempty[acc], 0);
-            if (++acc == 2) { acc = 0; acc_phase ^= 1; }
-        }
-    }
-    tc_fence_before();
-    cluster_sync_all();
-    tc_fence_after();
-    if (warp == 1) asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
-}
 
 bool make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t row_bytes, uint32_t box_in,
               uint32_t box_out) {
@@ -432,7 +248,8 @@ cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M,
                       int64_t m1, int64_t a_lo, cudaStream_t s, int64_t* launches) {
     (void)M;
     if (m1 <= m0) return cudaSuccess;
-    if (N % BN != 0 || K % BK != 0 || K >= (1ll << 31) || N >= (1ll << 31) || m1 >= (1ll << 31))
+    // N % 8: B rows are 16-byte multiples for the TMA and C rows take 128-bit stores
+    if (N % 8 != 0 || K % BK != 0 || K >= (1ll << 31) || N >= (1ll << 31) || m1 >= (1ll << 31))
         return cudaErrorNotSupported;
     // A's map starts at the first whole row of its allocation, so the TMA unit never addresses
     // rows outside it (row coordinates are relative to row_lo)
@@ -442,43 +259,11 @@ cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M,
     if (!make_map(&ma, A + row_lo * K, (uint64_t)K, (uint64_t)(m1 - row_lo), (uint64_t)K * 2, BK, BM))
         return cudaErrorNotSupported;
     if (!make_map(&mb, B, (uint64_t)N, (uint64_t)K, (uint64_t)N * 2, 64, BK)) return cudaErrorNotSupported;
-    static int sms = 0, impl = 0;
-    if (!sms) {
-        int dev = 0;
-        cudaGetDevice(&dev);
-        cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-        const char* v = getenv("ACCMG_GEMM_IMPL");
-        impl = v ? atoi(v) : 1;
-    }
-    if (impl == 2) {
-        // CTA pairs: A map boxes are 128 rows (each CTA loads its half of the 256-row tile)
-        const size_t smem = 1024 + (size_t)kStages2 * kStage2Bytes + 256;
-        cudaError_t e = kernel_prep(gemm2_kernel, kThreads, smem);
-        if (e != cudaSuccess) return e;
-        const int64_t tiles = ((m1 - m0 + BM2 - 1) / BM2) * (N / BN2);
-        int64_t pairs = sms / 2;
-        if (tiles < pairs) pairs = tiles;
-        cudaLaunchConfig_t cfg{};
-        cfg.gridDim = dim3((unsigned)(2 * pairs));
-        cfg.blockDim = dim3(kThreads);
-        cfg.dynamicSmemBytes = smem;
-        cfg.stream = s;
-        cudaLaunchAttribute at[1];
-        at[0].id = cudaLaunchAttributeClusterDimension;
-        at[0].val.clusterDim.x = 2;
-        at[0].val.clusterDim.y = 1;
-        at[0].val.clusterDim.z = 1;
-        cfg.attrs = at;
-        cfg.numAttrs = 1;
-        e = cudaLaunchKernelEx(&cfg, gemm2_kernel, ma, mb, C, N, K, m0, m1, row_lo);
-        if (e != cudaSuccess) return e;
-        if (launches) *launches += 1;
-        return cudaGetLastError();
-    }
+    const int sms = sm_count_cached();
     const size_t smem = 1024 + (size_t)kStages * kStageBytes + 256;
     cudaError_t e = kernel_prep(gemm_kernel, kThreads, smem);
     if (e != cudaSuccess) return e;
-    const int64_t tiles = ((m1 - m0 + BM - 1) / BM) * (N / BN);
+    const int64_t tiles = ((m1 - m0 + BM - 1) / BM) * ((N + BN - 1) / BN);
     const int grid = (int)(tiles < sms ? tiles : sms);
     gemm_kernel<<<grid, kThreads, smem, s>>>(ma, mb, C, N, K, m0, m1, row_lo);
     if (launches) *launches += 1;

@@ -128,7 +128,7 @@ jacobi_rows(const float* __restrict__ src, float* __restrict__ dst, int64_t cols
         rb[1] = rb[kUnroll + 1];
     }
     // fused dirty tracking of every element this warp wrote (rows [rs, re) of its strip)
-    if constexpr (TRACK) trk.mark_rows(t.l1, t.l2, t.l2_shift, rs, re, cols, cw, t.dbg);
+    if constexpr (TRACK) trk.mark_rows(t.l1, t.l2, t.l2_shift, rs, re, cols, cw);
 }
 
 template <int VEC>
@@ -183,15 +183,9 @@ cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, i
                      int64_t c0, int64_t c1, int64_t src_lo, int64_t src_hi, Track t, int impl, cudaStream_t s,
                      int64_t* launches, const HaloPush& push) {
     if (r1 <= r0 || c1 <= c0) return cudaSuccess;
+    // impl 0: TMA-staged tiles (measured faster, profiles/r01/jacobi_impl.log) where the shape
+    // allows; shapes the TMA body does not take (and impl 1) run the register row-marching kernel
     if (impl == 0) {
-        static int env = -1;
-        if (env < 0) {
-            const char* v = getenv("ACCMG_JACOBI_IMPL");
-            env = v ? atoi(v) : 2;  // TMA-staged tiles: measured faster (profiles/r01/jacobi_impl.log)
-        }
-        impl = env;
-    }
-    if (impl == 2) {
         cudaError_t e = jacobi2d_tma(src, dst, rows, cols, r0, r1, c0, c1, src_lo, src_hi, t, s, launches, push);
         if (e != cudaErrorNotSupported) return e;  // shapes the TMA variant does not take fall through
     }

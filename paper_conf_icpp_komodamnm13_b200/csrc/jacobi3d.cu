@@ -161,41 +161,19 @@ cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64
     CUtensorMap map;
     cuuint64_t dims[3] = {(cuuint64_t)n2, (cuuint64_t)n1, (cuuint64_t)(plane_hi - plane_lo)};
     cuuint64_t strides[2] = {(cuuint64_t)n2 * 4, (cuuint64_t)n1 * n2 * 4};
-    static int vbox = -1;
-    if (vbox < 0) {
-        const char* v = getenv("ACCMG_J3D_VARIANT");
-        vbox = v ? atoi(v) : 0;
-    }
-    cuuint32_t box[3] = {BOXK, (cuuint32_t)((vbox == 1 || vbox == 3 || vbox == 6) ? 34 : 18), 1};
+    cuuint32_t box[3] = {BOXK, 18, 1};  // 16 rows + 2 halo rows
     cuuint32_t es[3] = {1, 1, 1};
     if (!tma_encode_tiled(&map, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 3, const_cast<float*>(src) + plane_lo * pl, dims,
                           strides, box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
                           CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE))
         return cudaErrorNotSupported;
-    // tile variant (ACCMG_J3D_VARIANT): 0 = 16 rows x 32 planes, 4 stages; 1 = 32 x 32; 2 = 16 x 64;
-    // 3 = 32 x 64; 4 / 5 = 16 x 32 with 6 / 8 stages; 6 = 32 x 32, 6 stages; 7 = 16 x 64, 6 stages.
-    // Default (-1): 8 stages (more bytes in flight per SM, 2 CTAs/SM) when the grid is at least 16
-    // waves of them, else 4 stages (5 CTAs/SM, shorter tail) — profiles/r01/f2_variants.jsonl
-    static int variant = -2;
-    if (variant == -2) {
-        const char* v = getenv("ACCMG_J3D_VARIANT");
-        variant = v ? atoi(v) : -1;
-    }
-    int var = variant;
-    if (var < 0) {
-        const int64_t ctas = ((kh - (kl / 4) * 4 + TK - 1) / TK) * ((jh - jl + 15) / 16) * ((i1 - i0 + 31) / 32);
-        var = ctas >= 16 * 2 * 148 ? 5 : 0;
-    }
-    switch (var) {
-        case 1: return launch3d<32, 32>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
-        case 2: return launch3d<16, 64>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
-        case 3: return launch3d<32, 64>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
-        case 4: return launch3d<16, 32, 6>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
-        case 5: return launch3d<16, 32, 8>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
-        case 6: return launch3d<32, 32, 6>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
-        case 7: return launch3d<16, 64, 6>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
-        default: return launch3d<16, 32>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
-    }
+    // 16 rows x 32 planes per CTA; 8 stages (more bytes in flight per SM, 2 CTAs per SM) when the
+    // grid is at least 16 waves of them, else 4 stages (5 CTAs per SM, shorter tail); the other
+    // tile shapes measured (32-row tiles, 64-plane segments, 6 stages) were slower
+    // (profiles/r01/f2_variants.jsonl)
+    const int64_t ctas = ((kh - (kl / 4) * 4 + TK - 1) / TK) * ((jh - jl + 15) / 16) * ((i1 - i0 + 31) / 32);
+    if (ctas >= 16 * 2 * 148) return launch3d<16, 32, 8>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
+    return launch3d<16, 32>(map, dst, n1, n2, i0, i1, jl, jh, kl, kh, plane_lo, t, s, launches);
 }
 
 }  // namespace k

@@ -14,7 +14,6 @@ struct Track {
     uint32_t* l1;
     uint32_t* l2;
     int l2_shift;
-    int dbg;  // experiment knob (ACCMG_TRACK_DBG): bit0 skip L1 writes, bit1 skip L2 atomics
 };
 
 // Up to 64 device pointers passed by value in the kernel parameter block (no staging copy).
@@ -37,8 +36,8 @@ struct HaloPush {
 // ---- loop bodies -----------------------------------------------------------------------------
 // 5-point Jacobi on rows [r0, r1) x cols [c0, c1) of a rows x cols fp32 array (global indices);
 // [src_lo, src_hi) = elements allocated behind src.
-// impl: 0 = auto (ACCMG_JACOBI_IMPL env, default 2), 1 = register sliding window (LDG.128),
-// 2 = TMA-staged shared-memory tiles (jacobi2d_tma.cu).
+// impl 0: TMA-staged shared-memory tiles (jacobi2d_tma.cu) where the shape and alignment allow,
+// else the register row-marching kernel (LDG.128 sliding window); impl 1: always the latter.
 cudaError_t jacobi2d(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
                      int64_t c0, int64_t c1, int64_t src_lo, int64_t src_hi, Track t, int impl, cudaStream_t s,
                      int64_t* launches, const HaloPush& push = HaloPush{});
@@ -53,14 +52,7 @@ cudaError_t jacobi3d(const float* src, float* dst, int64_t n0, int64_t n1, int64
                      int64_t jl, int64_t jh, int64_t kl, int64_t kh, int64_t src_lo, int64_t src_hi, Track t,
                      cudaStream_t s, int64_t* launches);
 
-// Deep-halo body fused: h sweeps per tile in shared memory (TMA-loaded), rows [r0, r1) of dst
-// from src; update box rows [rlo, rhi), columns [c0, c1). cudaErrorNotSupported if the shape does
-// not fit (cols % 4, cols < 128, h > 8): the caller then runs h single sweeps.
-cudaError_t jacobi2d_deep(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
-                          int64_t rlo, int64_t rhi, int64_t c0, int64_t c1, int h, int64_t src_lo, int64_t src_hi,
-                          Track t, cudaStream_t s, int64_t* launches);
-
-// Same operation, register-streamed temporal blocking (one warp per 128-column strip marching
+// Deep-halo body fused (h sweeps per launch): register-streamed temporal blocking (one warp per 128-column strip marching
 // down the rows, all h levels advanced per input row); 2 <= h <= 8.
 cudaError_t jacobi2d_deep_stream(const float* src, float* dst, int64_t rows, int64_t cols, int64_t r0, int64_t r1,
                                  int64_t rlo, int64_t rhi, int64_t c0, int64_t c1, int h, int64_t src_lo,
@@ -124,10 +116,9 @@ cudaError_t compact_count(const uint32_t* l1, const uint32_t* l2, int64_t nwords
 cudaError_t compact_scan(const int64_t* tile_counts, int64_t ntiles, int64_t* tile_offs, int64_t* totals,
                          uint32_t* l2, int64_t nl2words, cudaStream_t s, int64_t* launches);
 // Pass 3: run starts/ends and payload into the canonical packed buffer; clears L1 words.
-// values holds elements [0, extent) (global indices). push.n > 0 (only when compact_can_push()):
+// values holds elements [0, extent) (global indices). push.n > 0:
 // every dirty element is also stored at its global index into each replica of push (the other
 // partitions' replicas, local or IPC-mapped peers): compaction and propagation in one pass.
-bool compact_can_push();
 cudaError_t compact_write(uint32_t* l1, int64_t nwords, int64_t extent, int64_t ntiles, const int64_t* tile_counts,
                           const int64_t* tile_offs, const uint32_t* tile_edges, const void* values,
                           int esize, uint8_t* packed, int64_t n_runs, const PtrList& push, cudaStream_t s,

@@ -412,14 +412,9 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
                           int64_t* launches) {
     if (p1 <= p0) return cudaSuccess;
     const int sms = sm_count();
-    // implementation (ACCMG_KMEANS_IMPL): 0 = tensor-core filter + exact re-check where supported
-    // (default), 1 = FP32-pipe kernels only
-    static int impl = -1;
-    if (impl < 0) {
-        const char* v = getenv("ACCMG_KMEANS_IMPL");
-        impl = v ? atoi(v) : 0;
-    }
-    if (impl == 0 && kmeans_tc_supported(x, d, kc)) {
+    // the tensor-core filter + exact re-check (kmeans_tc.cu) where supported (d = 16, k <= 256);
+    // the FP32-pipe kernels below otherwise
+    if (kmeans_tc_supported(x, d, kc)) {
         cudaError_t e = kmeans_assign_tc(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms);
         if (e == cudaSuccess) {
             if (launches) *launches += 1;
@@ -429,59 +424,18 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
         (void)cudaGetLastError();  // unsupported shape for the tensor-core kernel: FP32-pipe kernels below
     }
     if (d == 16 && (reinterpret_cast<uintptr_t>(x) % 16) == 0) {
-        // variant (tuning knob, default chosen from measurements in profiles/)
-        static int variant = -1;
-        if (variant < 0) {
-            const char* v = getenv("ACCMG_KMEANS_VARIANT");
-            variant = v ? atoi(v) : 0;
-        }
+        // centroids in constant memory when they fit (kc <= kConstCen), else the shared-memory
+        // kernel; measured on B200 (profiles/r01/kmeans_variants.txt): 3 blocks/SM (24 warps;
+        // ptxas keeps 80 registers + 24 B of spills outside the centroid loop): 21.05 ms vs 21.43
+        // for 2 blocks/SM
         cudaError_t e;
         const bool cu2 = kc % 2 == 0;
-        switch (variant) {
-            case 1: e = launch_assign16<2, 1, 256, 1>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 2: e = launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 3: e = launch_assign16<2, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 4: e = launch_assign16<4, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 5: e = launch_assign16<4, 1, 256, 1>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 6: e = cu2 ? launch_assign16<2, 2, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                            : launch_assign16<2, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 7: e = launch_assign16<1, 1, 128, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 8: e = launch_assign16<2, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 9: e = cu2 ? launch_assign16<2, 2, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                            : launch_assign16<2, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 10: e = cu2 ? launch_assign16<1, 2, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                             : launch_assign16<1, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 11: e = (kc % 4 == 0) ? launch_assign16<1, 4, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                                       : launch_assign16<1, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 12: e = cu2 ? launch_assign16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                             : launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 18: e = cu2 ? launch_assign_c16<2, 2, 256, 3, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                             : launch_assign_c16<2, 1, 256, 3, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 19: e = cu2 ? launch_assign_c16<2, 2, 256, 2, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                             : launch_assign_c16<2, 1, 256, 2, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 20: e = launch_assign_c16<2, 1, 256, 2, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 17: e = cu2 ? launch_assign_c16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                             : launch_assign_c16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 13: e = cu2 ? launch_assign_c16<2, 2, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                             : launch_assign_c16<2, 1, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 14: e = cu2 ? launch_assign_c16<2, 2, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                             : launch_assign_c16<2, 1, 128, 4>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 15: e = (kc % 4 == 0) ? launch_assign_c16<2, 4, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                                       : launch_assign_c16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            case 16: e = (kc % 4 == 0) ? launch_assign_c16<1, 4, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                                       : launch_assign_c16<1, 1, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms); break;
-            // default: centroids in constant memory when they fit (kc <= kConstCen), else the
-            // shared-memory kernel; measured on B200 (profiles/r01/kmeans_variants.txt)
-            default:
-                if (kc <= kConstCen)  // 3 blocks/SM (24 warps; ptxas keeps 80 registers + 24 B of spills
-                                      // outside the centroid loop): 21.05 ms vs 21.43 for 2 blocks/SM
-                    e = cu2 ? launch_assign_c16<2, 2, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                            : launch_assign_c16<2, 1, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms);
-                else
-                    e = cu2 ? launch_assign16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
-                            : launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms);
-                break;
-        }
+        if (kc <= kConstCen)
+            e = cu2 ? launch_assign_c16<2, 2, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                    : launch_assign_c16<2, 1, 256, 3>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms);
+        else
+            e = cu2 ? launch_assign16<2, 2, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms)
+                    : launch_assign16<2, 1, 256, 2>(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms);
         if (e != cudaSuccess) return e;
     } else {
         const size_t smem = (((size_t)kc * d * 4 + 15) / 16) * 16 + (size_t)kc * d * 8 + (size_t)kc * 8;

@@ -557,17 +557,6 @@ int ensure_recv(int64_t bytes) {
     return 0;
 }
 
-// ACCMG_DEEP_IMPL: 2 (default) register-streamed temporal blocking, 1 = levels through shared
-// memory per tile, 0 = h single-sweep launches through scratch buffers (the general path, also
-// taken by the fused kernels' unsupported shapes).
-int deep_impl() {
-    static const int v = [] {
-        const char* e = getenv("ACCMG_DEEP_IMPL");
-        return e ? atoi(e) : 2;
-    }();
-    return v;
-}
-
 // Scratch for the deep-halo body: element range [lo, hi) in two buffers (grow-only, system memory).
 int ensure_deep(int li, int64_t lo, int64_t hi) {
     if ((int)S.deep.size() < S.V) S.deep.resize(S.V);
@@ -589,12 +578,7 @@ int ensure_deep(int li, int64_t lo, int64_t hi) {
 }
 
 k::Track track_of(accmg_region_s* r, int li, bool on) {
-    static int dbg = -1;
-    if (dbg < 0) {
-        const char* e = std::getenv("ACCMG_TRACK_DBG");
-        dbg = e ? std::atoi(e) : 0;
-    }
-    k::Track t{nullptr, nullptr, 0, dbg};
+    k::Track t{nullptr, nullptr, 0};
     if (!on) return t;
     t.l1 = r->trk[li].l1;
     t.l2 = r->trk[li].l2;
@@ -702,7 +686,7 @@ int validate_body(const accmg_bounds* bd, int body, const accmg_access* d, const
             if (ext(0) != a->M * a->K || ext(1) != a->K * a->N || ext(2) != a->M * a->N) return bad("gemm: extents");
             if (bd->lo[0] < 0 || bd->hi[0] > a->M || bd->lo[1] != 0 || bd->hi[1] != a->N)
                 return bad("gemm: bounds must be rows within [0,M) x all of [0,N)");
-            if (a->N % 16 != 0 || a->K % 64 != 0) return fail(ACCMG_EUNSUPPORTED, "gemm: needs N % 16 == 0, K % 64 == 0", false);
+            if (a->N % 8 != 0 || a->K % 64 != 0) return fail(ACCMG_EUNSUPPORTED, "gemm: needs N % 8 == 0, K % 64 == 0", false);
             return 0;
         }
         case ACCMG_BODY_KMEANS_ASSIGN:
@@ -748,9 +732,8 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
             const int64_t C = x->cols, h = x->h, rlo = bd->lo[0], rhi = bd->hi[0];
             const int64_t lo = std::max<int64_t>(a - h, 0), hi = std::min<int64_t>(b + h, x->rows);
             const Ival al = d[0].region->arange[g];
-            if (deep_impl() >= 1 && h > 1) {  // fused: h sweeps per launch without scratch
-                auto fused = deep_impl() == 2 ? k::jacobi2d_deep_stream : k::jacobi2d_deep;
-                e = fused((const float*)P(0), (float*)P(1), x->rows, C, a, b, rlo, rhi, bd->lo[1], bd->hi[1], (int)h,
+            if (h > 1) {  // fused: h sweeps per launch without scratch (register-streamed levels)
+                e = k::jacobi2d_deep_stream((const float*)P(0), (float*)P(1), x->rows, C, a, b, rlo, rhi, bd->lo[1], bd->hi[1], (int)h,
                           al.lo, al.hi, T(1), S.stream, L);
                 if (e != cudaErrorNotSupported) break;
                 e = cudaSuccess;
@@ -841,7 +824,7 @@ k::PtrList push_list(accmg_region_s* r, int li) {
 int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
     // with the fused push nothing on the host needs the packet sizes before the write pass (the
     // packed buffer is not materialised): the loop does not synchronise, the sizes are booked later
-    const bool fused = !S.use_nccl && k::compact_can_push();
+    const bool fused = !S.use_nccl;
     const bool deferred = fused && !S.cfg.debug_checks && !S.chunks;
     if (deferred && S.pend.size() + regs.size() * S.V > (size_t)kAcctSlots) TRY(flush_acct());
     // 1. per local replica: (debug snapshot), count, scan
@@ -994,16 +977,7 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
                             chunk_elems(regs[ri]), multi);
     // 4. exchange + scatter
     ProfScope ps(2);
-    if (!multi) {
-        if (fused) return 0;  // pushed by the write pass
-        // sender-side push: one scatter kernel writes the runs into every other replica — the
-        // local ones and (P2P mode) the peers' replicas through their IPC mappings over NVLink
-        for (auto* r : regs)
-            for (int li = 0; li < S.V; ++li)
-                CUDA_TRY(k::scatter_packed(r->trk[li].packed, r->trk[li].n_runs, push_list(r, li), (int)r->esize,
-                                           S.scratch, S.stream, &S.st.kernel_launches));
-        return 0;
-    }
+    if (!multi) return 0;  // pushed into every other replica by the write pass
     // receive every packet that comes from another process (or, in NCCL_ALL mode, from anyone) once
     int64_t need = 0;
     std::vector<int64_t> roff(S.P * regs.size(), -1);

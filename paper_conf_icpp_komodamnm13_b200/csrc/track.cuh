@@ -134,7 +134,7 @@ struct WarpTracker {
     // the load pipeline): lane i handles (row, word) pair i, 32 at a time; each row's chunk range is
     // marked once unless the previous row already marked it.
     __device__ __forceinline__ void mark_rows(uint32_t* __restrict__ l1, uint32_t* __restrict__ l2, int l2_shift,
-                                              int64_t rs, int64_t re, int64_t cols, int64_t cw, int dbg = 0) {
+                                              int64_t rs, int64_t re, int64_t cols, int64_t cw) {
         if (first < 0) return;
         const int lane = threadIdx.x & 31;
         constexpr int NW = VEC + 1;
@@ -153,11 +153,11 @@ struct WarpTracker {
             const uint32_t v = (lo_q << s) | (s ? (hi_q >> (32 - s)) : 0u);
             const int64_t w = (E0 >> 5) + q;
             const bool inner = w * 32 >= E0 + first && w * 32 + 31 <= E0 + last;
-            if (v && !(dbg & 1)) {
+            if (v) {
                 if (inner) l1[w] = v;
                 else atomicOr(l1 + w, v);
             }
-            if (q == 0 && !(dbg & 2)) {
+            if (q == 0) {
                 const int64_t c0 = (E0 + first) >> l2_shift, c1 = (E0 + last) >> l2_shift;
                 const int64_t cp = r > rs ? (E0 - cols + last) >> l2_shift : -1;
                 for (int64_t c = c0; c <= c1; ++c)

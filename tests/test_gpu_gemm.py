@@ -77,15 +77,53 @@ def test_large_sampled_rows():
     assert np.array_equal(C[rows], R.astype(np.float32))
 
 
-@pytest.mark.skipif(bool(__import__("os").environ.get("ACCMG_GEMM_IMPL")), reason="already a per-impl run")
-def test_two_sm_variant_bitexact():
-    """ACCMG_GEMM_IMPL=2 (tcgen05.mma.cta_group::2 CTA pairs), read once per process: the GEMM
-    tests in a child process."""
-    import os
-    import subprocess
-    import sys
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-p", "no:cacheprovider", "tests/test_gpu_gemm.py",
-                        "-k", "not two_sm_variant"], cwd=root, env=dict(os.environ, ACCMG_GEMM_IMPL="2"),
-                       capture_output=True, text=True, timeout=900)
-    assert r.returncode == 0, r.stdout[-3000:]
+@pytest.mark.parametrize("N,P", [(8, 1), (136, 3), (272, 1), (272, 2), (1000, 3)])
+def test_partial_last_n_block_bitexact(N, P):
+    """N not a multiple of the 256-column tile: the last n-block's B columns past N are zero-filled
+    by the TMA and its accumulators past N are not stored (N % 8 == 0)."""
+    M, K = 300, 128
+    Ab = gen.bf16_matrix(11, M, K, gen.BF16_INTS)
+    Bb = gen.bf16_matrix(12, K, N, gen.BF16_INTS)
+    C, _ = _run(Ab, Bb, P)
+    R = oracle.gemm_rows_f64(Ab, Bb, np.arange(M))
+    assert np.array_equal(C, R.astype(np.float32))
+
+
+@pytest.mark.parametrize("N,K", [(12, 64), (256, 96)])
+def test_unsupported_shapes_rejected(N, K):
+    from paper_conf_icpp_komodamnm13_b200 import accmg as A
+    M = 128
+    Ab = gen.bf16_matrix(13, M, K, gen.BF16_INTS)
+    Bb = gen.bf16_matrix(14, K, N, gen.BF16_INTS)
+    with pytest.raises(A.AccmgError) as ei:
+        _run(Ab, Bb, 1)
+    assert ei.value.code == A.EUNSUPPORTED
+
+
+def test_uniform_inputs_full_4096():
+    """T11 in full: every element of a 4096^3 uniform (0,1] bf16 product against the fp64 oracle,
+    elementwise relative error <= 1e-2 (north star; fp32 accumulation of positive terms gives ~1e-6)."""
+    M = N = K = 4096
+    Ab = gen.bf16_matrix(15, M, K, gen.BF16_UNIT)
+    Bb = gen.bf16_matrix(16, K, N, gen.BF16_UNIT)
+    C, _ = _run(Ab, Bb, 2)
+    R = oracle.gemm_rows_f64(Ab, Bb, np.arange(M))
+    rel = np.abs(C - R) / np.abs(R)
+    assert rel.max() <= 1e-2
+    # positive terms: fp32 accumulation in any order (and rounding mode) is within (K - 1) 2^-23
+    assert rel.max() <= (K - 1) * 2.0 ** -23
+
+
+def test_uniform_inputs_sampled_32768():
+    """T11 at the C3 size: 32768^3 uniform (0,1] bf16, 64 sampled rows (the first and last row of
+    every partition at P = 4 plus spread rows) against the fp64 oracle."""
+    M = N = K = 32768
+    Ab = gen.bf16_matrix(17, M, K, gen.BF16_UNIT)
+    Bb = gen.bf16_matrix(18, K, N, gen.BF16_UNIT)
+    C, _ = _run(Ab, Bb, 4)
+    edges = [0, 8191, 8192, 16383, 16384, 24575, 24576, 32767]
+    rows = np.unique(np.concatenate([edges, np.linspace(1, M - 2, 56).astype(np.int64)]))
+    R = oracle.gemm_rows_f64(Ab, Bb, rows)
+    rel = np.abs(C[rows] - R) / np.abs(R)
+    assert rel.max() <= 1e-2
+    assert rel.max() <= (K - 1) * 2.0 ** -23

@@ -76,7 +76,7 @@ def test_fused_shapes_bitexact(N, P, h):
     oA, oB = _oracle(A0, 3, h)
     A, B, st = _gpu(A0, 3, h, P)
     assert np.array_equal(A, oA) and np.array_equal(B, oB)
-    if P == 1 and __import__("os").environ.get("ACCMG_DEEP_IMPL", "2") != "0":  # fused: one kernel per loop (no scratch sweeps, no frame copies)
+    if P == 1:  # fused: one kernel per loop (no scratch sweeps, no frame copies)
         assert st["kernel_launches"] == 3, st["kernel_launches"]
 
 
@@ -102,19 +102,3 @@ def test_deep_undeclared_tracked():
     with runtime(num_partitions=P):
         WL.jacobi_deep_run(A, B, 2 * h, h, declared=False)
     assert np.array_equal(A, oA) and np.array_equal(B, oB)
-
-
-@pytest.mark.skipif(bool(__import__("os").environ.get("ACCMG_DEEP_IMPL")), reason="already a per-impl run")
-@pytest.mark.parametrize("impl", ["0", "1"])
-def test_other_impls_bitexact(impl):
-    """The shared-memory levels kernel (impl 1) and the scratch-buffer path (impl 0) on the same
-    parity cases (the implementation is chosen once per process, so in a child process)."""
-    import os
-    import subprocess
-    import sys
-    env = dict(os.environ, ACCMG_DEEP_IMPL=impl)
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-x", "tests/test_gpu_jacobi_deep.py",
-                        "-k", "bitexact and not other_impls"], cwd=root, env=env, capture_output=True, text=True,
-                       timeout=600)
-    assert r.returncode == 0, r.stdout[-3000:] + r.stderr[-2000:]

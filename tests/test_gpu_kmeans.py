@@ -75,10 +75,10 @@ def test_off_grid_input_is_reported():
         assert e.value.code == A.EDATA
 
 
-@pytest.mark.parametrize("k", [37, 600])
+@pytest.mark.parametrize("k", [37, 258, 301, 600])
 def test_d16_odd_k_and_k_beyond_constant_memory(k):
-    """d = 16 fast paths: odd k (one centroid per step) and k > 512 (centroids no longer fit the
-    constant-memory kernel: the shared-memory kernel runs), with duplicated points (ties)."""
+    """d = 16: k <= 256 on the tensor cores (odd k), 256 < k <= 512 on the FP32-pipe constant-memory
+    kernel (odd and even k), k > 512 on the shared-memory kernel, with duplicated points (ties)."""
     from paper_conf_icpp_komodamnm13_b200 import workloads as WL
     n = 40000
     x = gen.kmeans_points(6, n, 16, k, gen.KM_OVERLAP)

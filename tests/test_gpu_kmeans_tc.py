@@ -77,17 +77,3 @@ def test_fixed_point_near_2_31():
     x[:, 3] = np.float32(2 ** 23 - 1)
     x[::2, 5] = np.float32(-(2 ** 23) + 1)
     _run(x, 200, 2, P=2, shift=8)
-
-
-def test_fp32_pipe_path_still_exact():
-    """ACCMG_KMEANS_IMPL=1 (the FP32-pipe kernels, read once per process) on the same parity cases,
-    in a child process: both implementations stay bit-exact with the oracle."""
-    import os
-    import subprocess
-    import sys
-    root = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
-    env = dict(os.environ, ACCMG_KMEANS_IMPL="1")
-    r = subprocess.run([sys.executable, "-m", "pytest", "-q", "-p", "no:cacheprovider",
-                        "tests/test_gpu_kmeans_tc.py", "-k", "not fp32_pipe_path"],
-                       cwd=root, env=env, capture_output=True, text=True, timeout=900)
-    assert r.returncode == 0, r.stdout[-3000:]
