@@ -26,7 +26,7 @@ gen/libaccgen.so: gen/accgen.c
 # The oracle: plain C, no FMA contraction, shares nothing with the product tree.
 oracle: oracle/liboracle.so
 oracle/liboracle.so: oracle/oracle.c
-	$(CC) -O2 -ffp-contract=off -fopenmp -shared -fPIC -Wall -o $@ $< -lm
+	$(CC) -O2 -ffp-contract=off -mfma -fopenmp -shared -fPIC -Wall -o $@ $< -lm
 
 accmg: $(PKG)/libaccmg.so
 $(OBJDIR)/%.o: $(CSRC)/%.cu $(HDRS)

@@ -39,7 +39,7 @@ def _oracle_point_window(field_seed, N, S, i, j):
     return F, G, i0, j0
 
 
-@pytest.mark.parametrize("P,declared", [(1, True), (2, True), (2, False)])
+@pytest.mark.parametrize("P,declared", [(1, True), (2, True), (8, True), (2, False)])
 def test_c2_c5_full_size_sampled(P, declared):
     from paper_conf_icpp_komodamnm13_b200 import workloads as WL
     N, S = 32768, 100
@@ -88,8 +88,28 @@ def test_c4_full_size_closed_form():
     assert np.array_equal(cen, (s / cnt[:, None]).astype(np.float32))
 
 
+@pytest.fixture(scope="module")
+def t14_oracle():
+    """T14's reference: 2^22 overlapping points, k = 256, 20 iterations, run once by the oracle."""
+    n, d, k, iters = 1 << 22, 16, 256, 20
+    x = gen.kmeans_points(5, n, d, k, gen.KM_OVERLAP)
+    ocen, omem = oracle.kmeans_run(x, k, iters)
+    return x, ocen, omem
+
+
+@pytest.mark.parametrize("P", [1, 2, 4, 8])
+def test_t14_overlapping_2_22_twenty_iterations(t14_oracle, P):
+    """T14: 2^22 overlapping points (near-ties occur), k = 256, 20 iterations,
+    bit-exact assignments and centroids against the oracle at P = 1, 2, 4, 8."""
+    from paper_conf_icpp_komodamnm13_b200 import workloads as WL
+    x, ocen, omem = t14_oracle
+    with runtime(num_partitions=P):
+        cen, mem = WL.kmeans_run(x, 256, 20)
+    assert np.array_equal(mem, omem) and np.array_equal(cen, ocen)
+
+
 def test_c4_overlapping_parity_2_20():
-    """T14 (reduced): overlapping clusters — near-ties occur — bit-exact vs the oracle."""
+    """Overlapping clusters, P = 3 (a partition count that does not divide n) — bit-exact."""
     from paper_conf_icpp_komodamnm13_b200 import workloads as WL
     n, d, k, iters = 1 << 20, 16, 256, 4
     x = gen.kmeans_points(5, n, d, k, gen.KM_OVERLAP)
