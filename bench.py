@@ -216,7 +216,8 @@ def run_accmg(args):
     barrier()
     stp = A.accmg_get_stats()
     t = torch.tensor([ms], dtype=torch.float64)
-    tb = torch.tensor([st["bytes_interpartition"], st["kernel_launches"]], dtype=torch.float64)
+    tb = torch.tensor([st["bytes_interpartition"], st["kernel_launches"], st["bytes_link"], st["bytes_link_remote"]],
+                      dtype=torch.float64)
     if dist:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         dist.all_reduce(tb, op=dist.ReduceOp.SUM)  # byte counters are per process
@@ -241,6 +242,7 @@ def run_accmg(args):
             # also against the 8 TB/s HBM3e specification the north star quotes
             "frac_of_spec_8000GBs": round(achieved / 8000.0, 4)}
     bytes_loop = float(tb[0]) / max(st["loops"], 1)
+    link_loop, link_remote_loop = float(tb[2]) / max(st["loops"], 1), float(tb[3]) / max(st["loops"], 1)
     launches = int(tb[1])
 
     A.accmg_region_destroy(rA)
@@ -264,6 +266,8 @@ def run_accmg(args):
                           "parallelism": f"row-block x{ws}"},
                "roofline": roof,
                "inter_gpu_bytes_per_loop": bytes_loop,
+               "link_bytes_per_loop": link_loop,
+               "link_remote_bytes_per_loop": link_remote_loop,
                "gpu_launches": launches,
                "clocks": clk.summary()}
         if e2e:

@@ -216,6 +216,14 @@ typedef struct accmg_stats {
     double  ms_body, ms_compact, ms_exchange; /* profile=1: summed CUDA-event times */
     int64_t write_misses;             /* distributed-array writes outside the writer's window (L137) */
     int64_t bytes_write_miss;         /* (index, value) records delivered to owners: 8 + esize each */
+    /* Bytes the transport actually moves between partitions' memories (the counters above are the
+       algorithmic volumes of reading W8): pulls and pushes as above; dirty elements pushed by the
+       compaction pass = payload only (no run headers or sizes); NCCL packets = headers + payload;
+       a P2P reductiontoarray reads the P-1 other partials on every process (P(P-1) extent esize
+       per loop with one partition per process); an in-process merge reads V-1 partials; a write
+       miss stores esize into the owner's replica. */
+    int64_t bytes_link;
+    int64_t bytes_link_remote;        /* subset of bytes_link that crossed processes (NVLink) */
 } accmg_stats;
 
 /* ---- entry points ------------------------------------------------------------------------- */

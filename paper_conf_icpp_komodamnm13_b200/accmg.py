@@ -94,7 +94,8 @@ _STAT_FIELDS = ["loops", "bytes_interpartition", "bytes_declared", "bytes_undecl
 class accmg_stats(ctypes.Structure):
     _fields_ = [(f, ctypes.c_int64) for f in _STAT_FIELDS] + [
         ("ms_body", ctypes.c_double), ("ms_compact", ctypes.c_double), ("ms_exchange", ctypes.c_double),
-        ("write_misses", ctypes.c_int64), ("bytes_write_miss", ctypes.c_int64)]
+        ("write_misses", ctypes.c_int64), ("bytes_write_miss", ctypes.c_int64),
+        ("bytes_link", ctypes.c_int64), ("bytes_link_remote", ctypes.c_int64)]
 
 
 _vp, _i32, _i64, _sz = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_size_t

@@ -309,6 +309,14 @@ void book_packet(int64_t runs, int64_t elems, int64_t chunks, int64_t es, int64_
     S.st.bytes_paper_protocol += (S.P - 1) * chunks * (ce * es + ce / 8);
     if (multi) S.st.bytes_remote += (int64_t)(S.W - 1 + (S.nccl_all ? 1 : 0)) * (hdr + pay);
     if (S.p2p) S.st.bytes_remote += (int64_t)(S.P - S.V) * (hdr + pay);
+    if (multi) {  // packets to the other ranks, payload stores into this rank's other replicas
+        const int64_t nr = (int64_t)(S.W - 1 + (S.nccl_all ? 1 : 0)) * (hdr + pay);
+        S.st.bytes_link += nr + (int64_t)(S.V - 1) * pay;
+        S.st.bytes_link_remote += nr;
+    } else {      // the write pass stores each dirty element into the P-1 other replicas
+        S.st.bytes_link += (int64_t)(S.P - 1) * pay;
+        if (S.p2p) S.st.bytes_link_remote += (int64_t)(S.P - S.V) * pay;
+    }
 }
 
 // Books the deferred packets (one stream synchronisation for all loops since the last call).
@@ -442,7 +450,11 @@ int run_xfers(const std::vector<Xfer>& xs) {
         if (x.src >= 0) {
             S.st.bytes_interpartition += nb;
             S.st.bytes_declared += nb;
-            if (rank_of(x.src) != rank_of(x.dst)) S.st.bytes_remote += nb;
+            S.st.bytes_link += nb;
+            if (rank_of(x.src) != rank_of(x.dst)) {
+                S.st.bytes_remote += nb;
+                S.st.bytes_link_remote += nb;
+            }
         } else {
             S.st.bytes_h2d += nb;
             if (!x.r->host_valid.contains(IntervalSet(x.lo, x.hi)))
@@ -964,6 +976,9 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
                 S.st.bytes_undeclared_payload += (S.P - 1) * regs[ri]->trk[li].dirty_chunks * ce * es;
                 S.st.bytes_undeclared_headers += (S.P - 1) * regs[ri]->trk[li].dirty_chunks * (ce / 8);
                 if (S.p2p) S.st.bytes_remote += (int64_t)(S.P - S.V) * regs[ri]->trk[li].dirty_chunks * (ce * es + ce / 8);
+                // the merge kernel reads the chunk bits locally and stores only the dirty elements
+                S.st.bytes_link += (int64_t)(S.P - 1) * regs[ri]->trk[li].n_elems * es;
+                if (S.p2p) S.st.bytes_link_remote += (int64_t)(S.P - S.V) * regs[ri]->trk[li].n_elems * es;
             }
         }
         return 0;
@@ -1299,7 +1314,11 @@ int plan_pushes(int body_id, const accmg_access* descs, const void* args,
             if (local(pc.h)) {  // bytes are counted by the receiving process (as for pulls)
                 S.st.bytes_interpartition += nb;
                 S.st.bytes_declared += nb;
-                if (rank_of(pc.g) != rank_of(pc.h)) S.st.bytes_remote += nb;
+                S.st.bytes_link += nb;
+                if (rank_of(pc.g) != rank_of(pc.h)) {
+                    S.st.bytes_remote += nb;
+                    S.st.bytes_link_remote += nb;
+                }
             }
             if (local(g) && !S.dry) {
                 k::HaloPush& hp = S.cur_push[lidx(g)];
@@ -1458,6 +1477,18 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
             const int64_t nb = 2 * (int64_t)(S.P - 1) * r->extent * 8 * S.V / S.P;
             S.st.bytes_reduce += nb;
             S.st.bytes_interpartition += nb;
+            const int64_t sb = r->extent * 8;
+            if (S.p2p) {  // every process reads the P-1 other partials (P-V of them remote)
+                S.st.bytes_link += (int64_t)(S.P - 1) * sb;
+                S.st.bytes_link_remote += (int64_t)(S.P - S.V) * sb;
+            } else {      // local merge of V partials, then (NCCL) the ring all-reduce's share
+                S.st.bytes_link += (int64_t)(S.V - 1) * sb;
+                if (S.use_nccl && S.W > 1) {
+                    const int64_t ring = 2 * (int64_t)(S.W - 1) * sb / S.W;
+                    S.st.bytes_link += ring;
+                    S.st.bytes_link_remote += ring;
+                }
+            }
             r->host_valid.clear();
         } else if (descs[i].mode & ACCMG_W) {
             if (descs[i].declared) {
@@ -1551,6 +1582,7 @@ int accmg_get_stats(accmg_stats* out) {
     }
     *out = S.st;
     out->bytes_interpartition += out->bytes_write_miss;
+    out->bytes_link += out->write_misses * 4;  // each completion stores the fp32 value in the owner's replica
     return 0;
 }
 

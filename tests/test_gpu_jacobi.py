@@ -39,6 +39,7 @@ def test_c1_declared_p2_bitexact_and_2048_bytes():
     A, B, per, st = _gpu_run(A0, S, 2, per_loop=True)
     assert np.array_equal(A, oA) and np.array_equal(B, oB)
     assert all(p["bytes_declared"] == 2048 for p in per[2:])
+    assert all(p["bytes_link"] == p["bytes_declared"] for p in per)  # halo rows move as counted
     assert st["body_launches"] == 2 * S
 
 
@@ -119,6 +120,8 @@ def test_undeclared_multi_sweep_bitexact(P):
     A, B, per, st = _gpu_run(A0, S, P, declared=False, per_loop=True, dirty_chunk_bytes=8192)
     assert np.array_equal(A, oA) and np.array_equal(B, oB)
     assert all(p["bytes_interpartition"] == (P - 1) * (16 * P + 16 * (N - 2) + 4 * (N - 2) ** 2) for p in per)
+    # the write pass pushes payload only: no run headers, no size words
+    assert all(p["bytes_link"] == (P - 1) * 4 * (N - 2) ** 2 for p in per)
 
 
 def test_undeclared_nccl_self_exchange():
@@ -177,6 +180,7 @@ def test_paper_chunk_protocol_bitexact(P, chunk):
             chunks += len({e // ce for r in range(a, b) for e in (r * N + 1, r * N + N - 2)} |
                           {c for r in range(a, b) for c in range((r * N + 1) // ce, (r * N + N - 2) // ce + 1)})
         assert p["bytes_interpartition"] == (P - 1) * chunks * (ce * 4 + ce // 8)
+        assert p["bytes_link"] == (P - 1) * 4 * (N - 2) ** 2   # the merge stores the dirty elements only
 
 
 def test_paper_chunk_protocol_sparse_rows():

@@ -28,6 +28,8 @@ def test_overlapping_set_bitexact(P):
     assert np.array_equal(mem, omem)
     assert np.array_equal(cen, ocen)
     assert st["bytes_reduce"] == iters * 2 * (P - 1) * (k * d + k) * 8
+    # in one process the merge reads the P-1 other partials (the ring figure above is algorithmic)
+    assert st["bytes_link"] == iters * (P - 1) * (k * d + k) * 8
 
 
 def test_lattice_closed_form_and_ragged_n():

@@ -76,6 +76,9 @@ def test_kmeans_multi_process(tmp_path, world, V):
     P = world * V
     # each rank books its integer share of every all-reduce (2 regions x 5 iterations)
     assert abs(sum(s["bytes_reduce"] for s in stats) - 5 * 2 * (P - 1) * (32 * 16 + 32) * 8) < world * 5 * 2
+    # every process reads the P-1 other partials over the IPC mappings: P(P-1) S in total
+    assert sum(s["bytes_link"] for s in stats) == world * 5 * (P - 1) * (32 * 16 + 32) * 8
+    assert sum(s["bytes_link_remote"] for s in stats) == world * 5 * (P - V) * (32 * 16 + 32) * 8
 
 
 def test_scatter_two_processes(tmp_path):
