@@ -118,15 +118,28 @@ def ncu_traffic(kernel_key: str):
 
 
 # ---- CPU oracle legs -----------------------------------------------------------------------------
-def oracle_jacobi_rate(n: int, target_s: float = 10.0, steps: int = 0, warmup: int = 0):
+def cpu_model() -> str:
+    try:
+        for line in open("/proc/cpuinfo"):
+            if line.startswith("model name"):
+                return line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    return "unknown"
+
+
+def oracle_jacobi_rate(n: int, target_s: float = 10.0, steps: int = 0, warmup: int = 0, threads: int = 0,
+                       max_rows: int = 8190):
     """The oracle (oracle/oracle.c, as it stands) on a bounded sample of the C2 workload: full-width
     row bands of the n x n field, repeated sweeps for ~target_s seconds (or, with steps > 0, warmup
     untimed sweeps then exactly `steps` timed sweeps: one step = one sweep of the band), on all
-    host cores."""
+    host cores (threads = 0) or on `threads` of them."""
     import gen
     import oracle
     cores = len(os.sched_getaffinity(0)) if hasattr(os, "sched_getaffinity") else (os.cpu_count() or 1)
-    rows = min(8190, n - 2)  # 8192 x n band at C2: 1 GiB per array, far larger than any host cache
+    if threads:
+        cores = min(threads, cores)
+    rows = min(max_rows, n - 2)  # 8192 x n band at C2: 1 GiB per array, far larger than any host cache
     band = gen.jacobi_field(2, n, 0, rows + 2)  # a band of the real field (rows 0..rows+1)
     band = np.ascontiguousarray(band)
     # the oracle sweeps a square array; use a (rows+2) x n band embedded as its own field:
@@ -405,7 +418,8 @@ def main():
                 "config": {"workload": f"C2: 2D 5-point Jacobi {args.size}x{args.size} fp32, row-block partition, "
                                        + ("undeclared (dirty-bit tracking)" if args.undeclared else "declared halo h=1"),
                            "n": args.size, "partitions": 1, "sweeps_per_step": 1, "parallelism": "oracle on host cores"},
-                "cpu_baseline": {"value": round(rate, 1), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample},
+                "cpu_baseline": {"value": round(rate, 1), "unit": UNIT, "cores": cores, "kind": "oracle", "sample": sample,
+                                 "cpu_model": cpu_model()},
                 "e2e": {"value": round(rate, 1), "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
         print(json.dumps(line), flush=True)
         return
@@ -413,8 +427,11 @@ def main():
     if rank == 0:
         if not args.no_cpu_baseline and ws == 1:  # the host baseline is taken at N = 1 only
             rate, cores, sample = oracle_jacobi_rate(args.size, target_s=10.0)
+            rate1, _, sample1 = oracle_jacobi_rate(args.size, target_s=4.0, threads=1, max_rows=1022)
             out["cpu_baseline"] = {"value": round(rate, 1), "unit": UNIT, "cores": cores, "kind": "oracle",
-                                   "sample": sample}
+                                   "sample": sample, "cpu_model": cpu_model(),
+                                   "single_core": {"value": round(rate1, 1), "unit": UNIT, "cores": 1,
+                                                   "sample": sample1}}
         print(json.dumps(out), flush=True)
 
 
