@@ -93,7 +93,7 @@ constexpr int OFF_X = OFF_OH + OS * kOHBytes;
 constexpr int kGrpBytes = 272;
 constexpr int OFF_PC = OFF_X + XS * kXBytes;
 constexpr int OFF_BAR = OFF_PC + (KMAX / 4) * kGrpBytes;
-constexpr int kNumBars = 2 * XS + 2 * AS + BS + 2 * NDB + 2 * OS + 1;
+constexpr int kNumBars = 2 * XS + 2 * AS + BS + 2 * NDB + 2 * OS + 2;
 constexpr int OFF_MISC = OFF_BAR + kNumBars * 8;    // tmem slot, Cinf bits, C2 bits
 constexpr int OFF_EQ = OFF_MISC + 16;               // float2 [BS][TM]: the point's E and Q (1 + 2^-17) + 2E
 // epilogue half exchange, double-buffered by tile parity: maxima [2][2][TM], verdicts [2][2][TM];
@@ -341,6 +341,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
     uint64_t* ofull = dempty + NDB;
     uint64_t* oempty = ofull + OS;
     uint64_t* sdone = oempty + OS;
+    uint64_t* h1go = sdone + 1;  // phase i: the half-1 MMAs of tile i are issued
     uint32_t* misc = reinterpret_cast<uint32_t*>(smem + OFF_MISC);  // [0] tmem, [1] Cinf bits, [2] C2 bits
 
     constexpr int kThreads = kThreadsTC;
@@ -375,6 +376,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
         for (int b = 0; b < NDB; ++b) { mbar_init(&dfull[b], 1); mbar_init(&dempty[b], 128); }
         for (int o = 0; o < OS; ++o) { mbar_init(&ofull[o], 128); mbar_init(&oempty[o], 1); }
         mbar_init(sdone, 1);
+        mbar_init(h1go, 1);
         dev::mbar_fence_init();
     }
     KPR(1, 0);
@@ -467,6 +469,10 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             KPR(5, i);
             const uint64_t ad = dAD + (uint64_t)((a * kADBytes) >> 4);
             const uint32_t u = (uint32_t)nq * i + (uint32_t)h, db = u % NDB;  // ring slot and its use count
+            // the tensor pipe takes MMAs in issue order: half 0 of tile i waits until half 1 of tile
+            // i-1 is issued, so the far-ahead half-0 stream does not queue in front of the half-1
+            // MMAs the epilogue is waiting for
+            if (h == 0 && nq == 2 && i > 0) mbar_wait_sleep(h1go, (i - 1) & 1u);
             mbar_wait_sleep(&dempty[db], ((u / NDB) & 1u) ^ 1u);
             KTR(kMmaWarp, 5);
             KTR(kMmaWarp1, 6);
@@ -479,6 +485,10 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                               bd + (uint64_t)((k * 32) >> 4), idesc, k ? 1u : 0u);
             tc_commit_elect(&dfull[db]);
             tc_commit_elect(&aempty[a]);
+            if (h == 1) {
+                __syncwarp();
+                if (lane == 0) mbar_arrive(h1go);
+            }
             KPR(7, i);
             KTR(kMmaWarp, 13);
             KTR(kMmaWarp1, 14);
@@ -625,7 +635,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             for (int b = 0; b < 8; ++b) bm[b] = -0x1p120f;
             if (have) {
                 const uint32_t u = (uint32_t)nq * i + (uint32_t)half, db = u % NDB;
-                mbar_wait_sleep(&dfull[db], (u / NDB) & 1u);
+                mbar_wait(&dfull[db], (u / NDB) & 1u);
                 tc_fence_after();
                 KTR(KTR_EPI, 11);
                 KTR(KTR_EPI + 4, 22);
