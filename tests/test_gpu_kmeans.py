@@ -28,8 +28,10 @@ def test_overlapping_set_bitexact(P):
     assert np.array_equal(mem, omem)
     assert np.array_equal(cen, ocen)
     assert st["bytes_reduce"] == iters * 2 * (P - 1) * (k * d + k) * 8
-    # in one process the merge reads the P-1 other partials (the ring figure above is algorithmic)
-    assert st["bytes_link"] == iters * (P - 1) * (k * d + k) * 8
+    # link bytes per iteration: the merge reads the P-1 other partials (the ring figure above is
+    # the algorithmic volume), and the update loop's writes to the replicated centroids (fp32) and
+    # sums / counts (int64, reset) are pushed to the P-1 other replicas, payload only
+    assert st["bytes_link"] == iters * (P - 1) * ((k * d + k) * 8 + k * d * 4 + (k * d + k) * 8)
 
 
 def test_lattice_closed_form_and_ragged_n():

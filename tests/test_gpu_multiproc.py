@@ -76,9 +76,16 @@ def test_kmeans_multi_process(tmp_path, world, V):
     P = world * V
     # each rank books its integer share of every all-reduce (2 regions x 5 iterations)
     assert abs(sum(s["bytes_reduce"] for s in stats) - 5 * 2 * (P - 1) * (32 * 16 + 32) * 8) < world * 5 * 2
-    # every process reads the P-1 other partials over the IPC mappings: P(P-1) S in total
-    assert sum(s["bytes_link"] for s in stats) == world * 5 * (P - 1) * (32 * 16 + 32) * 8
-    assert sum(s["bytes_link_remote"] for s in stats) == world * 5 * (P - V) * (32 * 16 + 32) * 8
+    # link bytes: every process reads the P-1 other partials of each reduction over the IPC
+    # mappings (P(P-1) S in total with one partition per process); the update loop's writes to the
+    # replicated centroids / sums / counts are pushed to the P-1 other replicas (payload only); the
+    # final non-owned sync_to_host of member pulls what each process does not hold
+    S, k, d, n, iters = (32 * 16 + 32) * 8, 32, 16, 20000, 5
+    upd = k * d * 4 + (k * d + k) * 8
+    exp = world * iters * (P - 1) * S + iters * (P - 1) * upd + (world - 1) * n * 4
+    assert sum(s["bytes_link"] for s in stats) == exp
+    exp_remote = world * iters * (P - V) * S + iters * (P - V) * upd + (world - 1) * n * 4
+    assert sum(s["bytes_link_remote"] for s in stats) == exp_remote
 
 
 def test_scatter_two_processes(tmp_path):
