@@ -60,6 +60,10 @@ extern "C" {
 #define ACCMG_HALO_AUTO 0      /* push predicted halos from the writing kernel when the body can */
 #define ACCMG_HALO_PULL 1      /* the paper's data loader only: pull before read (L119, L125) */
 
+#define ACCMG_MC_OFF  0        /* accmg_config.multicast */
+#define ACCMG_MC_AUTO 1
+#define ACCMG_MC_VMM  2
+
 typedef struct accmg_config {
     int32_t num_partitions;    /* P, the number of tasks groups every loop is divided into (L108);
                                   1..64; a multiple of world_size. P / world_size partitions live on
@@ -90,7 +94,16 @@ typedef struct accmg_config {
                                   replica) and the rows count as valid there, so the next reader
                                   pulls nothing; the bytes are accounted as declared transfers.
                                   ACCMG_HALO_PULL: pull-before-read only. */
-    int32_t pad_;
+    int32_t multicast;         /* §8 row f3, P2P mode (world_size > 1, one partition per process):
+                                  ACCMG_MC_OFF (default) CUDA-IPC replicas, unicast pushes;
+                                  ACCMG_MC_AUTO: replicas of arrays written without a declared
+                                  pattern (fp32 / 64-bit elements) are driver-VMM allocations
+                                  shared through file descriptors and, where the node can create
+                                  an NVLS multicast object (accmg_multicast_probe), bound to one:
+                                  the compaction pass stores every dirty element once, through
+                                  the multicast address (multimem.st), into all replicas;
+                                  otherwise (or ACCMG_MC_VMM) unicast pushes into the shared
+                                  VMM replicas. Ignored without the P2P transport. */
     uint8_t nccl_unique_id[128]; /* world_size > 1: the job's id, made on rank 0 by
                                     accmg_nccl_unique_id() (NCCL modes) or accmg_unique_id() (P2P),
                                     broadcast by the caller (e.g. torch.distributed); P2P mode names
@@ -224,6 +237,9 @@ typedef struct accmg_stats {
        miss stores esize into the owner's replica. */
     int64_t bytes_link;
     int64_t bytes_link_remote;        /* subset of bytes_link that crossed processes (NVLink) */
+    int64_t bytes_multicast;          /* dirty payload stored once through NVLS multicast addresses
+                                         (the switch delivers it to the other replicas) */
+    int64_t multicast_regions;        /* regions whose replicas are bound to a multicast object */
 } accmg_stats;
 
 /* ---- entry points ------------------------------------------------------------------------- */
@@ -285,6 +301,12 @@ int accmg_reset_stats(void);
    launched from now on. The events sit between consecutive kernels on the library stream, so they
    also stop a loop body from overlapping its launch with the previous body's tail. */
 int accmg_set_profile(int on);
+
+/* §8 row f3: can this node create an NVLS multicast object spanning `num_devices` GPUs (the
+   driver VMM entry points present and cuMulticastCreate accepted)? Returns 1 if so; 0 if not,
+   with the reason copied into why (NUL-terminated, at most cap bytes; may be NULL); negative on
+   an argument error. Needs no accmg_init; initialises the CUDA context of the current device. */
+int accmg_multicast_probe(int num_devices, char* why, int cap);
 
 /* Text of the sticky error (or the last argument error); never NULL. */
 const char* accmg_last_error(void);

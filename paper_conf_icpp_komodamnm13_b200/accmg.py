@@ -26,6 +26,7 @@ OK, EINVAL, ECUDA, ENCCL, ENOMEM, ESTATE, EUNSUPPORTED, ECONFLICT, EDATA = 0, -1
 XCHG_AUTO, XCHG_NCCL_ALL, XCHG_NCCL = 0, 1, 2
 DIRTY_RUNS, DIRTY_CHUNKS = 0, 1
 HALO_AUTO, HALO_PULL = 0, 1
+MC_OFF, MC_AUTO, MC_VMM = 0, 1, 2
 R, W, RW, REDUCE_SUM = 1, 2, 3, 4
 BODY_JACOBI2D_5PT, BODY_GEMM_BF16_F32, BODY_KMEANS_ASSIGN, BODY_KMEANS_UPDATE = 1, 2, 3, 4
 BODY_SCATTER = 5
@@ -39,7 +40,7 @@ class accmg_config(ctypes.Structure):
     _fields_ = [("num_partitions", ctypes.c_int32), ("world_size", ctypes.c_int32), ("rank", ctypes.c_int32),
                 ("device", ctypes.c_int32), ("dirty_chunk_bytes", ctypes.c_int64),
                 ("exchange_mode", ctypes.c_int32), ("debug_checks", ctypes.c_int32), ("profile", ctypes.c_int32),
-                ("dirty_protocol", ctypes.c_int32), ("halo_mode", ctypes.c_int32), ("pad_", ctypes.c_int32),
+                ("dirty_protocol", ctypes.c_int32), ("halo_mode", ctypes.c_int32), ("multicast", ctypes.c_int32),
                 ("nccl_unique_id", ctypes.c_uint8 * 128)]
 
 
@@ -95,7 +96,8 @@ class accmg_stats(ctypes.Structure):
     _fields_ = [(f, ctypes.c_int64) for f in _STAT_FIELDS] + [
         ("ms_body", ctypes.c_double), ("ms_compact", ctypes.c_double), ("ms_exchange", ctypes.c_double),
         ("write_misses", ctypes.c_int64), ("bytes_write_miss", ctypes.c_int64),
-        ("bytes_link", ctypes.c_int64), ("bytes_link_remote", ctypes.c_int64)]
+        ("bytes_link", ctypes.c_int64), ("bytes_link_remote", ctypes.c_int64),
+        ("bytes_multicast", ctypes.c_int64), ("multicast_regions", ctypes.c_int64)]
 
 
 _vp, _i32, _i64, _sz = ctypes.c_void_p, ctypes.c_int, ctypes.c_int64, ctypes.c_size_t
@@ -114,6 +116,7 @@ _SIGS = {
     "accmg_get_stats": [ctypes.POINTER(accmg_stats)],
     "accmg_reset_stats": [],
     "accmg_set_profile": [_i32],
+    "accmg_multicast_probe": [_i32, ctypes.c_char_p, _i32],
     "accmg_chunk": [_i64, _i64, _i32, _i32, _p64, _p64],
     "accmg_debug_dirty_bitmap": [_vp, _i32, _vp, _i64],
     "accmg_debug_chunk_bits": [_vp, _i32, _vp, _i64],
@@ -183,12 +186,21 @@ def accmg_unique_id() -> bytes:
 def accmg_init(num_partitions: int = 1, world_size: int = 1, rank: int = 0, device: int = 0,
                dirty_chunk_bytes: int = 0, exchange_mode: int = XCHG_AUTO, debug_checks: int = 0,
                profile: int = 0, nccl_unique_id: bytes | None = None, dirty_protocol: int = DIRTY_RUNS,
-               halo_mode: int = HALO_AUTO) -> None:
+               halo_mode: int = HALO_AUTO, multicast: int = MC_OFF) -> None:
     c = accmg_config(num_partitions, world_size, rank, device, dirty_chunk_bytes, exchange_mode, debug_checks,
-                     profile, dirty_protocol, halo_mode)
+                     profile, dirty_protocol, halo_mode, multicast)
     if nccl_unique_id is not None:
         ctypes.memmove(c.nccl_unique_id, nccl_unique_id, 128)
     _check(_lib.accmg_init(ctypes.byref(c)), "accmg_init")
+
+
+def accmg_multicast_probe(num_devices: int) -> tuple[bool, str]:
+    """(True, "") if an NVLS multicast object over num_devices GPUs can be created, else (False, why)."""
+    buf = ctypes.create_string_buffer(512)
+    rc = _lib.accmg_multicast_probe(num_devices, buf, 512)
+    if rc < 0:
+        raise AccmgError(rc, "accmg_multicast_probe")
+    return rc == 1, buf.value.decode()
 
 
 def accmg_finalize() -> None:

@@ -3,7 +3,9 @@
 #include <fcntl.h>
 #include <sched.h>
 #include <sys/mman.h>
+#include <sys/socket.h>
 #include <sys/stat.h>
+#include <sys/un.h>
 #include <unistd.h>
 
 #include <atomic>
@@ -27,6 +29,14 @@ struct Header {
 };
 
 Header* hdr(void* base) { return static_cast<Header*>(base); }
+
+// abstract-namespace socket address of `rank` in the job `name` (no file system entry)
+socklen_t sock_addr(const std::string& name, int rank, sockaddr_un* a) {
+    std::memset(a, 0, sizeof(*a));
+    a->sun_family = AF_UNIX;
+    const int n = std::snprintf(a->sun_path + 1, sizeof(a->sun_path) - 1, "%s_fd%d", name.c_str() + 1, rank);
+    return (socklen_t)(offsetof(sockaddr_un, sun_path) + 1 + n);
+}
 
 }  // namespace
 
@@ -69,6 +79,14 @@ bool Bootstrap::open(const uint8_t id[128], int rank, int world, std::string* er
     if (base_ == MAP_FAILED) {
         base_ = nullptr;
         *err = "bootstrap: mmap failed";
+        return false;
+    }
+    // this rank's descriptor-passing socket (listening before the first barrier)
+    listen_fd_ = socket(AF_UNIX, SOCK_STREAM | SOCK_CLOEXEC, 0);
+    sockaddr_un sa;
+    const socklen_t sl = sock_addr(name_, rank, &sa);
+    if (listen_fd_ < 0 || bind(listen_fd_, reinterpret_cast<sockaddr*>(&sa), sl) != 0 || listen(listen_fd_, kMaxRanks) != 0) {
+        *err = "bootstrap: cannot listen on the descriptor socket";
         return false;
     }
     Header* H = hdr(base_);
@@ -118,7 +136,85 @@ bool Bootstrap::barrier(std::string* err) {
 
 void* Bootstrap::slot(int r) { return static_cast<char*>(base_) + 4096 + (size_t)r * kSlotBytes; }
 
+bool Bootstrap::allgather_fds(const int* mine, int n, int* out, std::string* err) {
+    if (n < 1 || n > 64) {
+        *err = "bootstrap: 1..64 descriptors per rank";
+        return false;
+    }
+    for (int i = 0; i < world_ * n; ++i) out[i] = -1;
+    // send to every other rank (its listener queues the connection until it accepts)
+    for (int q = 0; q < world_; ++q) {
+        if (q == rank_) continue;
+        sockaddr_un sa;
+        const socklen_t sl = sock_addr(name_, q, &sa);
+        int c = socket(AF_UNIX, SOCK_STREAM | SOCK_CLOEXEC, 0);
+        const auto t0 = std::chrono::steady_clock::now();
+        while (c >= 0 && connect(c, reinterpret_cast<sockaddr*>(&sa), sl) != 0) {
+            if (std::chrono::steady_clock::now() - t0 > std::chrono::seconds(60)) {
+                ::close(c);
+                c = -1;
+                break;
+            }
+            usleep(1000);
+        }
+        if (c < 0) {
+            *err = "bootstrap: cannot connect to a peer's descriptor socket";
+            return false;
+        }
+        int hdr2[2] = {rank_, n};
+        iovec iov{hdr2, sizeof(hdr2)};
+        char ctl[CMSG_SPACE(sizeof(int) * 64)];
+        std::memset(ctl, 0, sizeof(ctl));
+        msghdr m{};
+        m.msg_iov = &iov;
+        m.msg_iovlen = 1;
+        m.msg_control = ctl;
+        m.msg_controllen = CMSG_SPACE(sizeof(int) * n);
+        cmsghdr* cm = CMSG_FIRSTHDR(&m);
+        cm->cmsg_level = SOL_SOCKET;
+        cm->cmsg_type = SCM_RIGHTS;
+        cm->cmsg_len = CMSG_LEN(sizeof(int) * n);
+        std::memcpy(CMSG_DATA(cm), mine, sizeof(int) * n);
+        const bool sent = sendmsg(c, &m, 0) == (ssize_t)sizeof(hdr2);
+        ::close(c);
+        if (!sent) {
+            *err = "bootstrap: sendmsg of descriptors failed";
+            return false;
+        }
+    }
+    // receive one message from every other rank
+    for (int k = 0; k < world_ - 1; ++k) {
+        const int c = accept(listen_fd_, nullptr, nullptr);
+        if (c < 0) {
+            *err = "bootstrap: accept on the descriptor socket failed";
+            return false;
+        }
+        int hdr2[2] = {-1, 0};
+        iovec iov{hdr2, sizeof(hdr2)};
+        char ctl[CMSG_SPACE(sizeof(int) * 64)];
+        msghdr m{};
+        m.msg_iov = &iov;
+        m.msg_iovlen = 1;
+        m.msg_control = ctl;
+        m.msg_controllen = sizeof(ctl);
+        const ssize_t got = recvmsg(c, &m, MSG_CMSG_CLOEXEC);
+        ::close(c);
+        cmsghdr* cm = CMSG_FIRSTHDR(&m);
+        if (got != (ssize_t)sizeof(hdr2) || hdr2[0] < 0 || hdr2[0] >= world_ || hdr2[1] != n || !cm ||
+            cm->cmsg_type != SCM_RIGHTS || cm->cmsg_len != CMSG_LEN(sizeof(int) * n)) {
+            *err = "bootstrap: malformed descriptor message";
+            return false;
+        }
+        std::memcpy(out + hdr2[0] * n, CMSG_DATA(cm), sizeof(int) * n);
+    }
+    return barrier(err);
+}
+
 void Bootstrap::close() {
+    if (listen_fd_ >= 0) {
+        ::close(listen_fd_);
+        listen_fd_ = -1;
+    }
     if (!base_) return;
     Header* H = hdr(base_);
     const bool last = H->closed.fetch_add(1) + 1 == (uint32_t)world_;

@@ -19,8 +19,13 @@ public:
     bool barrier(std::string* err);          // all ranks; times out after 300 s
     void* slot(int rank);                    // mailbox of `rank` (kSlotBytes)
     bool is_open() const { return base_ != nullptr; }
+    // All-gather of file descriptors (n per rank, the same n everywhere) over Unix-domain sockets
+    // (SCM_RIGHTS): out[q * n + i] = rank q's i-th descriptor, received as a new descriptor here
+    // (out[rank * n + i] = -1). Collective; ends with a barrier.
+    bool allgather_fds(const int* mine, int n, int* out, std::string* err);
 
 private:
+    int listen_fd_ = -1;
     void* base_ = nullptr;
     size_t bytes_ = 0;
     int rank_ = 0, world_ = 1;

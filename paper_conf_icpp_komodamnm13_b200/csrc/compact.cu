@@ -197,6 +197,27 @@ struct TileRec {  // one dirty tile, written by the producer before it arrives o
     int nw, dense;  // t < 0: end of this block's tiles
 };
 
+// A push store: into one replica, or (push.mc) through the multicast address into all of them.
+template <typename T>
+__device__ __forceinline__ void push_store(const PtrList& push, int d, int64_t e, T v) {
+    T* p = static_cast<T*>(push.p[d]) + e;
+    if constexpr (sizeof(T) == 4) {
+        if (push.mc) {
+            asm volatile("multimem.st.relaxed.sys.global.b32 [%0], %1;" ::"l"(p), "r"(*reinterpret_cast<uint32_t*>(&v))
+                         : "memory");
+            return;
+        }
+    } else if constexpr (sizeof(T) == 8) {
+        if (push.mc) {
+            asm volatile("multimem.st.relaxed.sys.global.b64 [%0], %1;" ::"l"(p),
+                         "l"(*reinterpret_cast<unsigned long long*>(&v))
+                         : "memory");
+            return;
+        }
+    }
+    *p = v;
+}
+
 template <typename T, int NST>
 __global__ void __launch_bounds__(kConsumers + 32)
 write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const int64_t* __restrict__ tile_counts,
@@ -336,12 +357,20 @@ write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const in
                 const int st = seq % NST;
                 dev::mbar_wait(&full[st], (seq / NST) & 1);
                 const T* V = reinterpret_cast<const T*>(ring + st * kStageBytes);
-                for (int d = 0; d < push.n; ++d) {
-                    T* const pd = static_cast<T*>(push.p[d]) + w0 * 32;
+                if (push.mc) {  // one store per dirty element, to every replica at once
 #pragma unroll
                     for (int j = warp; j < SCW; j += kConsumers / 32) {
                         const int i = q * SCW + j;
-                        if ((W[kPad + i] >> lane) & 1u) pd[i * 32 + lane] = V[j * 32 + lane];
+                        if ((W[kPad + i] >> lane) & 1u) push_store(push, 0, (w0 + i) * 32 + lane, V[j * 32 + lane]);
+                    }
+                } else {
+                    for (int d = 0; d < push.n; ++d) {
+                        T* const pd = static_cast<T*>(push.p[d]) + w0 * 32;
+#pragma unroll
+                        for (int j = warp; j < SCW; j += kConsumers / 32) {
+                            const int i = q * SCW + j;
+                            if ((W[kPad + i] >> lane) & 1u) pd[i * 32 + lane] = V[j * 32 + lane];
+                        }
                     }
                 }
                 __syncwarp();
@@ -360,7 +389,7 @@ write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const in
                         const T v = V[j * 32 + lane];
                         if (keep) tile_payload[spre[i] + __popc(m & lt)] = v;
                         const int64_t e = (w0 + i) * 32 + lane;
-                        for (int d = 0; d < push.n; ++d) static_cast<T*>(push.p[d])[e] = v;
+                        for (int d = 0; d < push.n; ++d) push_store(push, d, e, v);
                     }
                 }
                 __syncwarp();
@@ -381,7 +410,7 @@ write_pipe_k(uint32_t* __restrict__ l1, int64_t nwords, int64_t extent, const in
                     if ((m[u] >> lane) & 1u) {
                         if (keep) tile_payload[spre[base + u] + __popc(m[u] & lt)] = v[u];
                         const int64_t e = (w0 + base + u) * 32 + lane;
-                        for (int d = 0; d < push.n; ++d) static_cast<T*>(push.p[d])[e] = v[u];
+                        for (int d = 0; d < push.n; ++d) push_store(push, d, e, v[u]);
                     }
             }
         }

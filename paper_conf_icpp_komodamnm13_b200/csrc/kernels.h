@@ -21,6 +21,7 @@ constexpr int kMaxPtrs = 64;
 struct PtrList {
     void* p[kMaxPtrs];
     int n;
+    int mc;  // 1: p[0] is an NVLS multicast address (one multimem.st reaches every bound replica)
 };
 
 // Predicted-halo push of a row-block body: rows [lo[k], hi[k]) of its output are stored also into

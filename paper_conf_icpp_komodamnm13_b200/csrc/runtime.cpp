@@ -20,6 +20,8 @@
 #include "accmg.h"
 
 #include <cuda_runtime_api.h>
+#include <fcntl.h>
+#include <unistd.h>
 
 #include <algorithm>
 #include <cstdio>
@@ -32,6 +34,7 @@
 #include "intervals.h"
 #include "kernels.h"
 #include "nccl_dl.h"
+#include "vmm.h"
 
 using accmg::IntervalSet;
 using accmg::Ival;
@@ -79,6 +82,14 @@ struct accmg_region_s {
     int64_t* acc = nullptr;          // local reduction accumulator (P2P mode)
     std::vector<void*> opened;       // IPC mappings of the peers' replicas (re-opened when a hull grows)
     std::vector<void*> opened_partial;  // IPC mappings of the peers' reduction partials (opened once)
+    // §8 row f3 (config.multicast, P2P mode): the replica is a driver-VMM allocation shared with the
+    // peers through file descriptors (vpeer: their replicas mapped here), and, where the node can
+    // create one, bound to an NVLS multicast object mapped at mcmap
+    bool vmm = false;
+    accmg::vmm::Phys vphys;
+    std::vector<accmg::vmm::Map> vpeer;
+    unsigned long long mc = 0;
+    accmg::vmm::Map mcmap;
 };
 
 namespace {
@@ -135,9 +146,12 @@ struct State {
     struct Acct {
         int64_t esize, ce;
         int slot;
+        bool mc;
     };
     std::vector<Acct> pend;
     int64_t* h_acct = nullptr;  // kAcctSlots x 4 int64 (pinned)
+    bool mc_ok = false;         // multicast AUTO and the node can create multicast objects
+    std::string mc_why;
 };
 constexpr int kAcctSlots = 4096;
 
@@ -301,7 +315,7 @@ struct ProfScope {
 
 // Bytes of one partition's packet of undeclared writes (runs, elements, dirty chunks), delivered to
 // the P-1 other partitions (reading W8; booked by the sending process).
-void book_packet(int64_t runs, int64_t elems, int64_t chunks, int64_t es, int64_t ce, bool multi) {
+void book_packet(int64_t runs, int64_t elems, int64_t chunks, int64_t es, int64_t ce, bool multi, bool mc = false) {
     const int64_t hdr = 16 + 16 * runs, pay = es * elems;
     S.st.bytes_undeclared_headers += (S.P - 1) * hdr;
     S.st.bytes_undeclared_payload += (S.P - 1) * pay;
@@ -313,6 +327,10 @@ void book_packet(int64_t runs, int64_t elems, int64_t chunks, int64_t es, int64_
         const int64_t nr = (int64_t)(S.W - 1 + (S.nccl_all ? 1 : 0)) * (hdr + pay);
         S.st.bytes_link += nr + (int64_t)(S.V - 1) * pay;
         S.st.bytes_link_remote += nr;
+    } else if (mc) {  // one multimem store per dirty element; the switch replicates it
+        S.st.bytes_link += pay;
+        S.st.bytes_link_remote += pay;
+        S.st.bytes_multicast += pay;
     } else {      // the write pass stores each dirty element into the P-1 other replicas
         S.st.bytes_link += (int64_t)(S.P - 1) * pay;
         if (S.p2p) S.st.bytes_link_remote += (int64_t)(S.P - S.V) * pay;
@@ -329,7 +347,7 @@ int flush_acct() {
             S.pend.clear();
             return fail(ACCMG_ECUDA, "compaction: run starts != run ends", true);
         }
-        book_packet(v[0], v[1], v[2], a.esize, a.ce, false);
+        book_packet(v[0], v[1], v[2], a.esize, a.ce, false, a.mc);
     }
     S.pend.clear();
     return 0;
@@ -348,6 +366,81 @@ int collect_prof() {
     }
     S.prof.clear();
     return 0;
+}
+
+// ---- §8 row f3: VMM replicas shared through descriptors, NVLS multicast binding --------------------
+// Collective (every rank takes the same decision: it depends on the config, the global validity
+// tables and the init-time probe). Allocates the whole region on every rank as a driver-VMM
+// allocation, maps every peer's replica here from its exported descriptor, and, with multicast
+// available, binds all replicas to one multicast object (rank 0 creates it) mapped at mcmap.
+int setup_vmm_region(accmg_region_s* r) {
+    std::string err;
+    const bool want_mc = S.cfg.multicast == ACCMG_MC_AUTO && S.mc_ok;
+    const size_t bytes = accmg::vmm::round_up(S.cfg.device, (size_t)(r->extent * r->esize), want_mc);
+    int fd = -1;
+    if (accmg::vmm::alloc(S.cfg.device, bytes, &r->vphys, &err) != 0 || accmg::vmm::export_fd(r->vphys, &fd, &err) != 0)
+        return fail(ACCMG_ECUDA, "multicast replica: " + err, true);
+    std::vector<int> fds((size_t)S.W, -1);
+    const bool shared = S.boot.allgather_fds(&fd, 1, fds.data(), &err);
+    ::close(fd);
+    if (!shared) return fail(ACCMG_ESTATE, err, true);
+    r->vpeer.assign((size_t)S.W, accmg::vmm::Map{});
+    for (int q = 0; q < S.W; ++q) {
+        if (q == S.rank) continue;
+        if (accmg::vmm::import_map(S.cfg.device, fds[q], bytes, &r->vpeer[q], &err) != 0)
+            return fail(ACCMG_ECUDA, "multicast replica: " + err, true);
+    }
+    r->vmm = true;
+    r->dev[0] = static_cast<uint8_t*>(r->vphys.ptr);
+    r->abase[0] = r->dev[0];
+    for (int g = 0; g < S.P; ++g) {
+        r->arange[g] = Ival{0, r->extent};
+        r->gdev[g] = g == S.rank ? r->dev[0] : static_cast<uint8_t*>(r->vpeer[g].ptr);
+    }
+    S.st.device_bytes_user += (int64_t)bytes;
+    if (!want_mc) return 0;
+    // the multicast object: rank 0 creates and exports it; its status travels in rank 0's slot
+    int* flag = static_cast<int*>(S.boot.slot(0));
+    int mfd = -1;
+    if (S.rank == 0) {
+        const bool ok = accmg::vmm::mc_create(S.W, bytes, &r->mc, &err) == 0 && accmg::vmm::mc_export_fd(r->mc, &mfd, &err) == 0;
+        *flag = ok ? 1 : 0;
+        if (!ok) S.mc_why = err;
+    }
+    if (!S.boot.barrier(&err)) return fail(ACCMG_ESTATE, err, true);
+    const bool created = *flag == 1;
+    if (!S.boot.barrier(&err)) return fail(ACCMG_ESTATE, err, true);  // the slot may be reused after this
+    if (!created) return 0;  // unicast pushes into the shared VMM replicas
+    int send = S.rank == 0 ? mfd : ::open("/dev/null", O_RDONLY | O_CLOEXEC);  // placeholder descriptor
+    std::vector<int> mfds((size_t)S.W, -1);
+    const bool got = S.boot.allgather_fds(&send, 1, mfds.data(), &err);
+    ::close(send);
+    if (!got) return fail(ACCMG_ESTATE, err, true);
+    for (int q = 1; q < S.W; ++q)
+        if (q != S.rank && mfds[q] >= 0) ::close(mfds[q]);
+    if (S.rank != 0 && accmg::vmm::mc_import(mfds[0], &r->mc, &err) != 0)
+        return fail(ACCMG_ECUDA, "multicast: " + err, true);
+    if (accmg::vmm::mc_add_device(r->mc, S.cfg.device, &err) != 0) return fail(ACCMG_ECUDA, "multicast: " + err, true);
+    if (!S.boot.barrier(&err)) return fail(ACCMG_ESTATE, err, true);  // every device added before any bind
+    if (accmg::vmm::mc_bind(r->mc, r->vphys, &err) != 0) return fail(ACCMG_ECUDA, "multicast: " + err, true);
+    if (accmg::vmm::mc_map(S.cfg.device, r->mc, bytes, &r->mcmap, &err) != 0)
+        return fail(ACCMG_ECUDA, "multicast: " + err, true);
+    if (!S.boot.barrier(&err)) return fail(ACCMG_ESTATE, err, true);
+    S.st.multicast_regions += 1;
+    return 0;
+}
+
+void free_vmm_region(accmg_region_s* r) {
+    std::string err;
+    for (auto& m : r->vpeer) accmg::vmm::release(&m);
+    if (r->mcmap.ptr) accmg::vmm::unmap_only(&r->mcmap);
+    accmg::vmm::mc_release(r->mc, S.cfg.device, r->vphys.bytes, r->mc != 0);
+    r->mc = 0;
+    S.boot.barrier(&err);  // no peer still maps this replica
+    S.st.device_bytes_user -= (int64_t)r->vphys.bytes;
+    accmg::vmm::release(&r->vphys);
+    r->abase.assign(r->abase.size(), nullptr);
+    r->vmm = false;
 }
 
 // ---- window-sized replicas (§8 row f4) -------------------------------------------------------------
@@ -823,6 +916,12 @@ int launch_body(int body, const accmg_bounds* bd, const accmg_access* d, const v
 k::PtrList push_list(accmg_region_s* r, int li) {
     const int g = first_local() + li;
     k::PtrList dl{};
+    if (r->mcmap.ptr) {  // NVLS: one multicast address for all replicas (global-index base)
+        dl.p[0] = r->mcmap.ptr;
+        dl.n = 1;
+        dl.mc = 1;
+        return dl;
+    }
     if (S.p2p) {
         for (int h = 0; h < S.P; ++h)
             if (h != g) dl.p[dl.n++] = r->gdev[h];
@@ -883,7 +982,7 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
                 Trk& t = r->trk[li];
                 const int slot = (int)S.pend.size();
                 CUDA_TRY(cudaMemcpyAsync(S.h_acct + 4 * slot, t.totals, 32, cudaMemcpyDeviceToHost, S.stream));
-                S.pend.push_back({r->esize, chunk_elems(r), slot});
+                S.pend.push_back({r->esize, chunk_elems(r), slot, r->mcmap.ptr != nullptr});
                 CUDA_TRY(k::compact_write(t.l1, t.nwords, r->extent, t.ntiles, t.tile_counts, t.tile_offs, t.tile_edges,
                                           r->dev[li], (int)r->esize, nullptr, 0, push_list(r, li), S.stream,
                                           &S.st.kernel_launches, 0));
@@ -989,7 +1088,7 @@ int propagate_dirty(const std::vector<accmg_region_s*>& regs) {
         for (int g = 0; g < S.P; ++g)
             if (local(g))
                 book_packet(runs[ri * S.P + g], elems[ri * S.P + g], chunks[ri * S.P + g], regs[ri]->esize,
-                            chunk_elems(regs[ri]), multi);
+                            chunk_elems(regs[ri]), multi, regs[ri]->mcmap.ptr != nullptr);
     // 4. exchange + scatter
     ProfScope ps(2);
     if (!multi) return 0;  // pushed into every other replica by the write pass
@@ -1089,6 +1188,7 @@ void free_region(accmg_region_s* r) {
             std::string err;
             S.boot.barrier(&err);
         }
+        if (r->vmm) free_vmm_region(r);
         for (int li = 0; li < (int)r->abase.size(); ++li)
             if (r->abase[li]) {
                 const Ival& a = r->arange[first_local() + li];
@@ -1158,6 +1258,8 @@ int accmg_init(const accmg_config* cfg) {
     S.chunks = c.dirty_protocol == ACCMG_DIRTY_CHUNKS;
     if (c.halo_mode != ACCMG_HALO_AUTO && c.halo_mode != ACCMG_HALO_PULL)
         return fail(ACCMG_EINVAL, "init: bad halo_mode", false);
+    if (c.multicast != ACCMG_MC_OFF && c.multicast != ACCMG_MC_AUTO && c.multicast != ACCMG_MC_VMM)
+        return fail(ACCMG_EINVAL, "init: bad multicast", false);
     S.halo_pull = c.halo_mode == ACCMG_HALO_PULL;
     if (S.chunks && S.use_nccl) return fail(ACCMG_EUNSUPPORTED, "init: the chunk protocol needs a same-node transport", false);
     if (S.dry) {
@@ -1184,6 +1286,10 @@ int accmg_init(const accmg_config* cfg) {
         CUDA_TRY(cudaDeviceSynchronize());
         std::vector<void*> mine{S.sig};
         TRY(exchange_ptrs(mine, S.peer_sig, S.sig_opened));
+        if (c.multicast == ACCMG_MC_AUTO && S.V == 1) {
+            // the same answer on every rank of the node; a failure later still falls back per region
+            S.mc_ok = accmg::vmm::mc_probe(S.W, 2u << 20, &S.mc_why) == 0;
+        }
     }
     if (S.use_nccl) {
         const char* why = nullptr;
@@ -1378,6 +1484,17 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
                 for (int h = 0; h < g; ++h)
                     if (need[i][g].overlaps(need[i][h]))
                         return fail(ACCMG_ECONFLICT, "declared write windows of two partitions overlap (G14)", false);
+    // §8 f3: arrays written without a declared pattern get VMM replicas shared through descriptors
+    // (and a multicast binding where available) at their first allocation
+    if (S.p2p && S.V == 1 && S.cfg.multicast != ACCMG_MC_OFF)
+        for (int i = 0; i < n_descs; ++i) {
+            accmg_region_s* r = descs[i].region;
+            bool fresh = !r->vmm;
+            for (int g = 0; g < S.P && fresh; ++g) fresh = r->arange[g].hi <= r->arange[g].lo;
+            if (fresh && (descs[i].mode & ACCMG_W) && descs[i].mode != ACCMG_REDUCE_SUM && !descs[i].declared &&
+                (r->esize == 4 || r->esize == 8))
+                TRY(setup_vmm_region(r));
+        }
     // window-sized replicas: every partition's allocation covers what it needs (f4)
     for (int i = 0; i < n_descs; ++i) TRY(ensure_alloc(descs[i].region, need[i], descs[i].declared ? descs[i].stride : 0));
     // 3. data loader: plan all pulls from the pre-phase state, then run them
@@ -1610,6 +1727,21 @@ int accmg_set_profile(int on) {
 }
 
 const char* accmg_last_error(void) { return S.err.c_str(); }
+
+int accmg_multicast_probe(int num_devices, char* why, int cap) {
+    if (num_devices < 1 || cap < 0) return fail(ACCMG_EINVAL, "multicast_probe: bad arguments", false);
+    std::string w;
+    int ok = 0;
+    if (cudaFree(nullptr) != cudaSuccess) {  // context of the current device
+        w = "no CUDA device";
+    } else {
+        ok = accmg::vmm::mc_probe(num_devices, 2u << 20, &w) == 0 ? 1 : 0;
+    }
+    if (why && cap > 0) {
+        std::snprintf(why, (size_t)cap, "%s", ok ? "" : w.c_str());
+    }
+    return ok;
+}
 
 void* accmg_stream(void) { return S.init ? (void*)S.stream : nullptr; }
 

@@ -1,6 +1,6 @@
 """One rank of a multi-process (one process per GPU) run, used by tests/test_gpu_multiproc.py.
 
-usage: python tests/mp_worker.py RANK WORLD V UID_HEX WORKLOAD OUTDIR [EXCHANGE_MODE [DEVICE]]
+usage: python tests/mp_worker.py RANK WORLD V UID_HEX WORKLOAD OUTDIR [EXCHANGE_MODE [DEVICE [MULTICAST]]]
 Runs the workload through the C ABI with world_size = WORLD, num_partitions = WORLD * V, and
 saves its host arrays (after sync_to_host) and its stats under OUTDIR/rank<R>_*.npy/.json.
 DEVICE defaults to 0; the launching test passes rank % device_count (one process per GPU on a
@@ -26,7 +26,8 @@ def main():
     work, out = sys.argv[5], sys.argv[6]
     mode = int(sys.argv[7]) if len(sys.argv) > 7 else A.XCHG_AUTO
     device = int(sys.argv[8]) if len(sys.argv) > 8 else 0
-    A.accmg_init(num_partitions=world * V, world_size=world, rank=rank, device=device, nccl_unique_id=uid,
+    mc = int(sys.argv[9]) if len(sys.argv) > 9 else A.MC_OFF
+    A.accmg_init(num_partitions=world * V, world_size=world, rank=rank, device=device, nccl_unique_id=uid, multicast=mc,
                  exchange_mode=mode, dirty_chunk_bytes=8192)
     res = {}
     if work in ("jacobi_decl", "jacobi_undecl"):

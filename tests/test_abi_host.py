@@ -210,6 +210,14 @@ def test_state_errors():
     with pytest.raises(A.AccmgError) as e:
         A.accmg_init(num_partitions=1, device=-1, dirty_chunk_bytes=1000)
     assert e.value.code == A.EINVAL
+    with pytest.raises(A.AccmgError) as e:
+        A.accmg_init(num_partitions=1, device=-1, dirty_chunk_bytes=128)   # the header's minimum is 256
+    assert e.value.code == A.EINVAL
+    with pytest.raises(A.AccmgError) as e:
+        A.accmg_init(num_partitions=1, device=-1, multicast=7)
+    assert e.value.code == A.EINVAL
+    A.accmg_init(num_partitions=2, device=-1, multicast=A.MC_AUTO)  # dry run: accepted, nothing to bind
+    A.accmg_finalize()
 
 
 def test_scatter_requires_declared_dst(dry):

@@ -29,14 +29,14 @@ def _device_count():
     return torch.cuda.device_count()
 
 
-def _launch(world, V, work, tmp_path, mode=0, devices=None):
+def _launch(world, V, work, tmp_path, mode=0, devices=None, multicast=0):
     """One process per rank; rank r runs on devices[r] (default r % device_count: one GPU per rank
     on a multi-GPU box, all ranks on the one GPU otherwise)."""
     uid = os.urandom(128).hex()
     nd = _device_count()
     devices = devices or [r % nd for r in range(world)]
     procs = [subprocess.Popen([sys.executable, os.path.join(ROOT, "tests", "mp_worker.py"), str(r), str(world), str(V),
-                               uid, work, str(tmp_path), str(mode), str(devices[r])], cwd=ROOT)
+                               uid, work, str(tmp_path), str(mode), str(devices[r]), str(multicast)], cwd=ROOT)
              for r in range(world)]
     for p in procs:
         assert p.wait(timeout=600) == 0
@@ -179,3 +179,61 @@ def test_sync_to_host_right_after_loops(tmp_path, world, V):
     for r in range(world):
         assert np.array_equal(np.load(tmp_path / f"rank{r}_A.npy"), oA)
         assert np.array_equal(np.load(tmp_path / f"rank{r}_B.npy"), oB)
+
+
+def _expect(work):
+    if work.startswith("jacobi"):
+        N, S = 300, 6
+        A0 = gen.jacobi_field(5, N)
+        oA, oB = A0.copy(), A0.copy()
+        oracle.jacobi_run(oA, oB, S)
+        return {"A": oA, "B": oB}
+    n = (1 << 20) + 4321
+    src = (gen.u_fill(21, 0, n) >> np.uint64(40)).astype(np.float32) * np.float32(2.0 ** -24)
+    out = np.full(n, -1.0, dtype=np.float32)
+    for seed, dens, run in ((22, 0.5, 1), (23, 0.3, 70001), (24, 0.9, 40)):
+        oracle.masked_write(src, gen.write_mask(seed, n, dens, run), out)
+    return {"out": out}
+
+
+@pytest.mark.parametrize("work", ["jacobi_undecl", "masked"])
+def test_vmm_replicas_shared_through_descriptors(tmp_path, work):
+    """§8 f3 plumbing without the switch (ACCMG_MC_VMM): replicas of arrays written without a
+    declared pattern are driver-VMM allocations, exported as file descriptors, passed between the
+    processes over Unix sockets and mapped by every peer; the compaction pass pushes the dirty
+    elements into them. Two processes, bit-exact on both."""
+    from paper_conf_icpp_komodamnm13_b200 import accmg as A
+    stats = _launch(2, 1, work, tmp_path, multicast=A.MC_VMM)
+    for r in range(2):
+        for k, v in _expect(work).items():
+            assert np.array_equal(np.load(tmp_path / f"rank{r}_{k}.npy"), v), (r, k)
+    tot = stats if isinstance(stats[0], dict) and "multicast_regions" in stats[0] else [s["total"] for s in stats]
+    assert all(s["multicast_regions"] == 0 for s in tot)
+
+
+@pytest.mark.parametrize("work", ["jacobi_undecl", "masked"])
+def test_nvls_multicast_push(tmp_path, work):
+    """§8 f3: ACCMG_MC_AUTO — where the node can create an NVLS multicast object over the ranks'
+    GPUs, the compaction pass stores every dirty element once through the multicast address
+    (multimem.st) into all replicas; elsewhere the same run falls back to unicast pushes. Bit-exact
+    either way; the multicast assertions are skipped with the probe's reason when unavailable."""
+    from paper_conf_icpp_komodamnm13_b200 import accmg as A
+    nd = _device_count()
+    ok, why = A.accmg_multicast_probe(min(nd, 2))
+    stats = _launch(2, 1, work, tmp_path, multicast=A.MC_AUTO)
+    for r in range(2):
+        for k, v in _expect(work).items():
+            assert np.array_equal(np.load(tmp_path / f"rank{r}_{k}.npy"), v), (r, k)
+    tot = stats if "multicast_regions" in stats[0] else [s["total"] for s in stats]
+    if not (ok and nd >= 2):
+        assert all(s["multicast_regions"] == 0 for s in tot)
+        pytest.skip(f"NVLS multicast unavailable here (fell back to unicast pushes, bit-exact): {why or 'one GPU'}")
+    assert all(s["multicast_regions"] >= 1 for s in tot)
+    assert sum(s["bytes_multicast"] for s in tot) > 0
+
+
+def test_multicast_probe_reports():
+    from paper_conf_icpp_komodamnm13_b200 import accmg as A
+    ok, why = A.accmg_multicast_probe(1)
+    assert isinstance(ok, bool)
+    assert ok or why
