@@ -1,4 +1,4 @@
-// Deep-halo body, register-streamed (§8 row f2; ACCMG_DEEP_IMPL = 2, the default).
+// Deep-halo body, register-streamed (§8 row f2; the implementation for h <= 8, cols % 4 == 0).
 //
 // Temporal blocking along the streaming dimension: one warp owns a 128-column strip (4 columns per
 // lane: TK = 128 - 2*hc outputs plus hc >= h halo columns per side) and a segment of L output rows,
