@@ -9,13 +9,14 @@
 //     A = [x0 | x0 | x1 | 1 1 1], B = [c0 | c1 | c0 | h0 h1 h2] (bf16 pieces: x = x0 + x1 + e with
 //     |e| <= 2^-16 |x|, -|c|^2/2 = h0 + h1 + h2), four tcgen05.mma.kind::f16 (K = 64) give
 //     v = x0.c0 + x0.c1 + x1.c0 - |c|^2/2 in TMEM, fp32, one 128-column half of the centroids per
-//     accumulator; each half is handed back to the MMA warp as soon as the epilogue has read it,
-//     so the next tile's MMAs of that half overlap the epilogue's remaining work;
+//     accumulator (a ring of three 128-column TMEM slots), so the next tile's MMAs overlap the
+//     epilogue's reads of this one;
 //   * reductiontoarray: sums[c][(j, b)] = sum_p onehot[c][p] * byte_b(x[p][j] * 2^shift + 2^31) and
 //     counts[c] = sum_p onehot[c][p] * 1 — tcgen05.mma.kind::i8 (u8 x u8 -> s32, exact) with
 //     A = the one-hot assignment matrix [128 clusters][128 points] and B = the points' fixed-point
-//     byte planes [80 rows][128 points]; the s32 accumulators stay in TMEM across all the CTA's
-//     tiles and are read once at the end (no atomics per point).
+//     byte planes [64 rows (j, b)][128 points] (MN-major: a point's 64 bytes are its 16 words); the
+//     s32 accumulators stay in TMEM across all the CTA's tiles and are read once at the end; the
+//     counts are shared-memory integer atomics (no per-point global atomics).
 // Exactness of the assignment: every c with v(c) >= vmax - T is a candidate and is re-evaluated
 // with the exact fmaf chain (ascending c, strict <), T a rigorous bound of the filter error:
 // with Cinf = max |cen|, C2 = max |c|^2, L1 = sum |x_j|, Q = sum x_j^2,
@@ -27,17 +28,17 @@
 // D_f(c^), it can neither win nor tie. Inputs are on the 2^-shift grid (W4). CPU pins of this
 // reading: tests/test_kmeans_filter_bound.py.
 //
-// Warp roles (one CTA per SM, persistent over 128-point tiles):
+// Warp roles (one CTA per SM, persistent over 128-point tiles; 16 warps):
 //   w0 producer: TMA load (64-byte swizzle) of the tile's fp32 rows (8 KiB) into an mbarrier ring;
-//   w1 MMA issuer (one thread): distance MMAs of tile i, then the reduction MMAs of tile i-1;
+//   w15 / w1 distance-MMA issuers (centroid halves 0 / 1), w14 reduction-MMA issuer (one tile behind);
 //   w2-5 converters (one point per thread): bf16 pieces of x into the distance A operand, the
-//        fixed-point bytes into the reduction B operand, the 2^-shift grid check, the point's
+//        fixed-point words into the reduction B operand, the 2^-shift grid check, the point's
 //        bound terms E and Q(1 + 2^-17) + 2E for the epilogue;
-//   w6-9 epilogue (one point per thread = TMEM lane): pass 1 = maxima of 4-column groups (3-input
-//        FMNMX) over all k columns, then a candidate-group mask (sign bits of thr - max, packed
-//        FSUB2, funnel-shifted), the exact re-check of the candidate groups (packed FADD2 / FFMA2,
-//        each lane rounding like the scalar op), member[p] and the point's one-hot byte.
-// Same-box A/B measurements of the alternatives tried: profiles/r01/kmeans_tc.log.
+//   w6-13 epilogue, two sets of four (one per centroid half; warp % 4 = TMEM lane quarter, one point
+//        per thread): maxima over the orthogonal column groupings, one exchange of the halves'
+//        maxima and verdicts, the exact re-check only when the candidate is not proved unique,
+//        member[p], the count atomic and the point's one-hot byte.
+// DESIGN.md §6 has the measurements behind this layout.
 #include <cuda_bf16.h>
 
 #include <cstdio>
@@ -68,7 +69,7 @@ constexpr int OS = 2;                   // one-hot stages
 constexpr int kRows = 64;               // reduction B rows: 16 dims x 4 bytes (counts: shared atomics)
 constexpr int kXBytes = TM * 64;        // 8 KiB
 constexpr int kADBytes = TM * 128;      // 16 KiB
-constexpr int kABBytes = kRows * 128;   // 8 KiB
+constexpr int kABBytes = kRows * TM;    // 8 KiB: MN-major, point p's 64 bytes (16 dims x 4 bytes) at row p
 constexpr int kOHBytes = KMAX * 128;    // 32 KiB (two 128-cluster halves)
 constexpr int QW = 128;                 // centroid columns per distance accumulator (one MMA N)
 constexpr int NDB = 3;                  // distance accumulators: a ring of three 128-column halves
@@ -96,10 +97,7 @@ constexpr int OFF_BAR = OFF_PC + (KMAX / 4) * kGrpBytes;
 constexpr int kNumBars = 2 * XS + 2 * AS + BS + 2 * NDB + 2 * OS + 2;
 constexpr int OFF_MISC = OFF_BAR + kNumBars * 8;    // tmem slot, Cinf bits, C2 bits
 constexpr int OFF_EQ = OFF_MISC + 16;               // float2 [BS][TM]: the point's E and Q (1 + 2^-17) + 2E
-// epilogue half exchange, double-buffered by tile parity: maxima [2][2][TM], verdicts [2][2][TM];
-// half-1 winner of a re-check (d [TM], c [TM])
-constexpr int OFF_EX = OFF_EQ + BS * TM * 8;
-constexpr int OFF_CNT = OFF_EX + 10 * TM * 4;       // int32 [KMAX]: the CTA's cluster counts
+constexpr int OFF_CNT = OFF_EQ + BS * TM * 8;       // int32 [KMAX]: the CTA's cluster counts
 constexpr int kSmemTC = OFF_CNT + KMAX * 4 + 1024;  // + alignment slack
 static_assert(OFF_AB % 1024 == 0 && OFF_BD % 1024 == 0 && OFF_OH % 1024 == 0 && OFF_X % 1024 == 0, "align");
 static_assert(kColSum + 2 * kRows <= kTmemCols, "tmem");
@@ -156,6 +154,17 @@ __device__ __forceinline__ uint64_t sdesc_sw128(uint32_t saddr) {
     d |= (uint64_t)(1024 >> 4) << 32;
     d |= (uint64_t)1 << 46;
     d |= (uint64_t)2 << 61;
+    return d;
+}
+// MN-major operand, 64-byte swizzle, N = 64 one-byte elements: K row p (64 B) at 64 p, 8-row atoms
+// 512 B apart (SBO); one atom along N, so the leading-dimension offset is never stepped
+__device__ __forceinline__ uint64_t sdesc_mn_sw64(uint32_t saddr) {
+    uint64_t d = 0;
+    d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+    d |= (uint64_t)(kABBytes >> 4) << 16;
+    d |= (uint64_t)(512 >> 4) << 32;
+    d |= (uint64_t)1 << 46;
+    d |= (uint64_t)4 << 61;
     return d;
 }
 // byte offset of element k (byte k) of row m in a 128-byte-swizzled K-major operand
@@ -496,8 +505,9 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
     } else if (warp == kRedWarp) {
         // ---- reductiontoarray MMAs (u8 one-hot x byte planes -> s32), one tile behind the
         // epilogue's one-hot bytes
-        const uint32_t idesc_sum = (2u << 4) | ((uint32_t)(kRows >> 3) << 17) | ((uint32_t)(TM >> 4) << 24);
-        const uint64_t dAB = sdesc_sw128(sAB), dOH = sdesc_sw128(sOH);
+        // u8 x u8 -> s32, B (the byte planes) MN-major
+        const uint32_t idesc_sum = (2u << 4) | (1u << 16) | ((uint32_t)(kRows >> 3) << 17) | ((uint32_t)(TM >> 4) << 24);
+        const uint64_t dAB = sdesc_mn_sw64(sAB), dOH = sdesc_sw128(sOH);
         for (uint32_t j = 0; j < nt32; ++j) {
             const int o = (int)(j % OS);
             mbar_wait_sleep(&ofull[o], (uint32_t)((j / OS) & 1));
@@ -513,7 +523,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
 #pragma unroll
                 for (int k = 0; k < 4; ++k)
                     mma_i8_elect(tmem + kColSum + (uint32_t)(kRows * h), oh + (uint64_t)((h * 16384 + k * 32) >> 4),
-                                 b + (uint64_t)((k * 32) >> 4), idesc_sum, (j | k) ? 1u : 0u);
+                                 b + (uint64_t)((k * 32 * kRows) >> 4), idesc_sum, (j | k) ? 1u : 0u);
             tc_commit_elect(&oempty[o]);
             tc_commit_elect(&bempty[j % BS]);
             KPR(9, j);
@@ -558,27 +568,27 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             // arrive alone does not wait for the shared-memory loads to return their data, and the
             // producer refills the stage as soon as all converters have arrived)
             mbar_arrive(&xempty[s]);
-            // fixed point x * 2^shift, biased to unsigned: u = v + 2^31; byte b of dim j -> row 4j + b
-            // row m = 4j + b has swizzle phase m & 7 = 4 (j & 1) + b: eight per-thread base addresses,
-            // the row offset m * 128 is the store's immediate (st.shared.u8 keeps the low byte)
-            const uint32_t ab = sAB + bs * kABBytes;
-            uint32_t base[8];
-#pragma unroll
-            for (int k = 0; k < 8; ++k) base[k] = ab + ((((uint32_t)r >> 4) ^ (uint32_t)k) << 4) + ((uint32_t)r & 15u);
-            // grid check without branches: v = x 2^shift must equal rint(v) (every float of magnitude
+            // fixed point x * 2^shift, biased to unsigned: u = v + 2^31. The B operand is MN-major: the
+            // point's 64 bytes in order (j, b) are its 16 words u_j, little-endian, so four 16-byte
+            // stores write the row (64-byte swizzle: chunk c of row r at c ^ ((r >> 1) & 3)).
+            // Grid check without branches: v = x 2^shift must equal rint(v) (every float of magnitude
             // >= 2^23 is an integer) and |v| < 2^31; the largest |v - rint(v)| and |v| of the point
             // are tested once
             float fr = 0.f, vm = 0.f;
+            uint32_t uw[16];
 #pragma unroll
             for (int j = 0; j < 16; ++j) {
                 const float v = xv[j] * scale;  // exact: power-of-two scaling
                 const float rv = rintf(v);
                 fr = fmaxf(fr, fabsf(v - rv));  // exact difference (Sterbenz)
                 vm = fmaxf(vm, fabsf(v));
-                const uint32_t u = (uint32_t)__float2int_rn(rv) ^ 0x80000000u;
+                uw[j] = (uint32_t)__float2int_rn(rv) ^ 0x80000000u;
+            }
+            {
+                const uint32_t row = sAB + bs * kABBytes + (uint32_t)r * 64u, sw = ((uint32_t)r >> 1) & 3u;
 #pragma unroll
-                for (int b = 0; b < 4; ++b)
-                    sts_u8(base[4 * (j & 1) + b] + (uint32_t)((4 * j + b) * 128), u >> (8 * b));
+                for (int c = 0; c < 4; ++c)
+                    sts_v4(row + (((uint32_t)c ^ sw) << 4), make_uint4(uw[4 * c], uw[4 * c + 1], uw[4 * c + 2], uw[4 * c + 3]));
             }
             bad |= (fr != 0.f) | !(vm < 2147483648.0f);
             {  // the filter bound's per-point terms, for the epilogue (header: E, Dhat)
@@ -597,72 +607,63 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
         }
         if (bad) atomicOr(err, 1);
     } else if (warp >= 6 && warp < 14) {
-        // ---- epilogue, orthogonal groupings: point row r = TMEM lane; warp set `half` reads the
-        // 128 columns of centroids [128 half, 128 half + 128). Local column l = 16 b + a: the
-        // b-groups (16 consecutive columns, 8 per half) and the a-groups (columns with the same
-        // l mod 16, 16 per half) partition the columns two ways and (a, b) names one column, so
-        // when exactly one a-group and one b-group reach the threshold the candidate set is that
-        // single column: the argmin is proved without any re-check (the common case for separated
-        // clusters). Otherwise every 4-column group of the product set (candidate b-groups x
-        // quarters holding candidate a-groups) is re-checked with the exact fmaf chain.
+        // ---- epilogue: two sets of four warps take alternate tiles (set = tile parity), so each
+        // set has two tile periods for its tile and the sets never wait for each other. Point row
+        // r = TMEM lane (warp % 4 = lane quarter); the thread reads all k columns of its point
+        // (one 128-column ring slot per half, freed as soon as it is read) and keeps the maxima of
+        // two orthogonal column groupings of the 16 x 16 grid l = 16 b + a: b-groups (16
+        // consecutive columns) and a-groups (columns with the same l mod 16). (a, b) names one
+        // column, so when exactly one a-group and one b-group reach the threshold the candidate
+        // set is that single column: the argmin is proved without any re-check (the common case
+        // for separated clusters). Otherwise every 4-column group of the product set (candidate
+        // b-groups x quarters holding candidate a-groups) is re-checked with the exact fmaf chain.
         const int q = warp & 3;
         const int r = q * 32 + lane;
-        const int half = (warp - 6) >> 2;
-        float* exv0 = reinterpret_cast<float*>(smem + OFF_EX);  // [parity][half][TM] half maxima
-        int* exs0 = reinterpret_cast<int*>(exv0 + 4 * TM);      // [parity][half][TM] local verdicts
-        float* exd = exv0 + 8 * TM;                              // [TM] half-1 winner distance (re-check)
-        int* exi = reinterpret_cast<int*>(exv0 + 9 * TM);        // [TM] half-1 winner index (re-check)
-        int* s_cnt = reinterpret_cast<int*>(smem + OFF_CNT);   // the CTA's cluster counts
-        int32_t pend[OS];
-#pragma unroll
-        for (int o = 0; o < OS; ++o) pend[o] = -1;
-        const bool have = half < nq;  // this half holds centroids
-        const int ncq = have ? (((npad - QW * half) < QW ? (npad - QW * half) : QW) / 32) : 0;
+        const int half = (warp - 6) >> 2;  // the set (also its share of the final readout)
+        const int o = half;                // one-hot stage of the set's tiles (tile parity)
+        int* s_cnt = reinterpret_cast<int*>(smem + OFF_CNT);  // the CTA's cluster counts
+        int32_t pend = -1;                 // the one-hot byte this thread set in its stage
         const uint32_t tq = tmem + ((uint32_t)(q * 32) << 16);
-        for (uint32_t i = 0; i < nt32; ++i) {
+        for (uint32_t i = (uint32_t)half; i < nt32; i += 2) {
             const uint32_t t = blockIdx.x + i * gridDim.x;
-            const int s = (int)(i % XS);
             const uint32_t pr = t * TM + (uint32_t)r;  // row within the partition (< 2^31)
             const int64_t p = p0 + pr;
             const bool valid = pr < (uint32_t)(p1 - p0);
             KTR(KTR_EPI, 9);
             KTR(KTR_EPI + 4, 21);
             KPR(15, i);
-            float am[16], bm[8];
+            float am[16], bm[16];
 #pragma unroll
             for (int a = 0; a < 16; ++a) am[a] = -0x1p120f;
 #pragma unroll
-            for (int b = 0; b < 8; ++b) bm[b] = -0x1p120f;
-            if (have) {
-                const uint32_t u = (uint32_t)nq * i + (uint32_t)half, db = u % NDB;
+            for (int b = 0; b < 16; ++b) bm[b] = -0x1p120f;
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                if (h >= nq) break;
+                const int ncq = ((npad - QW * h) < QW ? (npad - QW * h) : QW) / 32;
+                const uint32_t u = (uint32_t)nq * i + (uint32_t)h, db = u % NDB;
                 mbar_wait(&dfull[db], (u / NDB) & 1u);
                 tc_fence_after();
-                KTR(KTR_EPI, 11);
-                KTR(KTR_EPI + 4, 22);
+                if (h == 0) { KTR(KTR_EPI, 11); KTR(KTR_EPI + 4, 22); }
                 KPR(16, i);
                 const uint32_t tb = tq + QW * db;
-#ifdef KM_ONE_LD
-                constexpr int kLd = 1;
-#else
-                constexpr int kLd = 2;  // 32-column chunks per tcgen05.wait::ld
-#endif
 #pragma unroll
-                for (int c2 = 0; c2 < 4; c2 += kLd) {
+                for (int c2 = 0; c2 < 4; c2 += 2) {  // two 32-column chunks per tcgen05.wait::ld
                     uint32_t v[2][32];
                     if (c2 < ncq) tmem_ld<32>(tb + c2 * 32, v[0]);
-                    if (kLd == 2 && c2 + 1 < ncq) tmem_ld<32>(tb + (c2 + 1) * 32, v[1]);
+                    if (c2 + 1 < ncq) tmem_ld<32>(tb + (c2 + 1) * 32, v[1]);
                     tmem_wait();
 #pragma unroll
-                    for (int e = 0; e < kLd; ++e) {
+                    for (int e = 0; e < 2; ++e) {
                         const int c = c2 + e;
                         if (c < ncq) {
 #define VF(k) __uint_as_float(v[e][k])
-                            bm[2 * c] = max3(max3(max3(VF(0), VF(1), VF(2)), max3(VF(3), VF(4), VF(5)),
-                                                  max3(VF(6), VF(7), VF(8))),
-                                             max3(VF(9), VF(10), VF(11)), max3(VF(12), VF(13), fmaxf(VF(14), VF(15))));
-                            bm[2 * c + 1] = max3(max3(max3(VF(16), VF(17), VF(18)), max3(VF(19), VF(20), VF(21)),
-                                                      max3(VF(22), VF(23), VF(24))),
-                                                 max3(VF(25), VF(26), VF(27)), max3(VF(28), VF(29), fmaxf(VF(30), VF(31))));
+                            bm[8 * h + 2 * c] = max3(max3(max3(VF(0), VF(1), VF(2)), max3(VF(3), VF(4), VF(5)),
+                                                          max3(VF(6), VF(7), VF(8))),
+                                                     max3(VF(9), VF(10), VF(11)), max3(VF(12), VF(13), fmaxf(VF(14), VF(15))));
+                            bm[8 * h + 2 * c + 1] = max3(max3(max3(VF(16), VF(17), VF(18)), max3(VF(19), VF(20), VF(21)),
+                                                              max3(VF(22), VF(23), VF(24))),
+                                                         max3(VF(25), VF(26), VF(27)), max3(VF(28), VF(29), fmaxf(VF(30), VF(31))));
 #pragma unroll
                             for (int a = 0; a < 16; ++a) am[a] = max3(am[a], VF(a), VF(16 + a));
 #undef VF
@@ -671,31 +672,24 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                 }
                 tc_fence_before();
                 mbar_arrive(&dempty[db]);  // the ring slot may take another half
-            } else {
-                // a half without centroids still reads the converter's E, Q terms of this tile:
-                // order it after them through the other half's accumulator (waiting only)
-                mbar_wait_sleep(&dfull[i % NDB], (i / NDB) & 1u);
             }
             KTR(KTR_EPI, 12);
             KTR(KTR_EPI + 4, 23);
-            // this half's own threshold, from its own maximum vh: thr_h <= the global threshold
-            // (a smaller maximum only raises Dhat), so its local candidates include the global ones
-            const float vh = max3(max3(bm[0], bm[1], bm[2]), max3(bm[3], bm[4], bm[5]), fmaxf(bm[6], bm[7]));
+            const float vmax = max3(max3(max3(bm[0], bm[1], bm[2]), max3(bm[3], bm[4], bm[5]), max3(bm[6], bm[7], bm[8])),
+                                    max3(bm[9], bm[10], bm[11]), max3(bm[12], bm[13], fmaxf(bm[14], bm[15])));
             float E, Qa;  // from the converter (stage i % BS is recycled only after this tile's reduction)
             asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(E), "=f"(Qa)
                          : "r"(sbase + OFF_EQ + ((uint32_t)(i % BS) * TM + r) * 8) : "memory");
-            auto thr_of = [&](float vm) {  // candidate <=> value >= vm - T <=> > thr (next float below)
-                const float Dhat = fmaxf(Qa - 2.f * vm, 0.f);
-                const float T = (2.f * E + 0x1p-16f * Dhat) * 1.001f;
-                return next_below(vm - T);
-            };
-            const float thr_h = thr_of(vh);
-            KTR(KTR_EPI, 15);
-            // sign bits of thr - max (packed FSUB2, each lane rounds alone) funnel-shifted into masks
-            const uint64_t thr2 = pk2(thr_h, thr_h);
-            uint32_t mA0 = 0, mA1 = 0, mB = 0;  // bit 15 - a (a < 8 in mA0 << 8) / 7 - b
+            // candidate <=> value >= vmax - T <=> > thr (the next float below)
+            const float Dhat = fmaxf(Qa - 2.f * vmax, 0.f);
+            const float T = (2.f * E + 0x1p-16f * Dhat) * 1.001f;
+            const float thr = next_below(vmax - T);
+            // sign bits of thr - max (packed FSUB2, each lane rounds alone) funnel-shifted into the
+            // masks: bit 15 - a of mA, bit 15 - b of mB; two independent chains each
+            const uint64_t thr2 = pk2(thr, thr);
+            uint32_t mA0 = 0, mA1 = 0, mB0 = 0, mB1 = 0;
 #pragma unroll
-            for (int a = 0; a < 8; a += 2) {  // two independent funnel chains for the a-groups
+            for (int a = 0; a < 8; a += 2) {
                 float d0, d1, d2, d3;
                 upk2(sub2(thr2, pk2(am[a], am[a + 1])), d0, d1);
                 upk2(sub2(thr2, pk2(am[8 + a], am[9 + a])), d2, d3);
@@ -703,47 +697,20 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                 mA1 = __funnelshift_l(__float_as_uint(d2), mA1, 1);
                 mA0 = __funnelshift_l(__float_as_uint(d1), mA0, 1);
                 mA1 = __funnelshift_l(__float_as_uint(d3), mA1, 1);
+                upk2(sub2(thr2, pk2(bm[a], bm[a + 1])), d0, d1);
+                upk2(sub2(thr2, pk2(bm[8 + a], bm[9 + a])), d2, d3);
+                mB0 = __funnelshift_l(__float_as_uint(d0), mB0, 1);
+                mB1 = __funnelshift_l(__float_as_uint(d2), mB1, 1);
+                mB0 = __funnelshift_l(__float_as_uint(d1), mB0, 1);
+                mB1 = __funnelshift_l(__float_as_uint(d3), mB1, 1);
             }
-            const uint32_t mA = (mA0 << 8) | mA1;
-#pragma unroll
-            for (int b = 0; b < 8; b += 2) {
-                float d0, d1;
-                upk2(sub2(thr2, pk2(bm[b], bm[b + 1])), d0, d1);
-                mB = __funnelshift_l(__float_as_uint(d0), mB, 1);
-                mB = __funnelshift_l(__float_as_uint(d1), mB, 1);
-            }
-            // local verdict: 0 none, 1 + c single candidate c (global index: the half's maximum), -1 several
-            int verdict = 0;
-            if (mB) {
-                if (__popc(mA) == 1 && __popc(mB) == 1)
-                    verdict = 1 + 128 * half + 16 * (7 - (31 - __clz(mB))) + (15 - (31 - __clz(mA)));
-                else
-                    verdict = -1;
-            }
+            const uint32_t mA = ((mA0 << 8) | mA1) & 0xFFFFu, mB = ((mB0 << 8) | mB1) & 0xFFFFu;
             KTR(KTR_EPI, 16);
-            // one exchange per tile: both halves' maxima and local verdicts (slots by tile parity: a
-            // warp reaches the next tile's write before its partner has read this tile's values)
-            float* exv = exv0 + (i & 1) * 2 * TM;
-            int* exs = exs0 + (i & 1) * 2 * TM;
-            exv[half * TM + r] = vh;
-            exs[half * TM + r] = verdict;
-            KPR(17, i);
-            named_bar(1 + q, 64);
-            KPR(18, i);
-            KTR(KTR_EPI, 18);
-            KTR(KTR_EPI + 4, 24);
-            const float m0 = exv[r], m1 = exv[TM + r];
-            const int v0 = exs[r], v1 = exs[TM + r];
-            // global threshold (the same in both warps); a half has global candidates only if its
-            // maximum exceeds it, and then they are among its local ones: the argmin is unique when
-            // exactly one half does and that half's local verdict is a single column
-            const float thr = thr_of(fmaxf(m0, m1));
-            const bool in0 = m0 > thr, in1 = m1 > thr;
-            const bool unique = in0 != in1 && (in0 ? v0 : v1) > 0;
-            float bd = __int_as_float(0x7f800000);
-            int bi = unique ? (in0 ? v0 : v1) - 1 : 0;
-            if (__any_sync(0xffffffffu, !unique)) {  // warp-uniform in both warps of the pair
-                if (!unique && mB && (half == 0 ? in0 : in1)) {
+            const bool unique = __popc(mA) == 1 && __popc(mB) == 1;
+            int bi = unique ? 16 * (15 - (31 - __clz(mB))) + (15 - (31 - __clz(mA))) : 0;
+            if (__any_sync(0xffffffffu, !unique)) {  // warp-uniform
+                if (!unique) {
+                    float bd = __int_as_float(0x7f800000);
                     // the point's coordinates (global memory: the tile's stage may be recycled)
                     float xv[16];
                     const float4* xp = reinterpret_cast<const float4*>(xg + (valid ? p : p0) * 16);
@@ -752,19 +719,20 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                         const float4 v = xp[j];
                         xv[4 * j] = v.x; xv[4 * j + 1] = v.y; xv[4 * j + 2] = v.z; xv[4 * j + 3] = v.w;
                     }
-                    // 4-column groups of the product set, ascending: b-group lb, quarter qq of it
+                    // 4-column groups of the product set, ascending (with the strict < the lowest
+                    // index wins ties, as in the scalar loop): b-group lb, quarter qq of it
                     uint32_t quarters = 0;  // quarter k holds a-groups 4k..4k+3 (bits 15-4k..12-4k)
 #pragma unroll
                     for (int k = 0; k < 4; ++k) quarters |= ((mA >> (12 - 4 * k)) & 0xFu) ? (1u << k) : 0u;
                     uint32_t mb = mB;
                     while (mb) {
-                        const int lb = __clz(mb) - 24;  // bit 7 - lb
-                        mb &= ~(0x80u >> lb);
+                        const int lb = __clz(mb) - 16;  // bit 15 - lb
+                        mb &= ~(0x8000u >> lb);
                         uint32_t qs = quarters;
                         while (qs) {
                             const int qq = __ffs(qs) - 1;
                             qs &= qs - 1;
-                            const int G = 32 * half + 4 * lb + qq;  // global 4-centroid group
+                            const int G = 4 * lb + qq;  // 4-centroid group: centroids 16 lb + 4 qq ..
                             const uint32_t gb = sPC + G * kGrpBytes;
                             uint64_t acc0 = 0ull, acc1 = 0ull;  // (4G, 4G+1), (4G+2, 4G+3)
 #pragma unroll
@@ -792,46 +760,25 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                         }
                     }
                 }
-                // half 1 hands its winner to half 0; the lower half wins ties (lower indices)
-                if (half == 1) { exd[r] = bd; exi[r] = bi; }
-                KPR(19, i);
-                named_bar(1 + q, 64);
-                KPR(20, i);
-                if (half == 0 && !unique) {
-                    const float d1 = exd[r];
-                    if (d1 < bd) { bd = d1; bi = exi[r]; }
-                }
             }
             KTR(KTR_EPI, 17);
-            // member[] and the reductiontoarray count (the sums go through the MMA): half 1 when the
-            // winner is proved unique (both halves know it), half 0 after a re-check
-            if (valid && unique == (half == 1)) {
+            // member[] and the reductiontoarray count (the sums go through the MMA)
+            if (valid) {
                 member[p] = bi;
                 atomicAdd(&s_cnt[bi], 1);
             }
-            if (half == 1) continue;
-            // the point's one-hot byte (cluster row bi, point column r); the byte this thread set
-            // in this stage OS tiles ago is cleared first
-            const int o = (int)(i % OS);
+            // the point's one-hot byte (cluster row bi, point column r) in the set's stage; the
+            // byte this thread set there two tiles ago is cleared first
             KPR(21, i);
             mbar_wait(&oempty[o], (uint32_t)((i / OS) & 1) ^ 1u);
             KTR(KTR_EPI, 19);
-            int32_t& pd = (o == 0) ? pend[0] : pend[1];
-            if (pd >= 0) sts_u8(sOH + o * kOHBytes + (uint32_t)pd, 0u);
-            if (valid) {
-                const uint32_t off = (uint32_t)(bi >> 7) * 16384u + sw_off((uint32_t)(bi & 127), (uint32_t)r);
-                sts_u8(sOH + o * kOHBytes + off, 1u);
-                pd = (int32_t)off;
-            } else {
-                pd = -1;
-            }
+            if (pend >= 0) sts_u8(sOH + o * kOHBytes + (uint32_t)pend, 0u);
+            pend = valid ? (int32_t)((uint32_t)(bi >> 7) * 16384u + sw_off((uint32_t)(bi & 127), (uint32_t)r)) : -1;
+            if (valid) sts_u8(sOH + o * kOHBytes + (uint32_t)pend, 1u);
             fence_async_smem();
             mbar_arrive(&ofull[o]);
             KPR(22, i);
             KTR(KTR_EPI, 20);
-            KTR(7, 26);
-            KTR(8, 27);
-            KTR(9, 28);
         }
         // reduction accumulators: lane = cluster (h*128 + r), columns 4j+b = byte sums; counts
         // from the shared atomics (every epilogue warp has passed its last tile: named barrier)
