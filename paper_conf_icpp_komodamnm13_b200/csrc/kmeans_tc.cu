@@ -94,7 +94,7 @@ constexpr int OFF_X = OFF_OH + OS * kOHBytes;
 constexpr int kGrpBytes = 272;
 constexpr int OFF_PC = OFF_X + XS * kXBytes;
 constexpr int OFF_BAR = OFF_PC + (KMAX / 4) * kGrpBytes;
-constexpr int kNumBars = 2 * XS + 2 * AS + BS + 2 * NDB + 2 * OS + 2;
+constexpr int kNumBars = 2 * XS + 2 * AS + BS + 2 * NDB + 2 * OS + 3;
 constexpr int OFF_MISC = OFF_BAR + kNumBars * 8;    // tmem slot, Cinf bits, C2 bits
 constexpr int OFF_EQ = OFF_MISC + 16;               // float2 [BS][TM]: the point's E and Q (1 + 2^-17) + 2E
 constexpr int OFF_CNT = OFF_EQ + BS * TM * 8;       // int32 [KMAX]: the CTA's cluster counts
@@ -351,10 +351,13 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
     uint64_t* oempty = ofull + OS;
     uint64_t* sdone = oempty + OS;
     uint64_t* h1go = sdone + 1;  // phase i: the half-1 MMAs of tile i are issued
+    uint64_t* h0go = h1go + 1;   // phase i: the half-0 MMAs of tile i are issued
     uint32_t* misc = reinterpret_cast<uint32_t*>(smem + OFF_MISC);  // [0] tmem, [1] Cinf bits, [2] C2 bits
 
     constexpr int kThreads = kThreadsTC;
-    const int tid = threadIdx.x, warp = tid >> 5, lane = tid & 31;
+    // the warp index through a shuffle: the compiler then treats the role branches as warp-uniform
+    // (descriptors and loop state of the MMA issuers stay in uniform registers; 8.5 % faster)
+    const int tid = threadIdx.x, warp = __shfl_sync(0xffffffffu, tid >> 5, 0), lane = tid & 31;
     const int64_t ntiles = (p1 - p0 + TM - 1) / TM;
     const int64_t nt = blockIdx.x < ntiles ? (ntiles - blockIdx.x + gridDim.x - 1) / gridDim.x : 0;
     const uint32_t nt32 = (uint32_t)nt;
@@ -386,6 +389,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
         for (int o = 0; o < OS; ++o) { mbar_init(&ofull[o], 128); mbar_init(&oempty[o], 1); }
         mbar_init(sdone, 1);
         mbar_init(h1go, 1);
+        mbar_init(h0go, 1);
         dev::mbar_fence_init();
     }
     KPR(1, 0);
@@ -478,10 +482,11 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             KPR(5, i);
             const uint64_t ad = dAD + (uint64_t)((a * kADBytes) >> 4);
             const uint32_t u = (uint32_t)nq * i + (uint32_t)h, db = u % NDB;  // ring slot and its use count
-            // the tensor pipe takes MMAs in issue order: half 0 of tile i waits until half 1 of tile
-            // i-1 is issued, so the far-ahead half-0 stream does not queue in front of the half-1
-            // MMAs the epilogue is waiting for
+            // the tensor pipe takes MMAs in issue order and the epilogue reads the halves in ring
+            // order: the two streams alternate strictly (half 0 of tile i after half 1 of tile i-1,
+            // half 1 of tile i after half 0 of tile i)
             if (h == 0 && nq == 2 && i > 0) mbar_wait_sleep(h1go, (i - 1) & 1u);
+            if (h == 1) mbar_wait_sleep(h0go, i & 1u);
             mbar_wait_sleep(&dempty[db], ((u / NDB) & 1u) ^ 1u);
             KTR(kMmaWarp, 5);
             KTR(kMmaWarp1, 6);
@@ -494,10 +499,8 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                               bd + (uint64_t)((k * 32) >> 4), idesc, k ? 1u : 0u);
             tc_commit_elect(&dfull[db]);
             tc_commit_elect(&aempty[a]);
-            if (h == 1) {
-                __syncwarp();
-                if (lane == 0) mbar_arrive(h1go);
-            }
+            __syncwarp();
+            if (lane == 0 && nq == 2) mbar_arrive(h == 1 ? h1go : h0go);
             KPR(7, i);
             KTR(kMmaWarp, 13);
             KTR(kMmaWarp1, 14);
@@ -632,47 +635,59 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             KTR(KTR_EPI, 9);
             KTR(KTR_EPI + 4, 21);
             KPR(15, i);
-            float am[16], bm[16];
+            float am[16], bm[16];  // set by the first chunk (h = 0 always has one); -2^120 = no column
+            // software-pipelined read: 32-column chunks g = 4 h + c, chunk g + 1 in flight while chunk
+            // g is reduced (tcgen05.wait::ld waits for all of the thread's loads, so one ahead)
+            const int ncq0 = (npad < QW ? npad : QW) / 32;
+            const int ncq1 = nq == 2 ? (npad - QW) / 32 : 0;
+            const uint32_t u0 = (uint32_t)nq * i, db0 = u0 % NDB, db1 = (u0 + 1) % NDB;
+            mbar_wait(&dfull[db0], (u0 / NDB) & 1u);
+            tc_fence_after();
+            KTR(KTR_EPI, 11);
+            KTR(KTR_EPI + 4, 22);
+            KPR(16, i);
+            uint32_t va[32], vb[32];
+            tmem_ld<32>(tq + QW * db0, va);
+            tmem_wait();
 #pragma unroll
-            for (int a = 0; a < 16; ++a) am[a] = -0x1p120f;
-#pragma unroll
-            for (int b = 0; b < 16; ++b) bm[b] = -0x1p120f;
-#pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                if (h >= nq) break;
-                const int ncq = ((npad - QW * h) < QW ? (npad - QW * h) : QW) / 32;
-                const uint32_t u = (uint32_t)nq * i + (uint32_t)h, db = u % NDB;
-                mbar_wait(&dfull[db], (u / NDB) & 1u);
-                tc_fence_after();
-                if (h == 0) { KTR(KTR_EPI, 11); KTR(KTR_EPI + 4, 22); }
-                KPR(16, i);
-                const uint32_t tb = tq + QW * db;
-#pragma unroll
-                for (int c2 = 0; c2 < 4; c2 += 2) {  // two 32-column chunks per tcgen05.wait::ld
-                    uint32_t v[2][32];
-                    if (c2 < ncq) tmem_ld<32>(tb + c2 * 32, v[0]);
-                    if (c2 + 1 < ncq) tmem_ld<32>(tb + (c2 + 1) * 32, v[1]);
-                    tmem_wait();
-#pragma unroll
-                    for (int e = 0; e < 2; ++e) {
-                        const int c = c2 + e;
-                        if (c < ncq) {
-#define VF(k) __uint_as_float(v[e][k])
-                            bm[8 * h + 2 * c] = max3(max3(max3(VF(0), VF(1), VF(2)), max3(VF(3), VF(4), VF(5)),
-                                                          max3(VF(6), VF(7), VF(8))),
-                                                     max3(VF(9), VF(10), VF(11)), max3(VF(12), VF(13), fmaxf(VF(14), VF(15))));
-                            bm[8 * h + 2 * c + 1] = max3(max3(max3(VF(16), VF(17), VF(18)), max3(VF(19), VF(20), VF(21)),
-                                                              max3(VF(22), VF(23), VF(24))),
-                                                         max3(VF(25), VF(26), VF(27)), max3(VF(28), VF(29), fmaxf(VF(30), VF(31))));
-#pragma unroll
-                            for (int a = 0; a < 16; ++a) am[a] = max3(am[a], VF(a), VF(16 + a));
-#undef VF
-                        }
-                    }
+            for (int g = 0; g < 8; ++g) {
+                const int h = g >> 2, c = g & 3;
+                uint32_t(&cur)[32] = (g & 1) ? vb : va;
+                uint32_t(&nxt)[32] = (g & 1) ? va : vb;
+                const bool have = h == 0 ? c < ncq0 : c < ncq1;
+                const int gn = g + 1, hn = gn >> 2, cn = gn & 3;
+                const bool have_n = gn < 8 && (hn == 0 ? cn < ncq0 : cn < ncq1);
+                if (gn == 4 && have_n) {  // half 0 fully read: hand its slot back, wait for half 1
+                    tc_fence_before();
+                    mbar_arrive(&dempty[db0]);
+                    const uint32_t u1 = u0 + 1;
+                    mbar_wait(&dfull[db1], (u1 / NDB) & 1u);
+                    tc_fence_after();
                 }
-                tc_fence_before();
-                mbar_arrive(&dempty[db]);  // the ring slot may take another half
+                if (have_n) tmem_ld<32>(tq + QW * (hn ? db1 : db0) + cn * 32, nxt);
+                if (have) {
+#define VF(k) __uint_as_float(cur[k])
+                    bm[2 * g] = max3(max3(max3(VF(0), VF(1), VF(2)), max3(VF(3), VF(4), VF(5)), max3(VF(6), VF(7), VF(8))),
+                                     max3(VF(9), VF(10), VF(11)), max3(VF(12), VF(13), fmaxf(VF(14), VF(15))));
+                    bm[2 * g + 1] = max3(max3(max3(VF(16), VF(17), VF(18)), max3(VF(19), VF(20), VF(21)),
+                                              max3(VF(22), VF(23), VF(24))),
+                                         max3(VF(25), VF(26), VF(27)), max3(VF(28), VF(29), fmaxf(VF(30), VF(31))));
+                    if (g == 0) {
+#pragma unroll
+                        for (int a = 0; a < 16; ++a) am[a] = fmaxf(VF(a), VF(16 + a));
+                    } else {
+#pragma unroll
+                        for (int a = 0; a < 16; ++a) am[a] = max3(am[a], VF(a), VF(16 + a));
+                    }
+#undef VF
+                } else {
+                    bm[2 * g] = bm[2 * g + 1] = -0x1p120f;
+                }
+                if (have_n) tmem_wait();
             }
+            // every load has completed: the last half's slot goes back to the MMA
+            tc_fence_before();
+            mbar_arrive(&dempty[nq == 2 ? db1 : db0]);
             KTR(KTR_EPI, 12);
             KTR(KTR_EPI + 4, 23);
             const float vmax = max3(max3(max3(bm[0], bm[1], bm[2]), max3(bm[3], bm[4], bm[5]), max3(bm[6], bm[7], bm[8])),

@@ -34,7 +34,8 @@ int main(int argc, char** argv) {
     cudaMalloc(&de, 4);
     cudaMemcpy(dx, x.data(), n * 64, cudaMemcpyHostToDevice);
     cudaMemcpy(dc, cen.data(), k * 64, cudaMemcpyHostToDevice);
-    for (int rep = 0; rep < 3; ++rep) {
+    float best = 1e30f;
+    for (int rep = 0; rep < 8; ++rep) {
         cudaMemset(ds, 0, k * 16 * 8);
         cudaMemset(dn, 0, k * 8);
         cudaEvent_t a, b;
@@ -49,9 +50,10 @@ int main(int argc, char** argv) {
         }
         float ms;
         cudaEventElapsedTime(&ms, a, b);
-        printf("# rep %d: %.3f ms for %lld points = %.1f cycles/tile at 1.965 GHz\n", rep, ms, (long long)n,
-               ms * 1.965e6 / tiles_per_cta);
+        if (rep > 0 && ms < best) best = ms;
     }
+    printf("# best of 7: %.4f ms for %lld points = %.1f cycles/tile at 1.965 GHz\n", best, (long long)n,
+           best * 1.965e6 / tiles_per_cta);
 #ifdef KM_TRACE
     unsigned long long tr[64][32];
     cudaMemcpyFromSymbol(tr, accmg::k::g_km_trace, sizeof(tr));
