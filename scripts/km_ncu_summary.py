@@ -5,7 +5,7 @@ raw = list(csv.reader(io.StringIO(subprocess.run(['ncu', '-i', rep, '--page', 'r
 h, v = raw[0], raw[2]
 m = {h[i]: v[i] for i in range(len(h))}
 def g(k): return float(m[k].replace(',', ''))
-tiles = g('smsp__inst_executed_op_tma_ld.sum')
+tiles = float(sys.argv[2]) if len(sys.argv) > 2 else 44400.0  # 5683200 points / 128 (scripts/km_prof)
 sms = 148
 print(f"duration {g('gpu__time_duration.sum') if 'gpu__time_duration.sum' in m else 0} tiles {tiles:.0f}  cycles/tile/SM {g('sm__cycles_elapsed.max') * sms / tiles:.0f}")
 for k in ['sm__inst_executed.sum', 'l1tex__data_pipe_lsu_wavefronts_mem_shared.sum', 'l1tex__data_pipe_tc_wavefronts_mem_shared.sum',
