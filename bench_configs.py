@@ -60,19 +60,52 @@ def wall(fn):
     return time.perf_counter() - t0
 
 
-def jacobi_cfg(name, N, sweeps, P, declared, check):
+def device_ms(fn):
+    """CUDA-event time of fn's launches on the library stream (ms), synchronised on both sides."""
+    import torch
+    A.accmg_barrier()
+    st = torch.cuda.ExternalStream(A.accmg_stream(), device=0)
+    e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    e0.record(st)
+    fn()
+    e1.record(st)
+    A.accmg_barrier()
+    e1.synchronize()
+    return e0.elapsed_time(e1)
+
+
+def jacobi_cfg(name, N, sweeps, P, declared, check, rounds=5):
+    """Alternating passes over the same loops, `rounds` times: unprofiled (no events between the
+    launches: the loop time on the device) and profiled (the library's per-phase events: body,
+    compaction, exchange time per loop). gap_us = the median over rounds of (unprofiled loop time -
+    profiled body time) of adjacent passes, so clock drift between passes cancels."""
     Ah = gen.jacobi_field(2 if N > 256 else 1, N)
     Bh = Ah.copy()
     A.accmg_init(num_partitions=P, device=0, profile=1)
     try:
         rA, rB = A.accmg_region_create(Ah), A.accmg_region_create(Bh)
-        warm = 2
-        for s in range(warm):
-            WL.jacobi_sweep(rA, rB, s, N, declared)
-        A.accmg_barrier()
-        A.accmg_reset_stats()
-        t = wall(lambda: [WL.jacobi_sweep(rA, rB, s, N, declared) for s in range(warm, warm + sweeps)])
-        st = A.accmg_get_stats()
+        s0 = [0]
+
+        def run():
+            for _ in range(sweeps):
+                WL.jacobi_sweep(rA, rB, s0[0], N, declared)
+                s0[0] += 1
+
+        for _ in range(2):
+            WL.jacobi_sweep(rA, rB, s0[0], N, declared)
+            s0[0] += 1
+        A.accmg_set_profile(False)
+        t = wall(run)
+        loops, bodies, profs, st = [], [], [], None
+        for _ in range(rounds):
+            A.accmg_set_profile(False)
+            loops.append(device_ms(run) / sweeps)
+            A.accmg_set_profile(True)
+            A.accmg_barrier()
+            A.accmg_reset_stats()
+            profs.append(device_ms(run) / sweeps)
+            st = A.accmg_get_stats()
+            bodies.append(st["ms_body"] / sweeps)
         A.accmg_sync_to_host(rA)
         A.accmg_sync_to_host(rB)
     finally:
@@ -80,8 +113,12 @@ def jacobi_cfg(name, N, sweeps, P, declared, check):
     pl = per_loop(st, sweeps)
     body_bytes = 8 * (N - 2) * (N - 2) / P  # per partition launch
     body_ms_launch = st["ms_body"] / max(st["body_launches"], 1)
-    out = {"config": name, "P": P, "N": N, "sweeps": sweeps, "declared": declared,
-           "iters_per_s": (N - 2) ** 2 * sweeps / t, "ms_per_loop": t / sweeps * 1e3, **pl,
+    gaps = sorted((l - b) * 1e3 for l, b in zip(loops, bodies))
+    ms_loop = float(np.median(loops))
+    out = {"config": name, "P": P, "N": N, "sweeps": sweeps, "rounds": rounds, "declared": declared,
+           "iters_per_s": (N - 2) ** 2 / (ms_loop / 1e3), "ms_per_loop": ms_loop,
+           "ms_per_loop_wall": t / sweeps * 1e3, "ms_per_loop_profiled": float(np.median(profs)), **pl,
+           "gap_us": float(np.median(gaps)), "gap_us_range": [gaps[0], gaps[-1]],
            "body_GBs": body_bytes / (body_ms_launch / 1e3) / 1e9}
     out["body_frac_of_measured_hbm"] = out["body_GBs"] / peaks()["hbm_gbs"]
     return out
