@@ -1,5 +1,5 @@
 #!/bin/bash
-# Round-2 evidence run (one B200): GPU suite, bench lines, all configs, ncu captures.
+# Round-2 evidence run (one B200): GPU suite, bench lines, all configs, ncu captures, k-means timeline.
 O=gpurun_out/r02
 mkdir -p $O
 python -m pytest tests -m gpu -q -rs > $O/pytest_gpu.log 2>&1
@@ -16,5 +16,10 @@ ncu --set full --clock-control none --import-source on -k regex:jacobi2d_tma_k -
 ncu --set full --clock-control none --import-source on -k regex:assign_tc -s 1 -c 1 -o $O/kmeans_assign_tc ./scripts/km_prof > /dev/null 2>&1
 ncu --set full --clock-control none -k regex:gemm_kernel -s 0 -c 1 -o $O/gemm \
     python bench_configs.py --configs c3 --partitions 1 --gemm-n 16384 --gemm-reps 1 > /dev/null 2>&1
+./scripts/km_prof > $O/km_prof.txt
+./scripts/km_trace > $O/kmeans_trace_cta0.txt
+python scripts/km_trace_summary.py $O/kmeans_trace_cta0.txt > $O/kmeans_trace_summary.txt
+for r in jacobi2d_tma kmeans_assign_tc gemm; do ncu -i $O/$r.ncu-rep --page raw --csv > $O/${r}_raw.csv 2>/dev/null; done
+python scripts/km_ncu_summary.py $O/kmeans_assign_tc.ncu-rep > $O/kmeans_assign_tc_summary.txt 2>&1
 ls -la $O
 tail -3 $O/pytest_gpu.log
