@@ -63,13 +63,12 @@ using dev::smem_u32;
 constexpr int TM = 128;                 // points per tile (distance MMA M, reduction MMA K)
 constexpr int KMAX = 256;               // centroids
 constexpr int XS = 4;                   // fp32 point-tile stages
-constexpr int AS = 2;                   // distance A operand stages (freed by the distance MMAs)
+constexpr int AS = 2;                   // distance A operand stages in TMEM (freed by the distance MMAs)
 constexpr int BS = 4;                   // reduction B operand stages (freed by the reduction MMAs)
 constexpr int OS = 2;                   // one-hot stages
-constexpr int kRows = 64;               // reduction B rows: 16 dims x 4 bytes (counts: shared atomics)
+constexpr int kRows = 32;               // reduction B rows: 16 dims x 2 bytes (counts: shared atomics)
 constexpr int kXBytes = TM * 64;        // 8 KiB
-constexpr int kADBytes = TM * 128;      // 16 KiB
-constexpr int kABBytes = kRows * TM;    // 8 KiB: MN-major, point p's 64 bytes (16 dims x 4 bytes) at row p
+constexpr int kABBytes = kRows * TM;    // 4 KiB: MN-major, point p's 32 bytes (16 dims x 2 bytes) at row p
 constexpr int kOHBytes = KMAX * 128;    // 32 KiB (two 128-cluster halves)
 constexpr int QW = 128;                 // centroid columns per distance accumulator (one MMA N)
 constexpr int NDB = 3;                  // distance accumulators: a ring of three 128-column halves
@@ -81,10 +80,9 @@ constexpr int NDB = 3;                  // distance accumulators: a ring of thre
 constexpr int kThreadsTC = 512;
 constexpr int kRedWarp = 14;
 constexpr int kTmemCols = 512;
-constexpr uint32_t kColSum = NDB * QW;  // reduction accumulators: cluster half h at 384 + 64 h
+constexpr uint32_t kColSum = NDB * QW;  // reduction accumulators: cluster half h at 384 + 32 h
 
-constexpr int OFF_AD = 0;
-constexpr int OFF_AB = OFF_AD + AS * kADBytes;
+constexpr int OFF_AB = 0;
 constexpr int OFF_BD = OFF_AB + BS * kABBytes;
 constexpr int OFF_OH = OFF_BD + KMAX * 128;
 constexpr int OFF_X = OFF_OH + OS * kOHBytes;
@@ -100,7 +98,11 @@ constexpr int OFF_EQ = OFF_MISC + 16;               // float2 [BS][TM]: the poin
 constexpr int OFF_CNT = OFF_EQ + BS * TM * 8;       // int32 [KMAX]: the CTA's cluster counts
 constexpr int kSmemTC = OFF_CNT + KMAX * 4 + 1024;  // + alignment slack
 static_assert(OFF_AB % 1024 == 0 && OFF_BD % 1024 == 0 && OFF_OH % 1024 == 0 && OFF_X % 1024 == 0, "align");
-static_assert(kColSum + 2 * kRows <= kTmemCols, "tmem");
+// distance A operand in TMEM (lane = point): the constant slice [1 1 1 0 ...] (8 columns of bf16
+// pairs) and AS stages of [x0 (8 columns) | x1 (8 columns)]
+constexpr uint32_t kColA1 = kColSum + 2 * kRows;
+constexpr uint32_t kColA = kColA1 + 8;
+static_assert(kColA + AS * 16 <= kTmemCols, "tmem");
 static_assert(kSmemTC <= 227 * 1024, "smem");
 
 __device__ __forceinline__ void tc_fence_before() { asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory"); }
@@ -119,11 +121,12 @@ __device__ __forceinline__ void mma_f16(uint32_t d, uint64_t da, uint64_t db, ui
         : "memory");
 }
 // warp-collective forms: every lane executes them with the same operands, one elected lane issues
-__device__ __forceinline__ void mma_f16_elect(uint32_t d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
+// A from tensor memory (K-major, lane = row): [d], [a], b-desc
+__device__ __forceinline__ void mma_f16_ts_elect(uint32_t d, uint32_t a_tmem, uint64_t db, uint32_t idesc, uint32_t acc) {
     asm volatile(
         "{\n\t.reg .pred p, e;\n\tsetp.ne.b32 p, %4, 0;\n\telect.sync _|e, 0xffffffff;\n\t"
-        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d),
-        "l"(da), "l"(db), "r"(idesc), "r"(acc)
+        "@e tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(d),
+        "r"(a_tmem), "l"(db), "r"(idesc), "r"(acc)
         : "memory");
 }
 __device__ __forceinline__ void mma_i8_elect(uint32_t d, uint64_t da, uint64_t db, uint32_t idesc, uint32_t acc) {
@@ -156,15 +159,15 @@ __device__ __forceinline__ uint64_t sdesc_sw128(uint32_t saddr) {
     d |= (uint64_t)2 << 61;
     return d;
 }
-// MN-major operand, 64-byte swizzle, N = 64 one-byte elements: K row p (64 B) at 64 p, 8-row atoms
-// 512 B apart (SBO); one atom along N, so the leading-dimension offset is never stepped
-__device__ __forceinline__ uint64_t sdesc_mn_sw64(uint32_t saddr) {
+// MN-major operand, 32-byte swizzle, N = 32 one-byte elements: K row p (32 B) at 32 p, 8-row atoms
+// 256 B apart (SBO); one atom along N, so the leading-dimension offset is never stepped
+__device__ __forceinline__ uint64_t sdesc_mn_sw32(uint32_t saddr) {
     uint64_t d = 0;
     d |= (uint64_t)((saddr >> 4) & 0x3FFF);
     d |= (uint64_t)(kABBytes >> 4) << 16;
-    d |= (uint64_t)(512 >> 4) << 32;
+    d |= (uint64_t)(256 >> 4) << 32;
     d |= (uint64_t)1 << 46;
-    d |= (uint64_t)4 << 61;
+    d |= (uint64_t)6 << 61;
     return d;
 }
 // byte offset of element k (byte k) of row m in a 128-byte-swizzled K-major operand
@@ -252,6 +255,19 @@ __device__ __forceinline__ void tmem_ld<16>(uint32_t taddr, uint32_t (&r)[16]) {
         : "r"(taddr));
 }
 __device__ __forceinline__ void tmem_wait() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+__device__ __forceinline__ void tmem_st16(uint32_t taddr, const uint32_t (&r)[16]) {
+    asm volatile(
+        "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(taddr),
+        "r"(r[0]), "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7]), "r"(r[8]), "r"(r[9]),
+        "r"(r[10]), "r"(r[11]), "r"(r[12]), "r"(r[13]), "r"(r[14]), "r"(r[15])
+        : "memory");
+}
+__device__ __forceinline__ void tmem_st8(uint32_t taddr, const uint32_t (&r)[8]) {
+    asm volatile("tcgen05.st.sync.aligned.32x32b.x8.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8};" ::"r"(taddr), "r"(r[0]),
+                 "r"(r[1]), "r"(r[2]), "r"(r[3]), "r"(r[4]), "r"(r[5]), "r"(r[6]), "r"(r[7])
+                 : "memory");
+}
+__device__ __forceinline__ void tmem_wait_st() { asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory"); }
 
 __device__ __forceinline__ uint64_t pk2(float a, float b) {
     uint64_t r;
@@ -338,7 +354,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
     const uint32_t pad = ((raw + 1023u) & ~1023u) - raw;
     unsigned char* smem = smem_raw + pad;
     const uint32_t sbase = raw + pad;
-    const uint32_t sAD = sbase + OFF_AD, sAB = sbase + OFF_AB, sBD = sbase + OFF_BD, sOH = sbase + OFF_OH;
+    const uint32_t sAB = sbase + OFF_AB, sBD = sbase + OFF_BD, sOH = sbase + OFF_OH;
     const uint32_t sX = sbase + OFF_X, sPC = sbase + OFF_PC;
     uint64_t* xfull = reinterpret_cast<uint64_t*>(smem + OFF_BAR);
     uint64_t* xempty = xfull + XS;
@@ -375,11 +391,6 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                      : "memory");
     }
     for (uint32_t i = tid; i < OS * kOHBytes / 16; i += kThreads) sts_v4(sOH + i * 16, make_uint4(0, 0, 0, 0));
-    for (int i = tid; i < AS * TM; i += kThreads) {  // distance A, slice 3 = [1 1 1 0 ...]
-        const uint32_t base = sAD + (i / TM) * kADBytes, r = i % TM;
-        sts_v4(base + sw_off(r, 96), make_uint4(0x3F803F80u, 0x00003F80u, 0, 0));
-        sts_v4(base + sw_off(r, 112), make_uint4(0, 0, 0, 0));
-    }
     for (int i = tid; i < KMAX; i += kThreads) reinterpret_cast<int*>(smem + OFF_CNT)[i] = 0;
     if (tid == 0) {
         for (int s = 0; s < XS; ++s) { mbar_init(&xfull[s], 1); mbar_init(&xempty[s], 128); }  // the converters
@@ -451,6 +462,26 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
     KPR(3, 0);
     const uint32_t tmem = misc[0];
 
+    // reductiontoarray MMAs of tile j (u8 one-hot x byte planes -> s32, B MN-major), issued by one
+    // warp after the epilogue has filled the tile's one-hot stage
+    auto issue_reduction = [&](uint32_t j) {
+        const uint32_t idesc_sum = (2u << 4) | (1u << 16) | ((uint32_t)(kRows >> 3) << 17) | ((uint32_t)(TM >> 4) << 24);
+        const uint64_t dAB = sdesc_mn_sw32(sAB), dOH = sdesc_sw128(sOH);
+        const int o = (int)(j % OS);
+        mbar_wait_sleep(&ofull[o], (uint32_t)((j / OS) & 1));
+        KPR(8, j);
+        tc_fence_after();
+        const uint64_t b = dAB + (uint64_t)(((j % BS) * kABBytes) >> 4);
+        const uint64_t oh = dOH + (uint64_t)((o * kOHBytes) >> 4);
+        for (int h = 0; h < nh; ++h)
+#pragma unroll
+            for (int k = 0; k < 4; ++k)
+                mma_i8_elect(tmem + kColSum + (uint32_t)(kRows * h), oh + (uint64_t)((h * 16384 + k * 32) >> 4),
+                             b + (uint64_t)((k * 32 * kRows) >> 4), idesc_sum, (j | k) ? 1u : 0u);
+        tc_commit_elect(&oempty[o]);
+        tc_commit_elect(&bempty[j % BS]);
+        KPR(9, j);
+    };
     if (warp == kProdWarp) {
         // ---- producer
         if (lane == 0) {
@@ -470,7 +501,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
         // whole warp runs the loop and one elected lane issues each tcgen05 instruction;
         // descriptors are the stage bases plus the 16-byte-unit offsets of the slices
         const int h = warp == kMmaWarp ? 0 : 1;
-        const uint64_t dAD = sdesc_sw128(sAD), dBD = sdesc_sw128(sBD);
+        const uint64_t dBD = sdesc_sw128(sBD);
         const int wq = (npad - QW * h) < QW ? (npad - QW * h) : QW;
         const uint32_t idesc = (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(wq >> 3) << 17) |
                                ((uint32_t)(TM >> 4) << 24);
@@ -480,7 +511,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             mbar_wait_sleep(&afull[a], (uint32_t)((i / AS) & 1));
             KTR(kMmaWarp, 4);
             KPR(5, i);
-            const uint64_t ad = dAD + (uint64_t)((a * kADBytes) >> 4);
+            const uint32_t at = tmem + kColA + 16u * (uint32_t)a;  // this tile's [x0 | x1] in TMEM
             const uint32_t u = (uint32_t)nq * i + (uint32_t)h, db = u % NDB;  // ring slot and its use count
             // the tensor pipe takes MMAs in issue order and the epilogue reads the halves in ring
             // order: the two streams alternate strictly (half 0 of tile i after half 1 of tile i-1,
@@ -494,9 +525,9 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             tc_fence_after();
 #pragma unroll
             for (int k = 0; k < 4; ++k)
-                // A slices x0, x0, x1, 1 (slice 0 read twice) against B slices c0, c1, c0, h
-                mma_f16_elect(tmem + QW * db, ad + (uint64_t)((k == 1 ? 0 : k * 32) >> 4),
-                              bd + (uint64_t)((k * 32) >> 4), idesc, k ? 1u : 0u);
+                // A slices x0, x0, x1, 1 (from TMEM; x0 read twice) against B slices c0, c1, c0, h
+                mma_f16_ts_elect(tmem + QW * db, k == 3 ? tmem + kColA1 : at + (k == 2 ? 8u : 0u),
+                                 bd + (uint64_t)((k * 32) >> 4), idesc, k ? 1u : 0u);
             tc_commit_elect(&dfull[db]);
             tc_commit_elect(&aempty[a]);
             __syncwarp();
@@ -506,36 +537,20 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             KTR(kMmaWarp1, 14);
         }
     } else if (warp == kRedWarp) {
-        // ---- reductiontoarray MMAs (u8 one-hot x byte planes -> s32), one tile behind the
-        // epilogue's one-hot bytes
-        // u8 x u8 -> s32, B (the byte planes) MN-major
-        const uint32_t idesc_sum = (2u << 4) | (1u << 16) | ((uint32_t)(kRows >> 3) << 17) | ((uint32_t)(TM >> 4) << 24);
-        const uint64_t dAB = sdesc_mn_sw64(sAB), dOH = sdesc_sw128(sOH);
-        for (uint32_t j = 0; j < nt32; ++j) {
-            const int o = (int)(j % OS);
-            mbar_wait_sleep(&ofull[o], (uint32_t)((j / OS) & 1));
-            {
-                const uint32_t i = j + 1;
-                KTR(kRedWarp, 7);
-            }
-            KPR(8, j);
-            tc_fence_after();
-            const uint64_t b = dAB + (uint64_t)(((j % BS) * kABBytes) >> 4);
-            const uint64_t oh = dOH + (uint64_t)((o * kOHBytes) >> 4);
-            for (int h = 0; h < nh; ++h)
-#pragma unroll
-                for (int k = 0; k < 4; ++k)
-                    mma_i8_elect(tmem + kColSum + (uint32_t)(kRows * h), oh + (uint64_t)((h * 16384 + k * 32) >> 4),
-                                 b + (uint64_t)((k * 32 * kRows) >> 4), idesc_sum, (j | k) ? 1u : 0u);
-            tc_commit_elect(&oempty[o]);
-            tc_commit_elect(&bempty[j % BS]);
-            KPR(9, j);
-        }
+        // (issuing the reductions from the last distance stream, right after its group, measured
+        // 4 % slower: scripts/r2_kab.sh)
+        for (uint32_t j = 0; j < nt32; ++j) issue_reduction(j);
         tc_commit_elect(sdone);
         KPR(10, 0);
     } else if (warp >= 2 && warp < 6) {
-        // ---- converters: point row r
-        const int r = tid - 64;
+        // ---- converters: point row r = TMEM lane of the warp's lane quarter (warp % 4)
+        const int r = 32 * (warp & 3) + lane;
+        const uint32_t tqc = tmem + ((uint32_t)(32 * (warp & 3)) << 16);
+        {  // the constant A slice [1 1 1 0 ... 0] (bf16 ones: the -|c|^2/2 pieces h0 + h1 + h2)
+            const uint32_t ones[8] = {0x3F803F80u, 0x00003F80u, 0u, 0u, 0u, 0u, 0u, 0u};
+            tmem_st8(tqc + kColA1, ones);
+            tmem_wait_st();
+        }
         const float scale = (float)(1 << shift);
         const float Cinf = __uint_as_float(misc[1]);
         const float C2 = __uint_as_float(misc[2]);
@@ -552,6 +567,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                 xv[4 * j] = v.x; xv[4 * j + 1] = v.y; xv[4 * j + 2] = v.z; xv[4 * j + 3] = v.w;
             }
             mbar_wait_sleep(&aempty[a], (uint32_t)((i / AS) & 1) ^ 1u);
+            tc_fence_after();
             KTR(2, 1);
             KPR(12, i);
             const int bs = (int)(i % BS);
@@ -561,37 +577,42 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             uint4 h0, l0, h1, l1;
             split8(xv, h0, l0);
             split8(xv + 8, h1, l1);
-            const uint32_t ad = sAD + a * kADBytes;
-            // slices 0 = x0, 2 = x1 (3 = the constant ones); the MMA reads slice 0 twice
-            sts_v4(ad + sw_off(r, 0), h0);
-            sts_v4(ad + sw_off(r, 16), h1);
-            sts_v4(ad + sw_off(r, 64), l0);
-            sts_v4(ad + sw_off(r, 80), l1);
+            {  // [x0 | x1] of the point into its TMEM lane (the MMA reads x0 twice)
+                const uint32_t w[16] = {h0.x, h0.y, h0.z, h0.w, h1.x, h1.y, h1.z, h1.w,
+                                        l0.x, l0.y, l0.z, l0.w, l1.x, l1.y, l1.z, l1.w};
+                tmem_st16(tqc + kColA + 16u * (uint32_t)a, w);
+            }
             // the stage is released only after instructions that consume the loaded values (the
             // arrive alone does not wait for the shared-memory loads to return their data, and the
             // producer refills the stage as soon as all converters have arrived)
             mbar_arrive(&xempty[s]);
-            // fixed point x * 2^shift, biased to unsigned: u = v + 2^31. The B operand is MN-major: the
-            // point's 64 bytes in order (j, b) are its 16 words u_j, little-endian, so four 16-byte
-            // stores write the row (64-byte swizzle: chunk c of row r at c ^ ((r >> 1) & 3)).
-            // Grid check without branches: v = x 2^shift must equal rint(v) (every float of magnitude
-            // >= 2^23 is an integer) and |v| < 2^31; the largest |v - rint(v)| and |v| of the point
-            // are tested once
+            // fixed point v = x * 2^shift, as 16-bit words biased to unsigned: u = v + 2^15 when every
+            // |v_j| < 2^15 (the point "fits"); otherwise u = 2^15 (v taken as 0 here) and the point is
+            // flagged for the exact int64 path in the epilogue. The B operand is MN-major: the point's
+            // 32 bytes in order (j, b) are its 16 halfwords, little-endian, so two 16-byte stores write
+            // the row (32-byte swizzle: chunk c of row r at c ^ ((r >> 2) & 1)).
+            // Grid check without branches: v must equal rint(v) (every float of magnitude >= 2^23 is
+            // an integer) and |v| < 2^31; the largest |v - rint(v)| and |v| of the point are tested once
             float fr = 0.f, vm = 0.f;
-            uint32_t uw[16];
+            int iv[16];
 #pragma unroll
             for (int j = 0; j < 16; ++j) {
                 const float v = xv[j] * scale;  // exact: power-of-two scaling
                 const float rv = rintf(v);
                 fr = fmaxf(fr, fabsf(v - rv));  // exact difference (Sterbenz)
                 vm = fmaxf(vm, fabsf(v));
-                uw[j] = (uint32_t)__float2int_rn(rv) ^ 0x80000000u;
+                iv[j] = __float2int_rn(rv);
             }
+            const bool fits = vm < 32768.0f;
             {
-                const uint32_t row = sAB + bs * kABBytes + (uint32_t)r * 64u, sw = ((uint32_t)r >> 1) & 3u;
+                uint32_t hw[8];
 #pragma unroll
-                for (int c = 0; c < 4; ++c)
-                    sts_v4(row + (((uint32_t)c ^ sw) << 4), make_uint4(uw[4 * c], uw[4 * c + 1], uw[4 * c + 2], uw[4 * c + 3]));
+                for (int j = 0; j < 8; ++j)
+                    hw[j] = fits ? __byte_perm((uint32_t)iv[2 * j] ^ 0x8000u, (uint32_t)iv[2 * j + 1] ^ 0x8000u, 0x5410)
+                                 : 0x80008000u;
+                const uint32_t row = sAB + bs * kABBytes + (uint32_t)r * 32u, sw = ((uint32_t)r >> 2) & 1u;
+                sts_v4(row + ((0u ^ sw) << 4), make_uint4(hw[0], hw[1], hw[2], hw[3]));
+                sts_v4(row + ((1u ^ sw) << 4), make_uint4(hw[4], hw[5], hw[6], hw[7]));
             }
             bad |= (fr != 0.f) | !(vm < 2147483648.0f);
             {  // the filter bound's per-point terms, for the epilogue (header: E, Dhat)
@@ -600,10 +621,14 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                 for (int j = 0; j < 16; ++j) { L1 += fabsf(xv[j]); Q = fmaf(xv[j], xv[j], Q); }
                 const float E = (0x1p-11f * (L1 * Cinf + C2)) * 1.001f + 0x1p-100f;
                 const float Qa = Q * (1.f + 0x1p-17f) + 2.f * E;
-                asm volatile("st.shared.v2.f32 [%0], {%1, %2};" ::"r"(sbase + OFF_EQ + (bs * TM + r) * 8), "f"(E), "f"(Qa)
+                // (the sign of E carries the point's "does not fit" flag; E > 0)
+                asm volatile("st.shared.v2.f32 [%0], {%1, %2};" ::"r"(sbase + OFF_EQ + (bs * TM + r) * 8),
+                             "f"(fits ? E : -E), "f"(Qa)
                              : "memory");
             }
-            fence_async_smem();
+            fence_async_smem();  // the B operand (shared memory) for the reduction MMAs
+            tmem_wait_st();      // the A operand (TMEM) for the distance MMAs
+            tc_fence_before();
             mbar_arrive(&afull[a]);
             KTR(2, 3);
             KPR(14, i);
@@ -697,7 +722,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                          : "r"(sbase + OFF_EQ + ((uint32_t)(i % BS) * TM + r) * 8) : "memory");
             // candidate <=> value >= vmax - T <=> > thr (the next float below)
             const float Dhat = fmaxf(Qa - 2.f * vmax, 0.f);
-            const float T = (2.f * E + 0x1p-16f * Dhat) * 1.001f;
+            const float T = (2.f * fabsf(E) + 0x1p-16f * Dhat) * 1.001f;
             const float thr = next_below(vmax - T);
             // sign bits of thr - max (packed FSUB2, each lane rounds alone) funnel-shifted into the
             // masks: bit 15 - a of mA, bit 15 - b of mB; two independent chains each
@@ -777,10 +802,26 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                 }
             }
             KTR(KTR_EPI, 17);
-            // member[] and the reductiontoarray count (the sums go through the MMA)
+            // member[] and the reductiontoarray count (the sums go through the MMA; a point whose
+            // fixed-point values do not fit 16 bits adds them here, exact int64, to the partials)
             if (valid) {
                 member[p] = bi;
                 atomicAdd(&s_cnt[bi], 1);
+                if (E < 0.f) {
+                    const float scale = (float)(1 << shift);
+                    const float4* xp = reinterpret_cast<const float4*>(xg + p * 16);
+#pragma unroll
+                    for (int j = 0; j < 4; ++j) {
+                        const float4 v = xp[j];
+                        const float e4[4] = {v.x, v.y, v.z, v.w};
+#pragma unroll
+                        for (int e = 0; e < 4; ++e) {
+                            const long long iv = (long long)__float2int_rn(e4[e] * scale);
+                            if (iv) atomicAdd(reinterpret_cast<unsigned long long*>(sums) + bi * 16 + 4 * j + e,
+                                              (unsigned long long)iv);
+                        }
+                    }
+                }
             }
             // the point's one-hot byte (cluster row bi, point column r) in the set's stage; the
             // byte this thread set there two tiles ago is cleared first
@@ -795,7 +836,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             KPR(22, i);
             KTR(KTR_EPI, 20);
         }
-        // reduction accumulators: lane = cluster (h*128 + r), columns 4j+b = byte sums; counts
+        // reduction accumulators: lane = cluster (h*128 + r), columns 2j+b = byte sums; counts
         // from the shared atomics (every epilogue warp has passed its last tile: named barrier)
         KPR(23, 0);
         named_bar(5, 256);
@@ -804,20 +845,17 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
         KPR(25, 0);
         tc_fence_after();
         for (int h = half; h < nh; h += 2) {
-            uint32_t v0[32], v1[32];
+            uint32_t v0[32];
             const uint32_t tb2 = tq + kColSum + (uint32_t)(kRows * h);
             tmem_ld<32>(tb2, v0);
-            tmem_ld<32>(tb2 + 32, v1);
             tmem_wait();
             const int c = 128 * h + r;
             const uint64_t cnt = c < kc ? (uint64_t)s_cnt[c] : 0ull;
             if (cnt) {
 #pragma unroll
                 for (int j = 0; j < 16; ++j) {
-                    const uint32_t* w = j < 8 ? &v0[4 * j] : &v1[4 * (j - 8)];
-                    const uint64_t su = (uint64_t)w[0] + ((uint64_t)w[1] << 8) + ((uint64_t)w[2] << 16) +
-                                        ((uint64_t)w[3] << 24);
-                    const int64_t sv = (int64_t)(su - (cnt << 31));  // remove the 2^31 bias
+                    const uint64_t su = (uint64_t)v0[2 * j] + ((uint64_t)v0[2 * j + 1] << 8);
+                    const int64_t sv = (int64_t)(su - (cnt << 15));  // remove the 2^15 bias
                     if (sv) atomicAdd(reinterpret_cast<unsigned long long*>(sums) + c * 16 + j, (unsigned long long)sv);
                 }
                 atomicAdd(reinterpret_cast<unsigned long long*>(counts) + c, (unsigned long long)cnt);
