@@ -182,10 +182,11 @@ def kmeans_cfg(n, iters, P, check):
     out["assign_frac_of_measured_hbm"] = out["assign_hbm_gbs"] / pk["hbm_gbs"]
     if impl == "tc":
         # tensor-pipe view of the tcgen05 formulation (kmeans_tc.cu): per 128-point tile 8 distance
-        # MMAs (M=128, N=128, K=16 bf16: 64 cycles each) + 8 reductiontoarray MMAs (M=128, N=64,
-        # K=32 u8: 32 cycles each) = 768 tensor cycles per tile per SM at 1.965 GHz
+        # MMAs (M=128, N=128, K=16 bf16: 64 cycles each) + 8 reductiontoarray MMAs (M=128, N=32,
+        # K=32 u8 at twice the bf16 rate: 16 cycles each) = 640 tensor cycles per tile per SM at
+        # 1.965 GHz (round 1's formulation, with 32-bit reduction words, was 768)
         tiles = -(-n // 128)
-        t_tensor = tiles / 148 * 768 / 1.965e9
+        t_tensor = tiles / 148 * 640 / 1.965e9
         out["assign_tensor_bound_ms"] = t_tensor * 1e3
         out["assign_frac_of_tensor_bound"] = t_tensor / (ms_assign / 1e3)
     else:
