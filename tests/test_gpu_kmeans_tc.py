@@ -77,3 +77,10 @@ def test_fixed_point_near_2_31():
     x[:, 3] = np.float32(2 ** 23 - 1)
     x[::2, 5] = np.float32(-(2 ** 23) + 1)
     _run(x, 200, 2, P=2, shift=8)
+
+
+def test_many_tiles_per_cta_k256():
+    """Every CTA runs dozens of 128-point tiles (steady state of the TMEM ring, the one-hot and
+    operand stages, and every epilogue set's second and later tiles), k = 256: both halves."""
+    x = gen.kmeans_points(21, 148 * 128 * 24 + 5, 16, 256, gen.KM_OVERLAP)
+    _run(x, 256, 2, P=1)
