@@ -37,7 +37,7 @@ constexpr int kBBytes = BK * BN * 2;            // 32 KiB
 constexpr int kStageBytes = kABytes + kBBytes;  // 48 KiB
 constexpr int kThreads = 192;                   // 6 warps
 constexpr int kTmemCols = 512;                  // 2 accumulators x 256 fp32 columns
-constexpr int kGroupM = 16;                     // tile raster: 16 m-blocks per group (L2 reuse)
+constexpr int kGroupM = 32;                     // tile raster: 32 m-blocks per group (L2 reuse)
 
 using dev::mbar_arrive;
 using dev::mbar_expect_tx;
@@ -80,8 +80,10 @@ constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((
                             ((uint32_t)(BM >> 4) << 24);
 
 // Tile raster: groups of `gm_` m-blocks swept across all n-blocks, so the tiles resident at once
-// (one per SM or SM pair) cover a near-square patch of C and share A row-blocks / B column-blocks
-// through L2.
+// (one per SM) cover a patch of C (32 x 4.6 blocks: 4096 rows x 1184 columns) and share A
+// row-blocks / B column-blocks through L2. Group size measured at C3 (32768^3, same box, two
+// rounds; profiles/r02/experiments/gemm_raster_ab.txt): 8 -> 1463, 16 -> 1468-1478, 24 -> 1455,
+// 32 -> 1498-1509, 40 -> 1490, 48 -> 1396-1413, 64 -> 1418-1424 TFLOP/s.
 __device__ __forceinline__ void tile_coords(int64_t t, int num_m, int num_n, int& mb, int& nb, int gm_ = kGroupM) {
     const int64_t per_group = (int64_t)gm_ * num_n;
     const int64_t g = t / per_group;
