@@ -255,3 +255,30 @@ def test_deep_halo_plan_vs_model(dry, P, h):
         A.accmg_loop_launch(A.bounds([1, 1], [N - 1, N - 1]), A.BODY_JACOBI2D_DEEP,
                             WL.jacobi_deep_descs(rA, rB, N, h), A.accmg_args_jacobi2d_deep(N, N, 0))
     assert e.value.code == A.EINVAL
+
+
+@pytest.mark.parametrize("P", [1, 2, 3, 8])
+def test_kmeans_assign_reduction_plan_vs_model(dry, P):
+    """The k-means assignment loop (reductiontoarray destinations, L89-91 / L112): byte counters and
+    validity after each loop match the model's REDUCE_SUM branch, and the reduction bytes equal
+    the closed form of reading W8 — 2 (P - 1) x (sums + counts bytes) per loop."""
+    n, d, k = 1000, 16, 37
+    dry(P)
+    hx, hc = np.zeros((n, d), np.float32), np.zeros((k, d), np.float32)
+    hm, hs, hn = np.zeros(n, np.int32), np.zeros((k, d), np.int64), np.zeros(k, np.int64)
+    rx, rc, rm, rs, rn = (A.accmg_region_create(a) for a in (hx, hc, hm, hs, hn))
+    mdl = M.Model(P)
+    mx, mc, mm = mdl.region(n * d, 4), mdl.region(k * d, 4), mdl.region(n, 4)
+    ms, mn = mdl.region(k * d, 8), mdl.region(k, 8)
+    for _ in range(2):
+        before = A.accmg_get_stats()
+        A.accmg_loop_launch(A.bounds([0], [n]), A.BODY_KMEANS_ASSIGN,
+                            [A.access(rx, A.R, True, d, 0, 0), A.access(rc, A.R), A.access(rm, A.W, True, 1, 0, 0),
+                             A.access(rs, A.REDUCE_SUM), A.access(rn, A.REDUCE_SUM)], A.accmg_args_kmeans(n, d, k, 8))
+        after = A.accmg_get_stats()
+        exp = mdl.loop(0, n, [(mx, M.R, 1, d, 0, 0), (mc, M.R, 0, 0, 0, 0), (mm, M.W, 1, 1, 0, 0),
+                              (ms, M.REDUCE_SUM, 0, 0, 0, 0), (mn, M.REDUCE_SUM, 0, 0, 0, 0)])
+        assert exp["reduce"] == 2 * (P - 1) * (k * d * 8 + k * 8)
+        for key in ("reduce", "declared", "h2d", "interpartition"):
+            assert after["bytes_" + key] - before["bytes_" + key] == exp[key], key
+        _compare_valid([rx, rc, rm, rs, rn], [mx, mc, mm, ms, mn], P)
