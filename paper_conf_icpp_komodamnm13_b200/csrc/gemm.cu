@@ -4,11 +4,13 @@
 // C are the partition's declared windows, B is replicated.
 //
 // This is a real contraction, so it runs on the 5th-generation tensor cores:
-//   * persistent kernel, one CTA per SM, 128 x 256 output tiles (the last n-block may be partial:
-//     N % 8 == 0), K-steps of 64;
-//   * warp 0 = TMA producer: A tile [128 rows][64 k] (K-major) and B tile [64 k][256 n]
-//     (N-major, four 64-column boxes), both 128-byte swizzled, into a 4-stage smem ring guarded by
-//     full/empty mbarriers;
+//   * persistent kernel, clusters of two CTAs (one CTA per SM), 128 x 256 output tiles per CTA (the
+//     last n-block may be partial: N % 8 == 0), K-steps of 64; the two CTAs of a cluster take
+//     vertically adjacent tiles of the same n-block (a pair tile: 2 m-blocks x 1 n-block);
+//   * warp 0 = TMA producer: its A tile [128 rows][64 k] (K-major) and half of the shared B tile
+//     [64 k][256 n] (N-major, two of its four 64-column boxes) multicast into both CTAs, all
+//     128-byte swizzled, into a 4-stage smem ring guarded by full/empty mbarriers (a stage's empty
+//     barrier counts both CTAs' MMA commits: the peer writes into it too);
 //   * warp 1 = MMA issuer: one elected thread issues tcgen05.mma.cta_group::1.kind::f16
 //     (M=128, N=256, K=16; A K-major, B MN-major via the instruction descriptor) accumulating in
 //     TMEM; tcgen05.commit frees smem stages and signals the epilogue;
@@ -37,7 +39,7 @@ constexpr int kBBytes = BK * BN * 2;            // 32 KiB
 constexpr int kStageBytes = kABytes + kBBytes;  // 48 KiB
 constexpr int kThreads = 192;                   // 6 warps
 constexpr int kTmemCols = 512;                  // 2 accumulators x 256 fp32 columns
-constexpr int kGroupM = 32;                     // tile raster: 32 m-blocks per group (L2 reuse)
+constexpr int kGroupM = 8;                      // tile raster: 8 pair tiles (16 m-blocks) per group
 
 using dev::mbar_arrive;
 using dev::mbar_expect_tx;
@@ -79,11 +81,14 @@ __device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo, uint32_t
 constexpr uint32_t kIdesc = (1u << 4) | (1u << 7) | (1u << 10) | (1u << 16) | ((uint32_t)(BN >> 3) << 17) |
                             ((uint32_t)(BM >> 4) << 24);
 
-// Tile raster: groups of `gm_` m-blocks swept across all n-blocks, so the tiles resident at once
-// (one per SM) cover a patch of C (32 x 4.6 blocks: 4096 rows x 1184 columns) and share A
-// row-blocks / B column-blocks through L2. Group size measured at C3 (32768^3, same box, two
-// rounds; profiles/r02/experiments/gemm_raster_ab.txt): 8 -> 1463, 16 -> 1468-1478, 24 -> 1455,
-// 32 -> 1498-1509, 40 -> 1490, 48 -> 1396-1413, 64 -> 1418-1424 TFLOP/s.
+// Tile raster: groups of `gm_` m-blocks (here: m-block pairs) swept across all n-blocks, so the
+// tiles resident at once cover a patch of C (16 m-blocks x 9.25 n-blocks: 2048 rows x 2368
+// columns) and share A row-blocks / B column-blocks through L2. Measured at C3 (32768^3, same-box
+// interleaved rounds; profiles/r02/experiments/gemm_raster_ab.txt, gemm_multicast_ab.txt):
+// single-CTA kernel (no multicast), groups of 8 / 16 / 24 / 32 / 40 / 48 / 64 m-blocks -> 1463 /
+// 1468-1478 / 1455 / 1498-1509 / 1490 / 1396-1413 / 1418-1424 TFLOP/s; this kernel with groups of
+// 4 / 8 / 12 / 16 / 32 pairs -> 1376-1379 / 1497-1525 / 1494-1496 / 1468-1473 / 1238-1282 (the
+// single-CTA kernel with 32 m-blocks at 1360-1405 on that box).
 __device__ __forceinline__ void tile_coords(int64_t t, int num_m, int num_n, int& mb, int& nb, int gm_ = kGroupM) {
     const int64_t per_group = (int64_t)gm_ * num_n;
     const int64_t g = t / per_group;
@@ -94,9 +99,39 @@ __device__ __forceinline__ void tile_coords(int64_t t, int num_m, int num_n, int
     nb = (int)(r / rows_in_group);
 }
 
+// ---- the kernel: the two CTAs of a cluster compute vertically adjacent 128 x 256 tiles of the same
+// n-block and share its B tile: CTA r loads B columns [128 r, 128 r + 128) of each k-step with a
+// TMA multicast into both CTAs' shared memory (L2 -> SM traffic per CTA and stage 48 -> 32 KiB,
+// which the power-capped chip turns into clock: +8-10 % over the single-CTA kernel); each CTA
+// issues its own tcgen05.mma.cta_group::1 (M = 128, N = 256). A stage is refilled only after both
+// CTAs' MMAs have read it: every MMA commit arrives on the stage's empty barrier of both CTAs.
+// (A 2-SM cta_group::2 kernel, M = 256, measured slower: profiles/r02/experiments/README.md.)
+__device__ __forceinline__ uint32_t cluster_rank() {
+    uint32_t r;
+    asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
+    return r;
+}
+__device__ __forceinline__ void cluster_sync_all() {
+    asm volatile("barrier.cluster.arrive.release.aligned;\n\tbarrier.cluster.wait.acquire.aligned;" ::: "memory");
+}
+__device__ __forceinline__ void tma_load_2d_mc(const CUtensorMap* map, uint64_t* bar, void* dst, int c0, int c1,
+                                               uint16_t mask) {
+    asm volatile(
+        "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster [%0], [%1, {%2, %3}], [%4], %5;" ::"r"(
+            smem_u32(dst)),
+        "l"(reinterpret_cast<uint64_t>(map)), "r"(c0), "r"(c1), "r"(smem_u32(bar)), "h"(mask)
+        : "memory");
+}
+__device__ __forceinline__ void tc_commit_mc1(uint64_t* bar, uint16_t mask) {
+    asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+                     smem_u32(bar)),
+                 "h"(mask)
+                 : "memory");
+}
+
 __global__ void __launch_bounds__(kThreads, 1)
 gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ CUtensorMap map_b,
-            float* __restrict__ C, int64_t N, int64_t K, int64_t m0, int64_t m1, int64_t row_lo) {
+               float* __restrict__ C, int64_t N, int64_t K, int64_t m0, int64_t m1, int64_t row_lo) {
     extern __shared__ __align__(1024) unsigned char smem_raw[];
     unsigned char* smem = reinterpret_cast<unsigned char*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + kStages * kStageBytes);
@@ -106,13 +141,16 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
     uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(tempty + 2);
 
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    const uint32_t rank = cluster_rank();
     const int num_m = (int)((m1 - m0 + BM - 1) / BM);
-    const int num_n = (int)((N + BN - 1) / BN);  // the last n-block may be partial (N % 8 == 0)
-    const int64_t num_tiles = (int64_t)num_m * num_n;
+    const int num_mp = (num_m + 1) / 2;  // m-block pairs
+    const int num_n = (int)((N + BN - 1) / BN);
+    const int64_t num_tiles = (int64_t)num_mp * num_n;
     const int nk = (int)(K / BK);
+    const int64_t cl = blockIdx.x >> 1, ncl = gridDim.x >> 1;
 
     if (warp == 0 && lane == 0) {
-        for (int s = 0; s < kStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 1); }
+        for (int s = 0; s < kStages; ++s) { mbar_init(&full[s], 1); mbar_init(&empty[s], 2); }
         for (int a = 0; a < 2; ++a) { mbar_init(&tfull[a], 1); mbar_init(&tempty[a], 128); }
         asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
         asm volatile("prefetch.tensormap [%0];" ::"l"(reinterpret_cast<uint64_t>(&map_a)) : "memory");
@@ -124,7 +162,7 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
         asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
     }
     tc_fence_before();
-    __syncthreads();
+    cluster_sync_all();  // both CTAs' barriers are initialised before any multicast reaches them
     tc_fence_after();
     const uint32_t tmem = *tmem_slot;
 
@@ -132,19 +170,21 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
         if (lane == 0) {
             int stage = 0;
             uint32_t phase = 0;
-            for (int64_t t = blockIdx.x; t < num_tiles; t += gridDim.x) {
-                int mb, nb;
-                tile_coords(t, num_m, num_n, mb, nb);
-                const int row = (int)(m0 + (int64_t)mb * BM);
-                const int col = nb * BN;
+            for (int64_t t = cl; t < num_tiles; t += ncl) {
+                int mp, nb;
+                tile_coords(t, num_mp, num_n, mp, nb);
+                const int row = (int)(m0 + (int64_t)(2 * mp + (int)rank) * BM);
+                const int col = nb * BN + 128 * (int)rank;
                 for (int kb = 0; kb < nk; ++kb) {
                     mbar_wait(&empty[stage], phase ^ 1);
                     unsigned char* sa = smem + stage * kStageBytes;
                     unsigned char* sb = sa + kABytes;
-                    mbar_expect_tx(&full[stage], kStageBytes);
+                    mbar_expect_tx(&full[stage], kStageBytes);  // own A + both halves of B
                     tma_load_2d(&map_a, &full[stage], sa, kb * BK, row - (int)row_lo);
 #pragma unroll
-                    for (int j = 0; j < BN / 64; ++j) tma_load_2d(&map_b, &full[stage], sb + j * (BK * 128), col + 64 * j, kb * BK);
+                    for (int j = 0; j < 2; ++j)
+                        tma_load_2d_mc(&map_b, &full[stage], sb + (2 * rank + j) * (BK * 128), col + 64 * j, kb * BK,
+                                       (uint16_t)0x3);
                     if (++stage == kStages) { stage = 0; phase ^= 1; }
                 }
             }
@@ -154,7 +194,7 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
         uint32_t phase = 0;
         int acc = 0;
         uint32_t acc_phase = 0;
-        for (int64_t t = blockIdx.x; t < num_tiles; t += gridDim.x) {
+        for (int64_t t = cl; t < num_tiles; t += ncl) {
             mbar_wait(&tempty[acc], acc_phase ^ 1);
             tc_fence_after();
             const uint32_t d = tmem + (uint32_t)(acc * BN);
@@ -166,14 +206,11 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
                     const uint32_t sb = sa + kABytes;
 #pragma unroll
                     for (int k = 0; k < BK / 16; ++k) {
-                        // A: K-major SW128, +32 B per 16-element K step; SBO = 8 rows x 128 B
                         const uint64_t da = sdesc(sa + k * 32, 16, 1024);
-                        // B: MN-major SW128, 64-column chunks 8 KiB apart (LBO), 8-row k groups 1 KiB
-                        // apart (SBO); +2 KiB per 16 k rows
                         const uint64_t db = sdesc(sb + k * 2048, BK * 128, 1024);
                         tc_mma(d, da, db, kIdesc, (kb | k) ? 1u : 0u);
                     }
-                    tc_commit(&empty[stage]);
+                    tc_commit_mc1(&empty[stage], (uint16_t)0x3);
                 }
                 __syncwarp();
                 if (++stage == kStages) { stage = 0; phase ^= 1; }
@@ -183,20 +220,17 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
             if (++acc == 2) { acc = 0; acc_phase ^= 1; }
         }
     } else {
-        // epilogue warps 2..5: TMEM lane quarter = warp % 4
         const int q = warp & 3;
         int acc = 0;
         uint32_t acc_phase = 0;
-        for (int64_t t = blockIdx.x; t < num_tiles; t += gridDim.x) {
-            int mb, nb;
-            tile_coords(t, num_m, num_n, mb, nb);
+        for (int64_t t = cl; t < num_tiles; t += ncl) {
+            int mp, nb;
+            tile_coords(t, num_mp, num_n, mp, nb);
             mbar_wait(&tfull[acc], acc_phase);
             tc_fence_after();
-            const int64_t row = m0 + (int64_t)mb * BM + q * 32 + lane;
+            const int64_t row = m0 + (int64_t)(2 * mp + (int)rank) * BM + q * 32 + lane;
             float* crow = C + row * N + (int64_t)nb * BN;
             const bool ok = row < m1;
-            // columns of this tile inside C (a partial last n-block: the TMA zero-filled B's columns
-            // past N, their accumulators are not stored)
             const int ncols = (int)((N - (int64_t)nb * BN) < BN ? (N - (int64_t)nb * BN) : BN);
 #pragma unroll 1
             for (int c = 0; c < BN / 32; ++c) {
@@ -227,11 +261,10 @@ gemm_kernel(const __grid_constant__ CUtensorMap map_a, const __grid_constant__ C
         }
     }
     tc_fence_before();
-    __syncthreads();
+    cluster_sync_all();  // no multicast or remote arrive may target a CTA that has exited
     tc_fence_after();
     if (warp == 1) asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem), "r"(kTmemCols));
 }
-
 
 bool make_map(CUtensorMap* m, const void* base, uint64_t inner, uint64_t outer, uint64_t row_bytes, uint32_t box_in,
               uint32_t box_out) {
@@ -265,9 +298,24 @@ cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M,
     const size_t smem = 1024 + (size_t)kStages * kStageBytes + 256;
     cudaError_t e = kernel_prep(gemm_kernel, kThreads, smem);
     if (e != cudaSuccess) return e;
-    const int64_t tiles = ((m1 - m0 + BM - 1) / BM) * ((N + BN - 1) / BN);
-    const int grid = (int)(tiles < sms ? tiles : sms);
-    gemm_kernel<<<grid, kThreads, smem, s>>>(ma, mb, C, N, K, m0, m1, row_lo);
+    // one cluster of two CTAs per SM pair, persistent over the pair tiles (2 m-blocks x 1 n-block)
+    const int64_t ptiles = ((m1 - m0 + 2 * BM - 1) / (2 * BM)) * ((N + BN - 1) / BN);
+    int64_t ncl = sms / 2;
+    if (ptiles < ncl) ncl = ptiles;
+    cudaLaunchConfig_t cfg{};
+    cfg.gridDim = dim3((unsigned)(2 * ncl));
+    cfg.blockDim = dim3(kThreads);
+    cfg.dynamicSmemBytes = smem;
+    cfg.stream = s;
+    cudaLaunchAttribute at[1];
+    at[0].id = cudaLaunchAttributeClusterDimension;
+    at[0].val.clusterDim.x = 2;
+    at[0].val.clusterDim.y = 1;
+    at[0].val.clusterDim.z = 1;
+    cfg.attrs = at;
+    cfg.numAttrs = 1;
+    e = cudaLaunchKernelEx(&cfg, gemm_kernel, ma, mb, C, N, K, m0, m1, row_lo);
+    if (e != cudaSuccess) return e;
     if (launches) *launches += 1;
     return cudaGetLastError();
 }

@@ -1,6 +1,6 @@
 #!/bin/bash
 # Round-2 evidence run (one B200): GPU suite, bench lines, all configs, ncu captures, k-means timeline.
-O=gpurun_out/r02
+O=${1:-gpurun_out/r02}
 mkdir -p $O
 python -m pytest tests -m gpu -q -rs > $O/pytest_gpu.log 2>&1
 python bench.py > $O/bench.jsonl 2> $O/bench.err
