@@ -140,3 +140,30 @@ def write_mask(seed: int, n: int, density: float, run: int = 1) -> np.ndarray:
 def bf16_to_f32(a: np.ndarray) -> np.ndarray:
     """Exact widening of bf16 bit patterns to fp32 (a bit shift, no rounding)."""
     return (a.astype(np.uint32) << 16).view(np.float32)
+
+
+def kmeans_points_real(seed: int, n: int, d: int, k: int) -> np.ndarray:
+    """Real-valued k-means input in the style of the paper's KMEANS data (kddcup feature vectors,
+    Table II): arbitrary fp32 values, not on any fixed-point grid. Per dimension a kind is drawn:
+    non-negative counts (integers, heavy tailed), rates in [0, 1] (full 24-bit mantissas), or
+    signed real values with magnitudes spread over ~40 binades; points scatter multiplicatively
+    around k seeded centres; about 10 % of the values are zero. Seeded numpy PCG64."""
+    rng = np.random.default_rng(seed)
+    kinds = rng.integers(0, 3, d)
+    centres = np.empty((k, d))
+    for j in range(d):
+        if kinds[j] == 0:
+            centres[:, j] = np.floor(rng.lognormal(3.0, 2.0, k))
+        elif kinds[j] == 1:
+            centres[:, j] = rng.random(k)
+        else:
+            centres[:, j] = rng.choice([-1.0, 1.0], k) * 2.0 ** rng.uniform(-20, 20, k)
+    lab = rng.integers(0, k, n)
+    x = centres[lab] * (1.0 + 0.05 * rng.standard_normal((n, d)))
+    for j in range(d):
+        if kinds[j] == 0:
+            x[:, j] = np.floor(np.abs(x[:, j]))
+        elif kinds[j] == 1:
+            x[:, j] = np.clip(x[:, j], 0.0, 1.0)
+    x[rng.random((n, d)) < 0.1] = 0.0
+    return np.ascontiguousarray(x.astype(np.float32))

@@ -182,6 +182,44 @@ def kmeans_run(x: np.ndarray, k: int, iters: int, nthreads: int = 0):
     return cen, m
 
 
+def kmeans_update_exact(x: np.ndarray, member: np.ndarray, cen: np.ndarray) -> np.ndarray:
+    """KMEANS update loop for arbitrary finite fp32 points (Table II; reductiontoarray
+    L75-77, L89-91; reading KM-X in DESIGN.md §2): the new centroid is the mean of its members,
+
+        cen[c][j] = (float)( RN64(sum over p in c of x[p][j]) / (double)cnt[c] )   if cnt[c] > 0,
+
+    the exact real sum rounded once to double (math.fsum is correctly rounded), then the fp64
+    division and the rounding to fp32; empty clusters keep their centroid. On points for which
+    every fp64 partial sum is exact (the 2^-shift grid of reading W4) this is the sequential-fp64
+    update of orc_kmeans_update. Updates cen in place; returns the counts."""
+    import math
+    k, d = cen.shape
+    assert np.all(np.isfinite(x)), "exact mode takes finite points"
+    cnt = np.bincount(member, minlength=k).astype(np.int64)
+    order = np.argsort(member, kind="stable")
+    bounds = np.concatenate(([0], np.cumsum(cnt)))
+    xs = x[order].astype(np.float64)  # fp32 -> fp64 is exact
+    for c in range(k):
+        if cnt[c] == 0:
+            continue
+        rows = xs[bounds[c]:bounds[c + 1]]
+        for j in range(d):
+            cen[c, j] = np.float32(math.fsum(rows[:, j].tolist()) / float(cnt[c]))
+    return cnt
+
+
+def kmeans_run_exact(x: np.ndarray, k: int, iters: int, nthreads: int = 0):
+    """cen[c] = x[c] for c < k, then `iters` x (assignment: orc_kmeans_assign, the scalar fmaf loop;
+    update: kmeans_update_exact). Returns (centroids after the last update, member of the last
+    assignment)."""
+    cen = np.ascontiguousarray(x[:k]).astype(np.float32).copy()
+    m = np.zeros(x.shape[0], dtype=np.int32)
+    for _ in range(iters):
+        m = kmeans_assign(x, cen, nthreads)
+        kmeans_update_exact(x, m, cen)
+    return cen, m
+
+
 def scatter(src: np.ndarray, idx: np.ndarray, dst: np.ndarray, P: int = 0):
     """dst[idx[i]] = src[i] in place; returns per-partition write-miss counts if P > 0."""
     miss = np.zeros(max(P, 1), dtype=np.int64)
