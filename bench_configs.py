@@ -150,7 +150,7 @@ def gemm_cfg(N, P, reps, check):
     return out
 
 
-def kmeans_cfg(n, iters, P, check):
+def kmeans_cfg(n, iters, P, check, exact=False):
     d, k = 16, 256
     pk = peaks()
     t0 = time.perf_counter()
@@ -158,15 +158,16 @@ def kmeans_cfg(n, iters, P, check):
     tgen = time.perf_counter() - t0
     cen = np.ascontiguousarray(x[:k]).copy()
     member = np.zeros(n, dtype=np.int32)
-    sums = np.zeros((k, d), dtype=np.int64)
+    shift = A.KMEANS_EXACT if exact else 8  # exact mode: the general-data path (nine windows per sum)
+    sums = np.zeros((k, d, A.KMEANS_WINDOWS) if exact else (k, d), dtype=np.int64)
     cnt = np.zeros(k, dtype=np.int64)
     A.accmg_init(num_partitions=P, device=0, profile=1)
     try:
         regs = [A.accmg_region_create(a) for a in (x, cen, member, sums, cnt)]
-        WL.kmeans_loops(*regs, n, d, k)  # iteration 1 (copy-in) untimed
+        WL.kmeans_loops(*regs, n, d, k, shift)  # iteration 1 (copy-in) untimed
         A.accmg_barrier()
         A.accmg_reset_stats()
-        t = wall(lambda: [WL.kmeans_loops(*regs, n, d, k) for _ in range(iters - 1)])
+        t = wall(lambda: [WL.kmeans_loops(*regs, n, d, k, shift) for _ in range(iters - 1)])
         st = A.accmg_get_stats()
         A.accmg_sync_to_host(regs[1])
         A.accmg_sync_to_host(regs[2])
@@ -174,9 +175,9 @@ def kmeans_cfg(n, iters, P, check):
         A.accmg_finalize()
     its = iters - 1
     ms_assign = st["ms_body"] / its  # body time includes the (tiny) update loop
-    out = {"config": "c4", "P": P, "n": n, "iters_timed": its, "iters_per_s": n * its / t,
+    out = {"config": "c4x" if exact else "c4", "P": P, "n": n, "iters_timed": its, "iters_per_s": n * its / t,
            "ms_per_iteration": t / its * 1e3, **per_loop(st, 2 * its), "gen_s": tgen}
-    impl = "tc" if k <= 256 else "fp32"
+    impl = "exact" if exact else ("tc" if k <= 256 else "fp32")
     # HBM view: 64 B of point coordinates read + 4 B of assignment written per point
     out["assign_hbm_gbs"] = n * (d * 4 + 4) / (ms_assign / 1e3) / 1e9
     out["assign_frac_of_measured_hbm"] = out["assign_hbm_gbs"] / pk["hbm_gbs"]
@@ -378,6 +379,8 @@ def main():
                     emit(scatter_cfg(1 << 26, P, 5))
                 elif cfg == "c4":
                     emit(kmeans_cfg(a.kmeans_n, a.kmeans_iters, P, a.check))
+                elif cfg == "c4x":  # C4 through exact mode (arbitrary-data path: scalar loop + windows)
+                    emit(kmeans_cfg(a.kmeans_n, a.kmeans_iters, P, a.check, exact=True))
             except Exception as e:  # report and continue with the next config
                 emit({"config": cfg, "P": P, "error": repr(e)})
 

@@ -160,9 +160,16 @@ typedef struct accmg_access {
  *   member[p] = argmin_c fmaf-chain sum_j (x[p][j]-cen[c][j])^2 (lowest c on ties);
  *   sums[member[p]][j] += x[p][j] * 2^shift (exact int64; x must lie on the 2^-shift grid with
  *   |x * 2^shift| < 2^31, else ACCMG_EDATA); counts[member[p]] += 1.
+ *   Exact mode, shift = ACCMG_KMEANS_EXACT (reading KM-X; arbitrary finite fp32 points, d <= 64,
+ *   k*d <= 16384): sums is int64 k*d*ACCMG_KMEANS_WINDOWS; the exact real sum of the members'
+ *   x[p][j] is kept as sum_w sums[c][j][w] * 2^(32w - 149) (every addend below 2^32 in
+ *   magnitude: exact for n < 2^31); a non-finite x gives ACCMG_EDATA.
  * ACCMG_BODY_KMEANS_UPDATE: bounds ndim=1 [0,k);
- *   descs [sums RW (int64 k*d), counts RW (int64 k), centroids W (fp32 k*d)];
+ *   descs [sums RW (int64 k*d, or k*d*ACCMG_KMEANS_WINDOWS in exact mode), counts RW (int64 k),
+ *   centroids W (fp32 k*d)];
  *   if counts[c] > 0: cen[c][j] = (float)(((double)sums[c][j] * 2^-shift) / (double)counts[c]);
+ *   exact mode: cen[c][j] = (float)(RN64(exact sum) / (double)counts[c]) (the mean of the members:
+ *   the exact sum rounded once to double, PAPER.md L219-226 / L89-91);
  *   then sums[c][*] = 0, counts[c] = 0.
  * ACCMG_BODY_JACOBI2D_DEEP: as ACCMG_BODY_JACOBI2D_5PT but each loop performs h sweeps (deep halos,
  *   §8 row f2): dst = J^h(src) on the bounds box, J the 5-point sweep above, rows/columns outside
@@ -202,6 +209,8 @@ typedef struct accmg_access {
 typedef struct { int64_t rows, cols; } accmg_args_jacobi2d;
 typedef struct { int64_t M, N, K; } accmg_args_gemm;
 typedef struct { int64_t n; int32_t d, k, shift, pad; } accmg_args_kmeans;
+#define ACCMG_KMEANS_EXACT   (-1) /* accmg_args_kmeans.shift: arbitrary finite points (exact sums) */
+#define ACCMG_KMEANS_WINDOWS 9    /* int64 windows per (cluster, dim) of the exact-mode sums */
 typedef struct { int64_t rows, cols, period; } accmg_args_sparse;
 typedef struct { int64_t n; } accmg_args_masked;
 typedef struct { int64_t n, m; } accmg_args_scatter;

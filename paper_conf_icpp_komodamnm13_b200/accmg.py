@@ -29,6 +29,7 @@ HALO_AUTO, HALO_PULL = 0, 1
 MC_OFF, MC_AUTO, MC_VMM = 0, 1, 2
 R, W, RW, REDUCE_SUM = 1, 2, 3, 4
 BODY_JACOBI2D_5PT, BODY_GEMM_BF16_F32, BODY_KMEANS_ASSIGN, BODY_KMEANS_UPDATE = 1, 2, 3, 4
+KMEANS_EXACT, KMEANS_WINDOWS = -1, 9  # accmg_args_kmeans.shift for arbitrary finite points; windows
 BODY_SCATTER = 5
 BODY_JACOBI3D_7PT = 6
 BODY_JACOBI2D_DEEP = 7

@@ -394,6 +394,192 @@ update_counts(int64_t* __restrict__ counts, int64_t c0, int64_t c1, Track t) {
     }
 }
 
+// ---- exact mode (args.shift = -1): arbitrary finite fp32 points (reading KM-X in DESIGN.md) -----
+// The centroid update needs RN64(exact sum of the members' values): each value x = m * 2^(o - 149)
+// (m the 24-bit significand, o = biased exponent - 1, or 0 for subnormals) is added exactly into
+// nine 32-bit-aligned windows, A_w of weight 2^(32 w - 149): m * 2^(o mod 32) < 2^55 splits into a
+// low 32-bit part for window o / 32 and a high part for the next one. Every addend is below 2^32
+// in magnitude, so an int64 window holds the sum of up to 2^31 of them exactly; the sums region
+// holds k * d * 9 such windows (REDUCE_SUM merges them elementwise like any int64 partials).
+constexpr int kSuperW = 9;
+
+__device__ __forceinline__ void superacc_add(unsigned long long* acc, float v, int* err) {
+    const uint32_t b = __float_as_uint(v);
+    const uint32_t ex = (b >> 23) & 255u;
+    if (ex == 255u) {  // inf / NaN: no exact mean
+        atomicOr(err, 1);
+        return;
+    }
+    uint32_t m = b & 0x7FFFFFu;
+    if (ex) m |= 0x800000u;
+    if (!m) return;
+    const int o = ex ? (int)ex - 1 : 0;
+    const uint64_t t = (uint64_t)m << (o & 31);
+    unsigned long long lo = t & 0xFFFFFFFFull, hi = t >> 32;
+    if (b >> 31) {
+        lo = 0ull - lo;
+        hi = 0ull - hi;
+    }
+    if (lo) atomicAdd(acc + (o >> 5), lo);
+    if (hi) atomicAdd(acc + (o >> 5) + 1, hi);
+}
+
+// Assignment (the scalar loop, any data) + exact reductiontoarray into the windows. DM >= d: the
+// point lives in registers. Windows and counts in shared memory when they fit (flushed once per
+// block), else straight into the partition's partials.
+template <int DM, bool SHARED_ACC>
+__global__ void __launch_bounds__(kThreads)
+assign_exact_k(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __restrict__ member,
+               int64_t* __restrict__ sacc, int64_t* __restrict__ counts, int64_t p0, int64_t p1, int d, int kc,
+               int* err) {
+    extern __shared__ __align__(16) unsigned char smem_e[];
+    unsigned long long* s_cnt = reinterpret_cast<unsigned long long*>(smem_e);
+    unsigned long long* s_acc = s_cnt + kc;
+    float* s_c = reinterpret_cast<float*>(SHARED_ACC ? s_acc + (size_t)kc * d * kSuperW : s_acc);
+    for (int i = threadIdx.x; i < kc * d; i += blockDim.x) s_c[i] = cen[i];
+    for (int i = threadIdx.x; i < kc; i += blockDim.x) s_cnt[i] = 0ull;
+    if constexpr (SHARED_ACC)
+        for (int i = threadIdx.x; i < kc * d * kSuperW; i += blockDim.x) s_acc[i] = 0ull;
+    __syncthreads();
+    unsigned long long* acc = SHARED_ACC ? s_acc : reinterpret_cast<unsigned long long*>(sacc);
+    for (int64_t p = p0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < p1; p += (int64_t)gridDim.x * blockDim.x) {
+        float xv[DM];
+#pragma unroll
+        for (int j = 0; j < DM; ++j) xv[j] = j < d ? x[p * d + j] : 0.f;
+        float bd = __int_as_float(0x7f800000);
+        int bi = 0;
+        for (int c = 0; c < kc; ++c) {
+            float a = 0.f;
+#pragma unroll
+            for (int j = 0; j < DM; ++j)
+                if (j < d) {
+                    const float df = __fsub_rn(xv[j], s_c[c * d + j]);
+                    a = __fmaf_rn(df, df, a);
+                }
+            if (a < bd) { bd = a; bi = c; }
+        }
+        member[p] = bi;
+        atomicAdd(s_cnt + bi, 1ull);
+#pragma unroll
+        for (int j = 0; j < DM; ++j)
+            if (j < d) superacc_add(acc + ((size_t)bi * d + j) * kSuperW, xv[j], err);
+    }
+    __syncthreads();
+    if constexpr (SHARED_ACC)
+        for (int i = threadIdx.x; i < kc * d * kSuperW; i += blockDim.x)
+            if (s_acc[i]) atomicAdd(reinterpret_cast<unsigned long long*>(sacc) + i, s_acc[i]);
+    for (int i = threadIdx.x; i < kc; i += blockDim.x)
+        if (s_cnt[i]) atomicAdd(reinterpret_cast<unsigned long long*>(counts) + i, s_cnt[i]);
+}
+
+// RN64 of sum_w A[w] * 2^(32 w - 149): carry-normalise to base-2^32 digits (two's complement over
+// ten digits), take the magnitude, round its leading 96 bits to 53 with a sticky bit for the rest
+// (ties to even). The exact sum of fp32 values is 0 or of magnitude in [2^-149, 2^160): a normal
+// double, so the scaling is exact.
+__device__ double superacc_round(const int64_t* __restrict__ A) {
+    uint32_t dg[kSuperW + 1];
+    long long carry = 0;
+#pragma unroll
+    for (int w = 0; w < kSuperW; ++w) {
+        const __int128 t = (__int128)A[w] + carry;
+        dg[w] = (uint32_t)(unsigned long long)t;
+        carry = (long long)(t >> 32);
+    }
+    dg[kSuperW] = (uint32_t)carry;
+    const bool neg = carry < 0;
+    if (neg) {  // magnitude: invert and add one
+        unsigned long long c1 = 1ull;
+#pragma unroll
+        for (int w = 0; w <= kSuperW; ++w) {
+            const unsigned long long t = (unsigned long long)(uint32_t)~dg[w] + c1;
+            dg[w] = (uint32_t)t;
+            c1 = t >> 32;
+        }
+    }
+    int top = -1;
+#pragma unroll
+    for (int w = 0; w <= kSuperW; ++w)
+        if (dg[w]) top = w;
+    if (top < 0) return 0.0;
+    uint32_t d1 = 0u, d2 = 0u;
+    bool sticky = false;
+#pragma unroll
+    for (int w = 0; w <= kSuperW; ++w) {
+        if (w == top - 1) d1 = dg[w];
+        if (w == top - 2) d2 = dg[w];
+        if (w < top - 2 && dg[w]) sticky = true;
+    }
+    const unsigned __int128 M = ((unsigned __int128)dg[top] << 64) | ((unsigned __int128)d1 << 32) | d2;
+    const int lead = 95 - __clz(dg[top]);  // leading bit of M
+    const int sh = lead - 52;              // 12..43
+    unsigned long long mant = (unsigned long long)(M >> sh);
+    const unsigned __int128 rem = M & ((((unsigned __int128)1) << sh) - 1);
+    const unsigned __int128 half = ((unsigned __int128)1) << (sh - 1);
+    if (rem > half || (rem == half && (sticky || (mant & 1ull)))) ++mant;  // 2^53 stays exact
+    const double r = ldexp((double)mant, sh + 32 * (top - 2) - 149);
+    return neg ? -r : r;
+}
+
+// Update, element pass (exact mode): if counts[c] > 0: cen[e] = (float)(RN64(sum) / counts[c]).
+template <bool TRACK>
+__global__ void __launch_bounds__(kThreads)
+update_exact_elems(const int64_t* __restrict__ sacc, const int64_t* __restrict__ counts, float* __restrict__ cen,
+                   int64_t c0, int64_t c1, int d, Track tc) {
+    const int64_t e0 = c0 * d, e1 = c1 * d;
+    int64_t cc = -1;
+    for (int64_t base = e0 + (int64_t)blockIdx.x * kThreads; base < e1; base += (int64_t)gridDim.x * kThreads) {
+        const int64_t e = base + threadIdx.x;
+        bool wc = false;
+        if (e < e1) {
+            const int64_t cnt = counts[e / d];
+            if (cnt > 0) {
+                cen[e] = __double2float_rn(__ddiv_rn(superacc_round(sacc + e * kSuperW), (double)cnt));
+                wc = true;
+            }
+        }
+        if constexpr (TRACK) {
+            if (tc.l1) dev::track_warp<1>(tc.l1, tc.l2, tc.l2_shift, base + (threadIdx.x & ~31), wc ? 1u : 0u, cc);
+        }
+    }
+}
+
+// Update, window pass (exact mode): sums[q] = 0 for the windows of clusters [c0, c1).
+template <bool TRACK>
+__global__ void __launch_bounds__(kThreads)
+update_exact_zero(int64_t* __restrict__ sacc, int64_t q0, int64_t q1, Track ts) {
+    int64_t cs = -1;
+    for (int64_t base = q0 + (int64_t)blockIdx.x * kThreads; base < q1; base += (int64_t)gridDim.x * kThreads) {
+        const int64_t q = base + threadIdx.x;
+        if (q < q1) sacc[q] = 0;
+        if constexpr (TRACK) {
+            if (ts.l1) dev::track_warp<1>(ts.l1, ts.l2, ts.l2_shift, base + (threadIdx.x & ~31), q < q1 ? 1u : 0u, cs);
+        }
+    }
+}
+
+template <int DM>
+cudaError_t launch_assign_exact(const float* x, const float* cen, int32_t* member, int64_t* sacc, int64_t* counts,
+                                int64_t p0, int64_t p1, int d, int kc, int* err, cudaStream_t s, int sms) {
+    const size_t base = (size_t)kc * 8 + (size_t)kc * d * 4;
+    const size_t shared_acc = base + (size_t)kc * d * kSuperW * 8;
+    const bool sh = shared_acc <= 160 * 1024;
+    const size_t smem = sh ? shared_acc : base;
+    cudaError_t e = sh ? kernel_prep(assign_exact_k<DM, true>, kThreads, smem)
+                       : kernel_prep(assign_exact_k<DM, false>, kThreads, smem);
+    if (e != cudaSuccess) return e;
+    int per_sm = 1;
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sh ? (const void*)assign_exact_k<DM, true>
+                                                              : (const void*)assign_exact_k<DM, false>, kThreads, smem);
+    if (per_sm < 1) per_sm = 1;
+    int64_t blocks = (p1 - p0 + kThreads - 1) / kThreads;
+    if (blocks > (int64_t)sms * per_sm) blocks = (int64_t)sms * per_sm;
+    if (sh)
+        assign_exact_k<DM, true><<<(unsigned)blocks, kThreads, smem, s>>>(x, cen, member, sacc, counts, p0, p1, d, kc, err);
+    else
+        assign_exact_k<DM, false><<<(unsigned)blocks, kThreads, smem, s>>>(x, cen, member, sacc, counts, p0, p1, d, kc, err);
+    return cudaGetLastError();
+}
+
 int sm_count() {
     static int n = 0;
     if (!n) {
@@ -412,6 +598,14 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
                           int64_t* launches) {
     if (p1 <= p0) return cudaSuccess;
     const int sms = sm_count();
+    if (shift < 0) {  // exact mode (arbitrary finite points; sums = k * d * 9 windows)
+        if (d > 64 || (int64_t)kc * d > 16384) return cudaErrorNotSupported;
+        cudaError_t e = d <= 16   ? launch_assign_exact<16>(x, cen, member, sums, counts, p0, p1, d, kc, err_flag, s, sms)
+                        : d <= 32 ? launch_assign_exact<32>(x, cen, member, sums, counts, p0, p1, d, kc, err_flag, s, sms)
+                                  : launch_assign_exact<64>(x, cen, member, sums, counts, p0, p1, d, kc, err_flag, s, sms);
+        if (e == cudaSuccess && launches) *launches += 1;
+        return e;
+    }
     // the tensor-core filter + exact re-check (kmeans_tc.cu) where supported (d = 16, k <= 256);
     // the FP32-pipe kernels below otherwise
     if (kmeans_tc_supported(x, d, kc)) {
@@ -456,6 +650,21 @@ cudaError_t kmeans_update(int64_t* sums, int64_t* counts, float* cen, int64_t c0
     const bool tr = t_sums.l1 || t_cen.l1;
     int64_t nb = ((c1 - c0) * d + kThreads - 1) / kThreads;
     if (nb > 1184) nb = 1184;
+    if (shift < 0) {  // exact mode: the element pass reads all windows before the window pass clears them
+        if (t_cen.l1) update_exact_elems<true><<<(unsigned)nb, kThreads, 0, s>>>(sums, counts, cen, c0, c1, d, t_cen);
+        else update_exact_elems<false><<<(unsigned)nb, kThreads, 0, s>>>(sums, counts, cen, c0, c1, d, t_cen);
+        const int64_t q0 = c0 * d * kSuperW, q1 = c1 * d * kSuperW;
+        int64_t nq = (q1 - q0 + kThreads - 1) / kThreads;
+        if (nq > 1184) nq = 1184;
+        if (t_sums.l1) update_exact_zero<true><<<(unsigned)nq, kThreads, 0, s>>>(sums, q0, q1, t_sums);
+        else update_exact_zero<false><<<(unsigned)nq, kThreads, 0, s>>>(sums, q0, q1, t_sums);
+        int64_t nc = (c1 - c0 + kThreads - 1) / kThreads;
+        if (nc > 1184) nc = 1184;
+        if (t_counts.l1) update_counts<true><<<(unsigned)nc, kThreads, 0, s>>>(counts, c0, c1, t_counts);
+        else update_counts<false><<<(unsigned)nc, kThreads, 0, s>>>(counts, c0, c1, t_counts);
+        if (launches) *launches += 3;
+        return cudaGetLastError();
+    }
     if (tr) update_elems<true><<<(unsigned)nb, kThreads, 0, s>>>(sums, counts, cen, c0, c1, d, shift, t_sums, t_cen);
     else update_elems<false><<<(unsigned)nb, kThreads, 0, s>>>(sums, counts, cen, c0, c1, d, shift, t_sums, t_cen);
     int64_t nc = (c1 - c0 + kThreads - 1) / kThreads;

@@ -797,15 +797,20 @@ int validate_body(const accmg_bounds* bd, int body, const accmg_access* d, const
         case ACCMG_BODY_KMEANS_ASSIGN:
         case ACCMG_BODY_KMEANS_UPDATE: {
             auto a = static_cast<const accmg_args_kmeans*>(args);
-            if (a->n < 1 || a->d < 1 || a->k < 1 || a->shift < 0 || a->shift > 30) return bad("kmeans: n, d, k >= 1, shift in [0,30]");
-            if (a->d > 32 || a->k > 1024) return fail(ACCMG_EUNSUPPORTED, "kmeans: d <= 32, k <= 1024", false);
+            if (a->n < 1 || a->d < 1 || a->k < 1 || a->shift < ACCMG_KMEANS_EXACT || a->shift > 30)
+                return bad("kmeans: n, d, k >= 1, shift in [0,30] or ACCMG_KMEANS_EXACT");
+            const bool exact = a->shift == ACCMG_KMEANS_EXACT;
+            if (exact ? (a->d > 64 || a->k > 1024 || (int64_t)a->k * a->d > 16384) : (a->d > 32 || a->k > 1024))
+                return fail(ACCMG_EUNSUPPORTED, "kmeans: d <= 32, k <= 1024 (exact mode: d <= 64, k*d <= 16384)", false);
+            // exact mode: the sums region holds ACCMG_KMEANS_WINDOWS int64 windows per (cluster, dim)
+            const int64_t sum_ext = (int64_t)a->k * a->d * (exact ? ACCMG_KMEANS_WINDOWS : 1);
             if (body == ACCMG_BODY_KMEANS_ASSIGN) {
                 if (ext(0) != a->n * a->d || ext(1) != (int64_t)a->k * a->d || ext(2) != a->n ||
-                    ext(3) != (int64_t)a->k * a->d || ext(4) != a->k)
+                    ext(3) != sum_ext || ext(4) != a->k)
                     return bad("kmeans_assign: extents");
                 if (bd->lo[0] < 0 || bd->hi[0] > a->n) return bad("kmeans_assign: bounds outside [0,n)");
             } else {
-                if (ext(0) != (int64_t)a->k * a->d || ext(1) != a->k || ext(2) != (int64_t)a->k * a->d)
+                if (ext(0) != sum_ext || ext(1) != a->k || ext(2) != (int64_t)a->k * a->d)
                     return bad("kmeans_update: extents");
                 if (bd->lo[0] < 0 || bd->hi[0] > a->k) return bad("kmeans_update: bounds outside [0,k)");
             }
@@ -1170,7 +1175,8 @@ int check_data_flag() {
         CUDA_TRY(cudaMemsetAsync(S.d_flag + 1, 0, 2 * sizeof(int), S.stream));
         CUDA_TRY(cudaStreamSynchronize(S.stream));
         if (grid)
-            return fail(ACCMG_EDATA, "kmeans: a point is not on the 2^-shift fixed-point grid (|x*2^shift| < 2^31)", false);
+            return fail(ACCMG_EDATA, "kmeans: a point is not on the 2^-shift fixed-point grid (|x*2^shift| < 2^31), "
+                                     "or not finite in exact mode", false);
         return fail(ACCMG_EDATA, "scatter: an index lies in no partition's write window (negative, >= m, or a gap); "
                                  "its write was dropped", false);
     }

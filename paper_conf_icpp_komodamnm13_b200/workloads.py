@@ -86,11 +86,13 @@ def kmeans_loops(rx, rcen, rmem, rsum, rcnt, n: int, d: int, k: int, shift: int 
 
 
 def kmeans_run(x: np.ndarray, k: int, iters: int, shift: int = 8):
-    """Rodinia-style k-means (centroids start at the first k points). Returns (centroids, member)."""
+    """Rodinia-style k-means (centroids start at the first k points). Returns (centroids, member).
+    shift = KMEANS_EXACT: arbitrary finite points (exact sums, centroid = RN64(sum) / count)."""
     n, d = x.shape
     cen = np.ascontiguousarray(x[:k]).copy()
     member = np.zeros(n, dtype=np.int32)
-    sums = np.zeros((k, d), dtype=np.int64)
+    # exact mode (shift = KMEANS_EXACT): nine int64 windows per (cluster, dim)
+    sums = np.zeros((k, d, A.KMEANS_WINDOWS) if shift == A.KMEANS_EXACT else (k, d), dtype=np.int64)
     cnt = np.zeros(k, dtype=np.int64)
     regs = [A.accmg_region_create(a) for a in (x, cen, member, sums, cnt)]
     try:

@@ -282,3 +282,29 @@ def test_kmeans_assign_reduction_plan_vs_model(dry, P):
         for key in ("reduce", "declared", "h2d", "interpartition"):
             assert after["bytes_" + key] - before["bytes_" + key] == exp[key], key
         _compare_valid([rx, rc, rm, rs, rn], [mx, mc, mm, ms, mn], P)
+
+
+def test_kmeans_exact_mode_extents(dry):
+    """Exact mode (shift = KMEANS_EXACT) takes a sums region of k*d*9 int64 windows (and rejects the
+    fixed-point extent k*d), accepts d up to 64, and counts the windows in the reduction bytes."""
+    n, d, k = 500, 40, 9
+    dry(2)
+    hx, hc, hm = np.zeros((n, d), np.float32), np.zeros((k, d), np.float32), np.zeros(n, np.int32)
+    hn = np.zeros(k, np.int64)
+    rx, rc, rm, rn = (A.accmg_region_create(a) for a in (hx, hc, hm, hn))
+    r_small = A.accmg_region_create(np.zeros((k, d), np.int64))
+    r_win = A.accmg_region_create(np.zeros((k, d, A.KMEANS_WINDOWS), np.int64))
+
+    def launch(rs, shift):
+        A.accmg_loop_launch(A.bounds([0], [n]), A.BODY_KMEANS_ASSIGN,
+                            [A.access(rx, A.R, True, d, 0, 0), A.access(rc, A.R), A.access(rm, A.W, True, 1, 0, 0),
+                             A.access(rs, A.REDUCE_SUM), A.access(rn, A.REDUCE_SUM)], A.accmg_args_kmeans(n, d, k, shift))
+    with pytest.raises(A.AccmgError) as ei:
+        launch(r_small, A.KMEANS_EXACT)
+    assert ei.value.code == A.EINVAL
+    with pytest.raises(A.AccmgError) as ei:
+        launch(r_win, 8)  # d = 40 > 32 in fixed-point mode
+    assert ei.value.code == A.EUNSUPPORTED
+    before = A.accmg_get_stats()["bytes_reduce"]
+    launch(r_win, A.KMEANS_EXACT)
+    assert A.accmg_get_stats()["bytes_reduce"] - before == 2 * (k * d * A.KMEANS_WINDOWS * 8 + k * 8)
