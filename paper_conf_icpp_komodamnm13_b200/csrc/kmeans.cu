@@ -425,44 +425,75 @@ __device__ __forceinline__ void superacc_add(unsigned long long* acc, float v, i
 }
 
 // Assignment (the scalar loop, any data) + exact reductiontoarray into the windows. DM >= d: the
-// point lives in registers. Windows and counts in shared memory when they fit (flushed once per
-// block), else straight into the partition's partials.
-template <int DM, bool SHARED_ACC>
+// points live in registers, NPT points per thread share every centroid load (rows padded to a
+// multiple of 4 floats in shared memory, one LDS.128 per 4 dims). Windows and counts in shared
+// memory when they fit (flushed once per block), else straight into the partition's partials.
+template <int DM, int NPT, bool SHARED_ACC>
 __global__ void __launch_bounds__(kThreads)
 assign_exact_k(const float* __restrict__ x, const float* __restrict__ cen, int32_t* __restrict__ member,
                int64_t* __restrict__ sacc, int64_t* __restrict__ counts, int64_t p0, int64_t p1, int d, int kc,
                int* err) {
     extern __shared__ __align__(16) unsigned char smem_e[];
-    unsigned long long* s_cnt = reinterpret_cast<unsigned long long*>(smem_e);
+    const int dp = (d + 3) & ~3;  // padded centroid row
+    float4* s_c4 = reinterpret_cast<float4*>(smem_e);
+    float* s_c = reinterpret_cast<float*>(smem_e);
+    unsigned long long* s_cnt = reinterpret_cast<unsigned long long*>(smem_e + (size_t)kc * dp * 4);
     unsigned long long* s_acc = s_cnt + kc;
-    float* s_c = reinterpret_cast<float*>(SHARED_ACC ? s_acc + (size_t)kc * d * kSuperW : s_acc);
-    for (int i = threadIdx.x; i < kc * d; i += blockDim.x) s_c[i] = cen[i];
+    for (int i = threadIdx.x; i < kc * dp; i += blockDim.x) {
+        const int c = i / dp, j = i - c * dp;
+        s_c[i] = j < d ? cen[c * d + j] : 0.f;
+    }
     for (int i = threadIdx.x; i < kc; i += blockDim.x) s_cnt[i] = 0ull;
     if constexpr (SHARED_ACC)
         for (int i = threadIdx.x; i < kc * d * kSuperW; i += blockDim.x) s_acc[i] = 0ull;
     __syncthreads();
     unsigned long long* acc = SHARED_ACC ? s_acc : reinterpret_cast<unsigned long long*>(sacc);
-    for (int64_t p = p0 + (int64_t)blockIdx.x * blockDim.x + threadIdx.x; p < p1; p += (int64_t)gridDim.x * blockDim.x) {
-        float xv[DM];
+    const int64_t step = (int64_t)gridDim.x * blockDim.x * NPT;
+    for (int64_t pb = p0 + (int64_t)blockIdx.x * blockDim.x * NPT + threadIdx.x; pb < p1; pb += step) {
+        float xv[NPT][DM];
 #pragma unroll
-        for (int j = 0; j < DM; ++j) xv[j] = j < d ? x[p * d + j] : 0.f;
-        float bd = __int_as_float(0x7f800000);
-        int bi = 0;
+        for (int q = 0; q < NPT; ++q) {
+            const int64_t p = pb + (int64_t)q * blockDim.x;
+#pragma unroll
+            for (int j = 0; j < DM; ++j) xv[q][j] = (j < d && p < p1) ? x[p * d + j] : 0.f;
+        }
+        float bd[NPT];
+        int bi[NPT];
+#pragma unroll
+        for (int q = 0; q < NPT; ++q) { bd[q] = __int_as_float(0x7f800000); bi[q] = 0; }
         for (int c = 0; c < kc; ++c) {
-            float a = 0.f;
+            float a[NPT];
+#pragma unroll
+            for (int q = 0; q < NPT; ++q) a[q] = 0.f;
+#pragma unroll
+            for (int j4 = 0; j4 < DM / 4; ++j4)
+                if (4 * j4 < d) {
+                    const float4 cv = s_c4[c * (dp >> 2) + j4];
+                    const float ce[4] = {cv.x, cv.y, cv.z, cv.w};
+#pragma unroll
+                    for (int e = 0; e < 4; ++e)
+                        if (4 * j4 + e < d) {
+#pragma unroll
+                            for (int q = 0; q < NPT; ++q) {
+                                const float df = __fsub_rn(xv[q][4 * j4 + e], ce[e]);
+                                a[q] = __fmaf_rn(df, df, a[q]);
+                            }
+                        }
+                }
+#pragma unroll
+            for (int q = 0; q < NPT; ++q)
+                if (a[q] < bd[q]) { bd[q] = a[q]; bi[q] = c; }
+        }
+#pragma unroll
+        for (int q = 0; q < NPT; ++q) {
+            const int64_t p = pb + (int64_t)q * blockDim.x;
+            if (p >= p1) continue;
+            member[p] = bi[q];
+            atomicAdd(s_cnt + bi[q], 1ull);
 #pragma unroll
             for (int j = 0; j < DM; ++j)
-                if (j < d) {
-                    const float df = __fsub_rn(xv[j], s_c[c * d + j]);
-                    a = __fmaf_rn(df, df, a);
-                }
-            if (a < bd) { bd = a; bi = c; }
+                if (j < d) superacc_add(acc + ((size_t)bi[q] * d + j) * kSuperW, xv[q][j], err);
         }
-        member[p] = bi;
-        atomicAdd(s_cnt + bi, 1ull);
-#pragma unroll
-        for (int j = 0; j < DM; ++j)
-            if (j < d) superacc_add(acc + ((size_t)bi * d + j) * kSuperW, xv[j], err);
     }
     __syncthreads();
     if constexpr (SHARED_ACC)
@@ -560,23 +591,24 @@ update_exact_zero(int64_t* __restrict__ sacc, int64_t q0, int64_t q1, Track ts) 
 template <int DM>
 cudaError_t launch_assign_exact(const float* x, const float* cen, int32_t* member, int64_t* sacc, int64_t* counts,
                                 int64_t p0, int64_t p1, int d, int kc, int* err, cudaStream_t s, int sms) {
-    const size_t base = (size_t)kc * 8 + (size_t)kc * d * 4;
+    constexpr int NPT = DM <= 16 ? 4 : DM <= 32 ? 2 : 1;
+    const size_t base = (size_t)kc * ((d + 3) & ~3) * 4 + (size_t)kc * 8;
     const size_t shared_acc = base + (size_t)kc * d * kSuperW * 8;
     const bool sh = shared_acc <= 160 * 1024;
     const size_t smem = sh ? shared_acc : base;
-    cudaError_t e = sh ? kernel_prep(assign_exact_k<DM, true>, kThreads, smem)
-                       : kernel_prep(assign_exact_k<DM, false>, kThreads, smem);
+    const void* fn = sh ? (const void*)assign_exact_k<DM, NPT, true> : (const void*)assign_exact_k<DM, NPT, false>;
+    cudaError_t e = sh ? kernel_prep(assign_exact_k<DM, NPT, true>, kThreads, smem)
+                       : kernel_prep(assign_exact_k<DM, NPT, false>, kThreads, smem);
     if (e != cudaSuccess) return e;
     int per_sm = 1;
-    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, sh ? (const void*)assign_exact_k<DM, true>
-                                                              : (const void*)assign_exact_k<DM, false>, kThreads, smem);
+    cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, fn, kThreads, smem);
     if (per_sm < 1) per_sm = 1;
-    int64_t blocks = (p1 - p0 + kThreads - 1) / kThreads;
+    int64_t blocks = (p1 - p0 + kThreads * NPT - 1) / (kThreads * NPT);
     if (blocks > (int64_t)sms * per_sm) blocks = (int64_t)sms * per_sm;
     if (sh)
-        assign_exact_k<DM, true><<<(unsigned)blocks, kThreads, smem, s>>>(x, cen, member, sacc, counts, p0, p1, d, kc, err);
+        assign_exact_k<DM, NPT, true><<<(unsigned)blocks, kThreads, smem, s>>>(x, cen, member, sacc, counts, p0, p1, d, kc, err);
     else
-        assign_exact_k<DM, false><<<(unsigned)blocks, kThreads, smem, s>>>(x, cen, member, sacc, counts, p0, p1, d, kc, err);
+        assign_exact_k<DM, NPT, false><<<(unsigned)blocks, kThreads, smem, s>>>(x, cen, member, sacc, counts, p0, p1, d, kc, err);
     return cudaGetLastError();
 }
 
