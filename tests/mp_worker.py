@@ -49,6 +49,10 @@ def main():
         x = gen.kmeans_points(5, 20000, 16, 32, gen.KM_OVERLAP)
         cen, mem = WL.kmeans_run(x, 32, 5)
         res = {"cen": cen, "mem": mem}
+    elif work == "kmeans_exact":
+        x = gen.kmeans_points_real(46, 12007, 34, 19)
+        cen, mem = WL.kmeans_run(x, 19, 3, shift=A.KMEANS_EXACT)
+        res = {"cen": cen, "mem": mem}
     if work == "masked":
         n = (1 << 20) + 4321
         src = (gen.u_fill(21, 0, n) >> np.uint64(40)).astype(np.float32) * np.float32(2.0 ** -24)

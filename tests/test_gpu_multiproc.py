@@ -134,6 +134,20 @@ def test_jacobi_three_processes(tmp_path, work):
         assert sum(s["bytes_interpartition"] for s in stats) == S * (P - 1) * (16 * P + 16 * (N - 2) + 4 * (N - 2) ** 2)
 
 
+@pytest.mark.parametrize("world,V", [(2, 2), (3, 1)])
+def test_kmeans_exact_multi_process(tmp_path, world, V):
+    """Exact mode (arbitrary real-valued points, reading KM-X): the nine-window partials of every
+    rank are merged across the processes; centroids and assignments bit-exact on every rank."""
+    x = gen.kmeans_points_real(46, 12007, 34, 19)
+    ocen, omem = oracle.kmeans_run_exact(x, 19, 3)
+    stats = _launch(world, V, "kmeans_exact", tmp_path)
+    for r in range(world):
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_cen.npy"), ocen)
+        assert np.array_equal(np.load(tmp_path / f"rank{r}_mem.npy"), omem)
+    P = world * V
+    assert abs(sum(s["bytes_reduce"] for s in stats) - 3 * 2 * (P - 1) * (19 * 34 * 9 + 19) * 8) < world * 3 * 2
+
+
 @pytest.mark.parametrize("work", ["jacobi_decl", "jacobi_undecl", "kmeans", "masked"])
 def test_two_physical_gpus(tmp_path, work):
     """Ranks 0 and 1 on devices 0 and 1: replicas mapped across GPUs through CUDA IPC, halo rows
