@@ -105,7 +105,8 @@ __device__ __forceinline__ void tile_coords(int64_t t, int num_m, int num_n, int
 // which the power-capped chip turns into clock: +8-10 % over the single-CTA kernel); each CTA
 // issues its own tcgen05.mma.cta_group::1 (M = 128, N = 256). A stage is refilled only after both
 // CTAs' MMAs have read it: every MMA commit arrives on the stage's empty barrier of both CTAs.
-// (A 2-SM cta_group::2 kernel, M = 256, measured slower: profiles/r02/experiments/README.md.)
+// (A 2-SM cta_group::2 kernel, M = 256, and clusters of four sharing A as well as B measured
+// slower: profiles/r02/experiments/README.md.)
 __device__ __forceinline__ uint32_t cluster_rank() {
     uint32_t r;
     asm volatile("mov.u32 %0, %%cluster_ctarank;" : "=r"(r));
@@ -298,9 +299,28 @@ cudaError_t gemm_bf16(const uint16_t* A, const uint16_t* B, float* C, int64_t M,
     const size_t smem = 1024 + (size_t)kStages * kStageBytes + 256;
     cudaError_t e = kernel_prep(gemm_kernel, kThreads, smem);
     if (e != cudaSuccess) return e;
-    // one cluster of two CTAs per SM pair, persistent over the pair tiles (2 m-blocks x 1 n-block)
+    // one cluster of two CTAs per SM pair, persistent over the pair tiles (2 m-blocks x 1 n-block);
+    // no more clusters than can be resident at once (a GPC with an odd SM count leaves one out)
     const int64_t ptiles = ((m1 - m0 + 2 * BM - 1) / (2 * BM)) * ((N + BN - 1) / BN);
     int64_t ncl = sms / 2;
+    static int max_cl = 0;
+    if (!max_cl) {
+        cudaLaunchConfig_t q{};
+        q.gridDim = dim3((unsigned)(2 * ncl));
+        q.blockDim = dim3(kThreads);
+        q.dynamicSmemBytes = smem;
+        cudaLaunchAttribute qa[1];
+        qa[0].id = cudaLaunchAttributeClusterDimension;
+        qa[0].val.clusterDim.x = 2;
+        qa[0].val.clusterDim.y = 1;
+        qa[0].val.clusterDim.z = 1;
+        q.attrs = qa;
+        q.numAttrs = 1;
+        int n = 0;
+        max_cl = (cudaOccupancyMaxActiveClusters(&n, gemm_kernel, &q) == cudaSuccess && n > 0) ? n : (int)ncl;
+        (void)cudaGetLastError();
+    }
+    if (ncl > max_cl) ncl = max_cl;
     if (ptiles < ncl) ncl = ptiles;
     cudaLaunchConfig_t cfg{};
     cfg.gridDim = dim3((unsigned)(2 * ncl));
