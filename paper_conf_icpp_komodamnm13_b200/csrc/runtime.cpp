@@ -24,6 +24,8 @@
 #include <unistd.h>
 
 #include <algorithm>
+#include <map>
+#include <unordered_map>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -138,6 +140,11 @@ struct State {
     int64_t miss_cap = 0;
     int64_t* d_miss = nullptr;       // [V] per-loop counters, [V] unused, [64] window bounds, total
     int64_t* d_miss_total = nullptr;
+    // device block cache (one-process runs): blocks freed by region_destroy / hull growth are kept
+    // by their allocated size and handed to the next allocation of that size (a region re-created
+    // every step, as in the e2e leg, then costs no cudaMalloc / cudaFree and no device-wide sync)
+    std::unordered_map<void*, size_t> blk;  // live dmalloc blocks -> allocated bytes
+    std::multimap<size_t, void*> cache;     // freed blocks by size
     std::vector<Prof> prof;
     std::vector<cudaEvent_t> ev_free;
     // deferred accounting of undeclared loops whose sizes the host does not need to launch the
@@ -266,21 +273,59 @@ IntervalSet window(const accmg_access& d, int64_t a, int64_t b, int64_t extent) 
     return IntervalSet(lo, hi);
 }
 
+// allocation granularity of the block cache: 2 MiB above 1 MiB (cudaMalloc's own page), else 512 B
+size_t blk_round(size_t b) {
+    return b >= ((size_t)1 << 20) ? (b + ((size_t)2 << 20) - 1) & ~(((size_t)2 << 20) - 1) : (b + 511) & ~(size_t)511;
+}
+
+void cache_release() {
+    for (auto& kv : S.cache) cudaFree(kv.second);
+    S.cache.clear();
+}
+
 int dmalloc(void** p, size_t bytes, bool system) {
     if (bytes == 0) bytes = 16;
-    cudaError_t e = cudaMalloc(p, bytes);
-    if (e != cudaSuccess) {
-        cudaGetLastError();
-        return fail(ACCMG_ENOMEM, std::string("cudaMalloc(") + std::to_string(bytes) + "): " + cudaGetErrorString(e),
-                    false);
+    const size_t rb = blk_round(bytes);
+    void* q = nullptr;
+    if (S.W == 1) {
+        auto it = S.cache.find(rb);
+        if (it != S.cache.end()) {
+            q = it->second;
+            S.cache.erase(it);
+        }
     }
+    if (!q) {
+        cudaError_t e = cudaMalloc(&q, rb);
+        if (e == cudaErrorMemoryAllocation && !S.cache.empty()) {  // give the cached blocks back, retry
+            cudaGetLastError();
+            cache_release();
+            e = cudaMalloc(&q, rb);
+        }
+        if (e != cudaSuccess) {
+            cudaGetLastError();
+            return fail(ACCMG_ENOMEM, std::string("cudaMalloc(") + std::to_string(bytes) + "): " + cudaGetErrorString(e),
+                        false);
+        }
+    }
+    S.blk[q] = rb;
+    *p = q;
     (system ? S.st.device_bytes_system : S.st.device_bytes_user) += (int64_t)bytes;
     return 0;
 }
 
 void dfree(void* p, size_t bytes, bool system) {
     if (!p) return;
-    cudaFree(p);
+    auto it = S.blk.find(p);
+    const size_t rb = it != S.blk.end() ? it->second : 0;
+    if (it != S.blk.end()) S.blk.erase(it);
+    if (S.W == 1 && rb) {
+        // the block's last users are on the library stream; the next owner may start with a copy on
+        // another stream, so drain it (cudaFree would have synchronised the whole device)
+        cudaStreamSynchronize(S.stream);
+        S.cache.emplace(rb, p);
+    } else {
+        cudaFree(p);
+    }
     (system ? S.st.device_bytes_system : S.st.device_bytes_user) -= (int64_t)bytes;
 }
 
@@ -1334,6 +1379,7 @@ int accmg_finalize(void) {
             for (int q = 0; q < 2; ++q) dfree(D.alloc[q], (D.hi - D.lo) * 4, true);
         for (auto p : S.miss_recs) dfree(p, 0, true);
         dfree(S.recv, 0, true);
+        cache_release();
         if (S.h_pin) cudaFreeHost(S.h_pin);
         if (S.h_acct) cudaFreeHost(S.h_acct);
         for (auto& p : S.prof) { cudaEventDestroy(p.a); cudaEventDestroy(p.b); }
