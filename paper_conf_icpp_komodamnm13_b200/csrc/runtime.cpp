@@ -38,6 +38,8 @@
 #include "nccl_dl.h"
 #include "vmm.h"
 
+#include <nvtx3/nvToolsExt.h>  // header-only NVTX v3: ranges cost a pointer test unless a tool is attached
+
 using accmg::IntervalSet;
 using accmg::Ival;
 namespace k = accmg::k;
@@ -340,10 +342,14 @@ cudaEvent_t ev_get() {
     return e;
 }
 
+// A loop phase: an NVTX range on the host (nsys / ncu timelines) and, with profiling on, a pair of
+// CUDA events on the library stream (the per-phase times of accmg_get_stats).
 struct ProfScope {
     int kind;
     cudaEvent_t a = nullptr;
     explicit ProfScope(int kd) : kind(kd) {
+        static const char* const kNames[3] = {"accmg body", "accmg compaction", "accmg exchange"};
+        nvtxRangePushA(kNames[kd < 0 || kd > 2 ? 2 : kd]);
         if (S.cfg.profile && !S.dry) {
             a = ev_get();
             cudaEventRecord(a, S.stream);
@@ -355,7 +361,14 @@ struct ProfScope {
             cudaEventRecord(b, S.stream);
             S.prof.push_back({a, b, kind});
         }
+        nvtxRangePop();
     }
+};
+
+// Host-side NVTX range for the ABI calls (loop launch, region create / destroy, sync to host).
+struct NvtxScope {
+    explicit NvtxScope(const char* n) { nvtxRangePushA(n); }
+    ~NvtxScope() { nvtxRangePop(); }
 };
 
 // Bytes of one partition's packet of undeclared writes (runs, elements, dirty chunks), delivered to
@@ -1393,6 +1406,7 @@ int accmg_finalize(void) {
 
 int accmg_region_create(void* host_array, size_t elem_size, int64_t extent, accmg_region* out) {
     GUARD();
+    NvtxScope nv("accmg_region_create");
     if (!host_array || !out || extent < 1) return fail(ACCMG_EINVAL, "region_create: null pointer or extent < 1", false);
     if (elem_size != 1 && elem_size != 2 && elem_size != 4 && elem_size != 8)
         return fail(ACCMG_EINVAL, "region_create: elem_size must be 1, 2, 4 or 8", false);
@@ -1418,6 +1432,7 @@ int accmg_region_create(void* host_array, size_t elem_size, int64_t extent, accm
 
 int accmg_region_destroy(accmg_region r) {
     GUARD();
+    NvtxScope nv("accmg_region_destroy");
     auto it = std::find(S.regions.begin(), S.regions.end(), r);
     if (it == S.regions.end()) return fail(ACCMG_EINVAL, "region_destroy: unknown region", false);
     S.regions.erase(it);
@@ -1495,6 +1510,7 @@ int plan_pushes(int body_id, const accmg_access* descs, const void* args,
 int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_access* descs, int n_descs,
                       const void* args, size_t args_bytes) {
     GUARD();
+    NvtxScope nv("accmg_loop_launch");
     if (!bounds || !descs || !args) return fail(ACCMG_EINVAL, "loop_launch: null argument", false);
     if (n_descs < 1 || n_descs > 16) return fail(ACCMG_EINVAL, "loop_launch: n_descs must be 1..16", false);
     BodySpec spec;
@@ -1685,6 +1701,7 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
 }
 
 static int sync_host_impl(accmg_region r, bool owned) {
+    NvtxScope nv(owned ? "accmg_sync_to_host_owned" : "accmg_sync_to_host");
     GUARD();
     if (std::find(S.regions.begin(), S.regions.end(), r) == S.regions.end())
         return fail(ACCMG_EINVAL, "sync_to_host: unknown region", false);
