@@ -631,6 +631,15 @@ cudaError_t kmeans_assign(const float* x, const float* cen, int32_t* member, int
     if (p1 <= p0) return cudaSuccess;
     const int sms = sm_count();
     if (shift < 0) {  // exact mode (arbitrary finite points; sums = k * d * 9 windows)
+        if (kmeans_tc_supported(x, d, kc)) {  // d = 16, k <= 256: the tensor-core filter serves it too
+            cudaError_t e = kmeans_assign_tc(x, cen, member, sums, counts, p0, p1, kc, shift, err_flag, s, sms);
+            if (e == cudaSuccess) {
+                if (launches) *launches += 1;
+                return cudaSuccess;
+            }
+            if (e != cudaErrorNotSupported) return e;
+            (void)cudaGetLastError();
+        }
         if (d > 64 || (int64_t)kc * d > 16384) return cudaErrorNotSupported;
         cudaError_t e = d <= 16   ? launch_assign_exact<16>(x, cen, member, sums, counts, p0, p1, d, kc, err_flag, s, sms)
                         : d <= 32 ? launch_assign_exact<32>(x, cen, member, sums, counts, p0, p1, d, kc, err_flag, s, sms)

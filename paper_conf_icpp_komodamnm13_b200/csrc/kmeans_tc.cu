@@ -332,6 +332,26 @@ __device__ unsigned long long g_km_trace[64][32];
 
 constexpr int kProdWarp = 0, kMmaWarp = 15, kMmaWarp1 = 1;
 
+// exact mode: v added exactly into two of the nine 32-bit-aligned int64 windows of its sum
+// (weight of window w: 2^(32 w - 149)); the same representation as kmeans.cu's exact kernels
+// (the converter has rejected non-finite points)
+__device__ __forceinline__ void superacc_add_tc(unsigned long long* acc, float v) {
+    const uint32_t b = __float_as_uint(v);
+    const uint32_t ex = (b >> 23) & 255u;
+    uint32_t m = b & 0x7FFFFFu;
+    if (ex) m |= 0x800000u;
+    if (!m || ex == 255u) return;
+    const int o = ex ? (int)ex - 1 : 0;
+    const uint64_t t = (uint64_t)m << (o & 31);
+    unsigned long long lo = t & 0xFFFFFFFFull, hi = t >> 32;
+    if (b >> 31) {
+        lo = 0ull - lo;
+        hi = 0ull - hi;
+    }
+    if (lo) atomicAdd(acc + (o >> 5), lo);
+    if (hi) atomicAdd(acc + (o >> 5) + 1, hi);
+}
+
 __device__ __forceinline__ void named_bar(uint32_t id, uint32_t n) {
     // non-aligned form: a warp may arrive diverged (after data-dependent re-check loops)
     __syncwarp();
@@ -343,6 +363,12 @@ __device__ __forceinline__ void named_bar(uint32_t id, uint32_t n) {
 // tile for the 128 KiB of distances. The distance accumulators form a ring of three 128-column
 // buffers (half h of tile i in buffer (nq i + h) mod 3), so the MMAs of the next tile's first half
 // run while the epilogue still reads this tile's two halves.
+// EXACT (shift = ACCMG_KMEANS_EXACT, reading KM-X): any finite points. The assignment is the same
+// filter + exact re-check; a point with |x| > 2^60 (or centroids beyond 2^60, where x.c could
+// overflow the fp32 accumulation) skips the filter and re-checks every centroid. The sums go to
+// nine 32-bit-aligned int64 windows per (cluster, dim) through the epilogue's global-atomic path
+// (every point takes it: no fixed-point words for the reduction MMA).
+template <bool EXACT>
 __global__ void __launch_bounds__(kThreadsTC, 1)
 assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg, const float* __restrict__ cen,
           int32_t* __restrict__ member,
@@ -551,7 +577,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
             tmem_st8(tqc + kColA1, ones);
             tmem_wait_st();
         }
-        const float scale = (float)(1 << shift);
+        const float scale = EXACT ? 1.f : (float)(1 << shift);
         const float Cinf = __uint_as_float(misc[1]);
         const float C2 = __uint_as_float(misc[2]);
         int bad = 0;
@@ -603,7 +629,7 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                 vm = fmaxf(vm, fabsf(v));
                 iv[j] = __float2int_rn(rv);
             }
-            const bool fits = vm < 32768.0f;
+            const bool fits = !EXACT && vm < 32768.0f;
             {
                 uint32_t hw[8];
 #pragma unroll
@@ -614,7 +640,14 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                 sts_v4(row + ((0u ^ sw) << 4), make_uint4(hw[0], hw[1], hw[2], hw[3]));
                 sts_v4(row + ((1u ^ sw) << 4), make_uint4(hw[4], hw[5], hw[6], hw[7]));
             }
-            bad |= (fr != 0.f) | !(vm < 2147483648.0f);
+            if constexpr (EXACT) {
+                bool nf = false;
+#pragma unroll
+                for (int j = 0; j < 16; ++j) nf |= !(fabsf(xv[j]) <= 3.40282347e38f);  // inf or NaN
+                bad |= nf;
+            } else {
+                bad |= (fr != 0.f) | !(vm < 2147483648.0f);
+            }
             {  // the filter bound's per-point terms, for the epilogue (header: E, Dhat)
                 float L1 = 0.f, Q = 0.f;
 #pragma unroll
@@ -622,8 +655,10 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                 const float E = (0x1p-11f * (L1 * Cinf + C2)) * 1.001f + 0x1p-100f;
                 const float Qa = Q * (1.f + 0x1p-17f) + 2.f * E;
                 // (the sign of E carries the point's "does not fit" flag; E > 0)
+                // exact mode: E = -inf marks a point whose distances the filter cannot bound
+                const bool unsafe = EXACT && !(vm <= 0x1p60f && Cinf <= 0x1p60f);
                 asm volatile("st.shared.v2.f32 [%0], {%1, %2};" ::"r"(sbase + OFF_EQ + (bs * TM + r) * 8),
-                             "f"(fits ? E : -E), "f"(Qa)
+                             "f"(unsafe ? -__int_as_float(0x7f800000) : (fits ? E : -E)), "f"(Qa)
                              : "memory");
             }
             fence_async_smem();  // the B operand (shared memory) for the reduction MMAs
@@ -744,7 +779,8 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                 mB0 = __funnelshift_l(__float_as_uint(d1), mB0, 1);
                 mB1 = __funnelshift_l(__float_as_uint(d3), mB1, 1);
             }
-            const uint32_t mA = ((mA0 << 8) | mA1) & 0xFFFFu, mB = ((mB0 << 8) | mB1) & 0xFFFFu;
+            uint32_t mA = ((mA0 << 8) | mA1) & 0xFFFFu, mB = ((mB0 << 8) | mB1) & 0xFFFFu;
+            if (EXACT && E == -__int_as_float(0x7f800000)) mA = mB = 0xFFFFu;  // re-check every centroid
             KTR(KTR_EPI, 16);
             const bool unique = __popc(mA) == 1 && __popc(mB) == 1;
             int bi = unique ? 16 * (15 - (31 - __clz(mB))) + (15 - (31 - __clz(mA))) : 0;
@@ -808,7 +844,6 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                 member[p] = bi;
                 atomicAdd(&s_cnt[bi], 1);
                 if (E < 0.f) {
-                    const float scale = (float)(1 << shift);
                     const float4* xp = reinterpret_cast<const float4*>(xg + p * 16);
 #pragma unroll
                     for (int j = 0; j < 4; ++j) {
@@ -816,9 +851,15 @@ assign_tc(const __grid_constant__ CUtensorMap xmap, const float* __restrict__ xg
                         const float e4[4] = {v.x, v.y, v.z, v.w};
 #pragma unroll
                         for (int e = 0; e < 4; ++e) {
-                            const long long iv = (long long)__float2int_rn(e4[e] * scale);
-                            if (iv) atomicAdd(reinterpret_cast<unsigned long long*>(sums) + bi * 16 + 4 * j + e,
-                                              (unsigned long long)iv);
+                            if constexpr (EXACT) {
+                                superacc_add_tc(reinterpret_cast<unsigned long long*>(sums) + (bi * 16 + 4 * j + e) * 9,
+                                                e4[e]);
+                            } else {
+                                const float scale = (float)(1 << shift);
+                                const long long iv = (long long)__float2int_rn(e4[e] * scale);
+                                if (iv) atomicAdd(reinterpret_cast<unsigned long long*>(sums) + bi * 16 + 4 * j + e,
+                                                  (unsigned long long)iv);
+                            }
                         }
                     }
                 }
@@ -909,7 +950,8 @@ cudaError_t kmeans_assign_tc(const float* x, const float* cen, int32_t* member, 
     if (p1 <= p0) return cudaSuccess;
     if (p1 - p0 > (int64_t)INT32_MAX - TM) return cudaErrorNotSupported;  // TMA row coordinates are int32
     const int npad = ((kc + 31) / 32) * 32;
-    cudaError_t e = kernel_prep(assign_tc, kThreadsTC, kSmemTC);
+    const bool exact = shift < 0;  // ACCMG_KMEANS_EXACT
+    cudaError_t e = exact ? kernel_prep(assign_tc<true>, kThreadsTC, kSmemTC) : kernel_prep(assign_tc<false>, kThreadsTC, kSmemTC);
     if (e != cudaSuccess) return e;
     const int64_t ntiles = (p1 - p0 + TM - 1) / TM;
     // s32 reduction accumulators: byte sums <= 255 per point, so at most 2^23 points (65536 tiles)
@@ -928,7 +970,11 @@ cudaError_t kmeans_assign_tc(const float* x, const float* cen, int32_t* member, 
                           box, es, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B,
                           CU_TENSOR_MAP_L2_PROMOTION_L2_128B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE))
         return cudaErrorNotSupported;
-    assign_tc<<<(unsigned)blocks, kThreadsTC, kSmemTC, s>>>(xmap, x, cen, member, sums, counts, p0, p1, kc, npad, shift,
+    if (exact)
+        assign_tc<true><<<(unsigned)blocks, kThreadsTC, kSmemTC, s>>>(xmap, x, cen, member, sums, counts, p0, p1, kc, npad,
+                                                                     shift, err_flag);
+    else
+        assign_tc<false><<<(unsigned)blocks, kThreadsTC, kSmemTC, s>>>(xmap, x, cen, member, sums, counts, p0, p1, kc, npad, shift,
                                                             err_flag);
     return cudaGetLastError();
 }

@@ -81,3 +81,30 @@ def test_non_finite_point_is_reported():
     with pytest.raises(Amod.AccmgError) as ei:
         _run(x, 6, 1, 1)
     assert ei.value.code == Amod.EDATA
+
+
+def test_tensor_core_path_extreme_points():
+    """d = 16, k <= 256 takes the tensor-core filter in exact mode too: points beyond 2^60 (whose
+    x.c could overflow the fp32 accumulation) re-check every centroid, the rest are filtered;
+    subnormals, zeros and cancelling 2^90 values in the sums."""
+    rng = np.random.default_rng(47)
+    n, d, k = 40000, 16, 96
+    x = (rng.standard_normal((n, d)) * 2.0 ** rng.integers(-30, 30, (n, 1))).astype(np.float32)
+    x[100:2100:2, 3] = np.float32(2.0 ** 90)
+    x[101:2101:2, 3] = np.float32(-(2.0 ** 90))
+    x[5000:5100, :] *= np.float32(2.0 ** 70)   # beyond 2^60: unfiltered points
+    x[7000:7400, 5] = np.float32(1.4e-45) * rng.integers(1, 5, 400).astype(np.float32)
+    x[rng.random((n, d)) < 0.05] = 0.0
+    ocen, omem = oracle.kmeans_run_exact(x, k, 3)
+    cen, mem = _run(x, k, 3, 2)
+    assert np.array_equal(mem, omem), f"{int((mem != omem).sum())} assignments differ"
+    assert np.array_equal(cen.view(np.uint32), ocen.view(np.uint32))
+
+
+def test_tensor_core_path_centroids_beyond_2_60():
+    """Every centroid coordinate large (> 2^60 after the first update): no point is filtered."""
+    rng = np.random.default_rng(48)
+    x = (rng.standard_normal((6000, 16)) * np.float32(2.0 ** 80)).astype(np.float32)
+    ocen, omem = oracle.kmeans_run_exact(x, 40, 2)
+    cen, mem = _run(x, 40, 2, 1)
+    assert np.array_equal(mem, omem) and np.array_equal(cen, ocen)
