@@ -1569,6 +1569,12 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
     std::vector<Xfer> xs;
     for (int i = 0; i < n_descs; ++i) plan_pulls(descs[i].region, need[i], xs);
     TRY(run_xfers(xs));
+    // P2P: peers write into this process's replicas during the loop (the dirty-element pushes of
+    // undeclared writes, the writing body's predicted halo pushes), so the loader's copies into
+    // them (host copy-in, pulls) must have landed before any peer's body starts; without this a
+    // fast peer's push of loop 0 could be overwritten by a slow rank's copy-in of the same rows.
+    // The plan covers every partition, so every rank takes this branch (barrier epochs in step).
+    if (S.p2p && !xs.empty()) TRY(dev_barrier());
     for (int i = 0; i < n_descs; ++i)
         for (int g = 0; g < S.P; ++g) descs[i].region->valid[g].add(need[i][g]);
     // predicted-halo push (halo_mode AUTO, L125: iterative codes reuse their access patterns)

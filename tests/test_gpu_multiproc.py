@@ -117,6 +117,25 @@ def test_masked_writes_multi_process(tmp_path, world, V):
         assert np.array_equal(np.load(tmp_path / f"rank{r}_out.npy"), exp)
 
 
+def test_undeclared_first_loop_copy_in_before_peer_pushes(tmp_path):
+    """Regression: in the first undeclared loop every rank copies the host array into its replica
+    while its peers, after their bodies, push their dirty rows into it. Without a barrier between
+    the loader's copies and the bodies, a slow rank's copy-in could overwrite a fast peer's pushed
+    rows (it did in ~1 of 8 three-rank runs on one GPU: wrong values around the partition
+    boundaries, identical on every rank). Eight repetitions, each bit-exact."""
+    N, S = 300, 6
+    A0 = gen.jacobi_field(5, N)
+    oA, oB = A0.copy(), A0.copy()
+    oracle.jacobi_run(oA, oB, S)
+    for rep in range(8):
+        d = tmp_path / f"rep{rep}"
+        d.mkdir()
+        _launch(3, 1, "jacobi_undecl", d)
+        for r in range(3):
+            assert np.array_equal(np.load(d / f"rank{r}_A.npy"), oA), (rep, r)
+            assert np.array_equal(np.load(d / f"rank{r}_B.npy"), oB), (rep, r)
+
+
 @pytest.mark.parametrize("work", ["jacobi_decl", "jacobi_undecl"])
 def test_jacobi_three_processes(tmp_path, work):
     """Three ranks (partitions 0-2 in three CUDA contexts): the middle rank pushes halos / dirty
