@@ -264,7 +264,8 @@ int accmg_unique_id(uint8_t out[128]);
    the process's stream and (world_size > 1) the NCCL communicator. ACCMG_ESTATE if initialised. */
 int accmg_init(const accmg_config* cfg);
 
-/* Frees every region and runtime buffer, destroys the stream and communicator. */
+/* Frees every region and runtime buffer (and the block cache), destroys the stream and
+   communicator. */
 int accmg_finalize(void);
 
 /* Data-region entry (copyin semantics, L119 §IV.C). Registers `extent` elements of `elem_size`
@@ -277,7 +278,10 @@ int accmg_finalize(void);
    (L119, L125). elem_size in {1,2,4,8}. */
 int accmg_region_create(void* host_array, size_t elem_size, int64_t extent, accmg_region* out);
 
-/* Data-region exit without copy-out (OpenACC `delete`); frees the region's device memory. */
+/* Data-region exit without copy-out (OpenACC `delete`); frees the region's device memory. In a
+   one-process run (world_size 1) the freed blocks stay in the runtime's block cache and serve
+   later allocations of the same size (no cudaMalloc / cudaFree per re-created region); the cache
+   is emptied when an allocation fails (then retried) and at accmg_finalize. */
 int accmg_region_destroy(accmg_region r);
 
 /* One offloaded parallel loop (L64 §III.A): partition dim 0 of `bounds` into P chunks
