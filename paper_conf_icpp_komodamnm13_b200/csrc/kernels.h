@@ -101,7 +101,7 @@ cudaError_t scatter_body(const float* src, const int32_t* idx, float* dst, int64
 // no window holds is dropped and sets *bad.
 cudaError_t apply_misses(const uint64_t* recs, const int64_t* count, int64_t cap, const PtrList& dsts,
                          const int64_t* bounds_dev, const int64_t* his_dev, int nb, int64_t* total, int* bad,
-                         cudaStream_t s, int64_t* launches);
+                         int64_t extent, cudaStream_t s, int64_t* launches);
 
 // ---- coherence: compaction of dirty runs, scatter into peer replicas -------------------------
 constexpr int kTileWords = 2048;   // bitmap words per compaction tile (65536 elements)

@@ -1651,7 +1651,7 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
             CUDA_TRY(cudaMemcpyAsync(S.d_miss + 2 * 64, wb, sizeof(int64_t) * 128, cudaMemcpyHostToDevice, S.stream));
             for (int li = 0; li < S.V; ++li)
                 CUDA_TRY(k::apply_misses(S.miss_recs[li], S.d_miss + li, S.miss_cap, dl, S.d_miss + 2 * 64,
-                                         S.d_miss + 3 * 64, nb, S.d_miss_total, S.d_flag + 2, S.stream,
+                                         S.d_miss + 3 * 64, nb, S.d_miss_total, S.d_flag + 2, r->extent, S.stream,
                                          &S.st.kernel_launches));
         }
         if (!tracked_regs.empty()) TRY(propagate_dirty(tracked_regs));

@@ -74,3 +74,30 @@ def test_index_outside_every_window_is_edata(bad, P):
     ok = np.arange(n) != 777
     exp[idx[ok]] = src[ok]
     assert np.array_equal(dst, exp)
+
+
+@pytest.mark.parametrize("P", [1, 2])
+def test_full_size_sliced_passes_bitexact(P):
+    """f1 at full size (2^26 + 3 elements: a 256 MB window at P = 1, written in L2-sized slices by
+    several passes of the body, and 128 MB-window owners of the P = 2 misses): bit-exact, every
+    element written once, miss counts as the oracle's."""
+    n = (1 << 26) + 3
+    src = (gen.u_fill(31, 0, n) >> np.uint64(40)).astype(np.float32) * np.float32(2.0 ** -24)
+    idx = gen.permutation(32, n)
+    exp = np.zeros(n, np.float32)
+    miss = oracle.scatter(src, idx, exp, P=P)
+    got, st = _run(src, idx, P)
+    assert np.array_equal(got, exp)
+    assert st["write_misses"] == int(miss.sum())
+
+
+def test_full_size_index_outside_every_window_is_edata():
+    """The window check of the sliced passes: a bad index among 2^26 is still reported."""
+    from paper_conf_icpp_komodamnm13_b200 import accmg as A
+    n = 1 << 26
+    src = np.ones(n, np.float32)
+    idx = gen.permutation(33, n)
+    idx[12345678] = -5
+    with pytest.raises(A.AccmgError) as ei:
+        _run(src, idx, 1)
+    assert ei.value.code == A.EDATA
