@@ -1615,9 +1615,9 @@ int accmg_loop_launch(const accmg_bounds* bounds, int body_id, const accmg_acces
             for (int g = 0; g < S.P; ++g) cap = std::max(cap, cb[g] - ca[g]);
             if (cap > S.miss_cap) {
                 CUDA_TRY(cudaStreamSynchronize(S.stream));
-                for (auto p : S.miss_recs) dfree(p, S.miss_cap * 16, true);
+                for (auto p : S.miss_recs) dfree(p, S.miss_cap * 8, true);
                 S.miss_recs.assign(S.V, nullptr);
-                for (int li = 0; li < S.V; ++li) TRY(dmalloc((void**)&S.miss_recs[li], cap * 16, true));
+                for (int li = 0; li < S.V; ++li) TRY(dmalloc((void**)&S.miss_recs[li], cap * 8, true));  // 8-byte records
                 S.miss_cap = cap;
             }
             CUDA_TRY(cudaMemsetAsync(S.d_miss, 0, sizeof(int64_t) * S.V, S.stream));
